@@ -1,0 +1,172 @@
+/*
+ * sw.h — C-ABI of libsw: score-only Smith-Waterman/Gotoh protein database search on
+ * B200 (sm_100a), scheduled over 1..8 GPUs with the paper's PSS policy and workload
+ * adjustment (WA).
+ *
+ * Paper: Mendonca & Melo, "Biological Sequence Comparison on Hybrid Platforms with
+ * Dynamic Workload Adjustment", IPDPSW 2013 (PAPER.md; "P<n>" = line n, one PDF page).
+ *
+ *   The problem (P14 §II.B): "a set of x query sequences (q 1,q 2,...,q x ) will be
+ *   compared to a set of y database sequences (d 1,d 2,...,d y )" (x << y); the user
+ *   provides query and database (P16 §IV) and the allocation policy (P18 §IV.A); the
+ *   master "merges" the slaves' results (P16 §IV).
+ *
+ *   Every (query, database sequence) score is the Smith-Waterman local-alignment score
+ *   (P12 §II.A.1, Eq. 1, zero first row/column) with Gotoh's affine gaps (P12 §II.A.3,
+ *   "3 Dynamic Programming (DP) matrices: H, E and F"), i.e. with alpha = open + extend,
+ *   beta = extend:
+ *     E(i,j) = max(E(i,j-1) - beta, H(i,j-1) - alpha)
+ *     F(i,j) = max(F(i-1,j) - beta, H(i-1,j) - alpha)
+ *     H(i,j) = max(0, H(i-1,j-1) + S[q_i][d_j], E(i,j), F(i,j)),   score = max H.
+ *   A gap of length L costs gap_open + L*gap_extend (reading R3).
+ *
+ * Residues: ASCII letters of the NCBI protein alphabet ARNDCQEGHILKMFPSTWYVBZX*
+ * (case-insensitive); the substitution matrix is 24x24 int8 in that order with the
+ * QUERY residue as the row.  NULL matrix = BLOSUM62 (reading R1), the default gaps
+ * are open 10 / extend 2 (reading R2).
+ *
+ * Errors: every int-returning entry point returns SW_OK (0) or a negative SW_E* code;
+ * sw_last_error() then returns a thread-local message valid until the next call on
+ * that thread.  No entry point aborts the process.  There is no CPU fallback: without
+ * a usable CUDA device the search entry points return SW_ECUDA.
+ *
+ * Ownership: inputs are borrowed for the duration of a call (sw_db_create copies what
+ * it needs); outputs are caller-allocated; a sw_db owns its device memory until
+ * sw_db_destroy.  One sw_search per sw_db at a time (SW_EBUSY otherwise).
+ */
+#ifndef SW_H
+#define SW_H
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum {
+  SW_OK = 0,
+  SW_EINVAL = -1,   /* bad argument (message says which) */
+  SW_ERESIDUE = -2, /* letter outside the alphabet (message names the sequence index) */
+  SW_ENOMEM = -3,   /* host or device allocation failed */
+  SW_ECUDA = -4,    /* CUDA error or no device */
+  SW_ENET = -5,     /* multi-process control-plane error (TCP master/worker) */
+  SW_EBUSY = -6     /* a search is already running on this sw_db */
+};
+
+/* Task allocation policies (P18 §IV.A). */
+enum {
+  SW_POLICY_SS = 0, /* Self-Scheduling: Allocate(N, p_i) = 1 (P18 §IV.A.1) */
+  SW_POLICY_PSS = 1 /* Package Weighted Adaptive Self-Scheduling, Eq. 2 (P18 §IV.A.2);
+                       the paper's default ("The PSS policy was used in all the tests", P20) */
+};
+
+/* The paper's indexed sequence format (P20 §IV.B: "the total number of sequences, the
+ * size of the biggest sequence and the offset that marks the beginning of each
+ * sequence").  Sequence k is residues[offsets[k] .. offsets[k+1]). */
+typedef struct {
+  int32_t n;              /* number of sequences, >= 0 */
+  const int64_t *offsets; /* n+1 entries, offsets[0] = 0, non-decreasing (host memory) */
+  const char *residues;   /* ASCII residues (host memory), offsets[n] bytes */
+  int32_t max_len;        /* optional hint ("size of the biggest sequence"); 0 = compute */
+} sw_seqset;
+
+/* One top-k hit: score and ORIGINAL database index; {0, -1} marks an empty slot. */
+typedef struct {
+  int32_t score;
+  int32_t db_index;
+} sw_hit;
+
+typedef struct {
+  int32_t policy;            /* SW_POLICY_SS | SW_POLICY_PSS (default PSS) */
+  int32_t workload_adjust;   /* 1 = WA on (default, P20 "always activated"), 0 = off */
+  int32_t omega;             /* PSS history length (Omega, P18 §IV.A.2); default 4 (reading R10) */
+  int32_t streams_per_device;/* units in flight per GPU (default 3) */
+  int64_t target_unit_cells; /* cells per work unit; 0 = auto; INT64_MAX = one unit per
+                                query pair and kernel kind (the paper's very coarse
+                                "comparison of one query sequence to one genomic database",
+                                P16 §IV) */
+  int32_t long_threshold;    /* DB sequences longer than this go to the intra-task
+                                (warp wavefront) kernel; 0 = auto (3072), <0 = never */
+  int32_t outputs_on_device; /* 1: `scores` / `hits` are device pointers on the first
+                                device of the sw_db (inputs-resident timing mode) */
+  uint64_t straggler_mask;   /* bench/tests: worker w is throttled if bit w is set */
+  int32_t straggler_slowdown;/* throttle factor (grid capped to 1/slowdown of the SMs) */
+  /* multi-process mode (one process per GPU, torchrun): world > 1 makes every rank a
+     worker of one master, run as a thread of rank 0 and reached over TCP */
+  int32_t dist_rank;
+  int32_t dist_world;        /* 0/1 = single process (in-process master) */
+  int32_t dist_port;         /* TCP port of the master (on dist_host) */
+  const char *dist_host;     /* master address, e.g. "127.0.0.1" */
+  int32_t reserved[8];
+} sw_opts;
+
+typedef struct {
+  int64_t cells;            /* sum over (query, db) pairs of |q|*|d| (real residues; each
+                               pair once even when WA duplicated it) */
+  double seconds_device;    /* whole-box device time: max over GPUs of their last event
+                               minus the common start (host barrier, then start events) */
+  double seconds_wall;      /* host wall clock of the same span */
+  double gcups;             /* cells / seconds_device / 1e9 */
+  int64_t duplicated_cells; /* cells of WA replicas that lost the race (wasted work) */
+  int32_t n_units;          /* work units in the plan */
+  int32_t n_overflow_pairs; /* pairs re-scored by the int32 kernel after saturation */
+  int32_t n_wa_grants;      /* duplicates granted by workload adjustment */
+  int32_t n_requests;       /* master interactions (task requests) */
+  int32_t kernel_launches;  /* CUDA kernels launched by this process for the search */
+  int32_t n_devices;        /* devices (in-process) or 1 (per rank) */
+  double kernel_seconds_k1; /* summed device time of the inter-task kernel launches */
+  double kernel_seconds_k3; /* summed device time of the intra-task kernel launches */
+  int64_t cells_k1;         /* real cells computed by inter-task launches (incl. duplicates) */
+  int64_t cells_k3;         /* real cells computed by intra-task launches (incl. duplicates) */
+  double tail_seconds;      /* makespan minus the median per-worker finish time */
+  const char *unit_log_json;/* per-unit log (worker, replica, t_grant, t_start, t_end, cells,
+                               committed); owned by the sw_db, valid until its next search */
+} sw_stats;
+
+typedef struct sw_db sw_db; /* opaque: host index + packed replica on each device */
+
+/* Default options (PSS, WA on, Omega 4, auto unit size, auto long threshold). */
+void sw_opts_default(sw_opts *opts);
+
+/* Validate and encode `db`, sort by length, pack into interleaved warp groups and
+ * upload one replica to each of devices[0..n_devices) (NULL / 0 devices = device 0).
+ * The packed layout is DESIGN.md §5.  Returns SW_OK and *out, or an error. */
+int sw_db_create(const sw_seqset *db, const int *devices, int n_devices, sw_db **out);
+
+void sw_db_destroy(sw_db *db);
+
+/* Number of sequences, residues and devices of a database (for the binding). */
+int64_t sw_db_residues(const sw_db *db);
+int32_t sw_db_size(const sw_db *db);
+int32_t sw_db_devices(const sw_db *db);
+
+/* Compare every query with every database sequence.
+ *   matrix      24x24 int8, row-major, query residue = row; NULL = BLOSUM62
+ *   gap_open, gap_extend  >= 0, gap_open + 2*gap_extend <= 2^20
+ *   top_k       >= 0 hits per query under (score desc, db_index asc)
+ *   scores      [nq][ndb] int32 in the ORIGINAL orders, or NULL
+ *   hits        [nq][top_k] sw_hit, or NULL
+ *   (host pointers, or device pointers on the sw_db's first device when
+ *    opts->outputs_on_device)
+ * In multi-process mode every rank passes the same inputs; each rank's `scores` then
+ * holds the pairs of the units it committed (others = -1) and `hits` the top-k over
+ * those; the binding merges them across ranks (NCCL).
+ * Results are bit-identical for every GPU count, policy and WA setting. */
+int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t gap_open,
+              int32_t gap_extend, int32_t top_k, int32_t *scores, sw_hit *hits,
+              const sw_opts *opts, sw_stats *stats);
+
+/* Top-k of a device score matrix [nq][ndb] (entries < 0 are ignored) on the sw_db's
+ * first device, hits into device memory [nq][top_k].  Used by the binding to finish a
+ * cross-rank reduction.  */
+int sw_topk_device(sw_db *db, const int32_t *scores_dev, int32_t nq, int32_t ndb, int32_t top_k,
+                   sw_hit *hits_dev);
+
+/* Thread-local message of the last error on this thread ("" if none). */
+const char *sw_last_error(void);
+
+/* Library version string. */
+const char *sw_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

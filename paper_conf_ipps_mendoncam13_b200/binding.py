@@ -1,0 +1,315 @@
+"""Thin ctypes binding of libsw (include/sw.h, include/sw_sched.h).
+
+Argument marshalling only: every step of the search runs in libsw's kernels and host
+runtime.  There is no CPU fallback; if libsw.so cannot be loaded this module raises.
+PyTorch is used (optionally) only for device buffers when outputs stay on the GPU.
+"""
+from __future__ import annotations
+
+import ctypes
+import json
+import os
+from dataclasses import dataclass
+
+import numpy as np
+
+from . import _build
+
+_lib = None
+
+SW_OK, SW_EINVAL, SW_ERESIDUE, SW_ENOMEM, SW_ECUDA, SW_ENET, SW_EBUSY = 0, -1, -2, -3, -4, -5, -6
+SW_POLICY_SS, SW_POLICY_PSS = 0, 1
+SW_TASK_READY, SW_TASK_EXECUTING, SW_TASK_FINISHED = 0, 1, 2
+
+
+class SwError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__(f"libsw error {code}: {msg}")
+        self.code = code
+
+
+class sw_seqset(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int32), ("offsets", ctypes.POINTER(ctypes.c_int64)),
+                ("residues", ctypes.c_void_p), ("max_len", ctypes.c_int32)]
+
+
+class sw_opts(ctypes.Structure):
+    _fields_ = [("policy", ctypes.c_int32), ("workload_adjust", ctypes.c_int32),
+                ("omega", ctypes.c_int32), ("streams_per_device", ctypes.c_int32),
+                ("target_unit_cells", ctypes.c_int64), ("long_threshold", ctypes.c_int32),
+                ("outputs_on_device", ctypes.c_int32), ("straggler_mask", ctypes.c_uint64),
+                ("straggler_slowdown", ctypes.c_int32), ("dist_rank", ctypes.c_int32),
+                ("dist_world", ctypes.c_int32), ("dist_port", ctypes.c_int32),
+                ("dist_host", ctypes.c_char_p), ("reserved", ctypes.c_int32 * 8)]
+
+
+class sw_stats(ctypes.Structure):
+    _fields_ = [("cells", ctypes.c_int64), ("seconds_device", ctypes.c_double),
+                ("seconds_wall", ctypes.c_double), ("gcups", ctypes.c_double),
+                ("duplicated_cells", ctypes.c_int64), ("n_units", ctypes.c_int32),
+                ("n_overflow_pairs", ctypes.c_int32), ("n_wa_grants", ctypes.c_int32),
+                ("n_requests", ctypes.c_int32), ("kernel_launches", ctypes.c_int32),
+                ("n_devices", ctypes.c_int32), ("kernel_seconds_k1", ctypes.c_double),
+                ("kernel_seconds_k3", ctypes.c_double), ("cells_k1", ctypes.c_int64),
+                ("cells_k3", ctypes.c_int64), ("tail_seconds", ctypes.c_double),
+                ("unit_log_json", ctypes.c_char_p)]
+
+
+# every symbol include/*.h declares (tests check the library exports all of them)
+EXPORTS = ["sw_opts_default", "sw_db_create", "sw_db_destroy", "sw_db_residues", "sw_db_size",
+           "sw_db_devices", "sw_search", "sw_topk_device", "sw_last_error", "sw_version",
+           "sw_sched_create", "sw_sched_destroy", "sw_sched_report", "sw_sched_request",
+           "sw_sched_complete", "sw_sched_abandon", "sw_sched_is_finished", "sw_sched_state",
+           "sw_sched_committed_by", "sw_sched_replicas", "sw_sched_phi", "sw_sched_rate",
+           "sw_sched_counter", "sw_sched_log_json"]
+
+
+def lib():
+    """Load libsw.so (building it in-tree first if it is missing or stale)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    path = _build.LIB
+    try:
+        if _build._stale():
+            _build.build()
+    except Exception as e:  # nvcc missing etc.: only fatal if there is no library at all
+        if not os.path.exists(path):
+            raise ImportError(f"libsw.so is missing and could not be built: {e}") from e
+    if not os.path.exists(path):
+        raise ImportError(f"libsw.so not found at {path}")
+    L = ctypes.CDLL(path)
+    P = ctypes.POINTER
+    L.sw_opts_default.argtypes = [P(sw_opts)]
+    L.sw_db_create.argtypes = [P(sw_seqset), P(ctypes.c_int), ctypes.c_int, P(ctypes.c_void_p)]
+    L.sw_db_create.restype = ctypes.c_int
+    L.sw_db_destroy.argtypes = [ctypes.c_void_p]
+    L.sw_db_residues.argtypes = [ctypes.c_void_p]
+    L.sw_db_residues.restype = ctypes.c_int64
+    L.sw_db_size.argtypes = [ctypes.c_void_p]
+    L.sw_db_size.restype = ctypes.c_int32
+    L.sw_db_devices.argtypes = [ctypes.c_void_p]
+    L.sw_db_devices.restype = ctypes.c_int32
+    L.sw_search.argtypes = [P(sw_seqset), ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32,
+                            ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p,
+                            P(sw_opts), P(sw_stats)]
+    L.sw_search.restype = ctypes.c_int
+    L.sw_topk_device.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32,
+                                 ctypes.c_int32, ctypes.c_void_p]
+    L.sw_topk_device.restype = ctypes.c_int
+    L.sw_last_error.restype = ctypes.c_char_p
+    L.sw_version.restype = ctypes.c_char_p
+    L.sw_sched_create.argtypes = [ctypes.c_int32, ctypes.c_int32, P(ctypes.c_int64), ctypes.c_int32,
+                                  ctypes.c_int32, ctypes.c_int32]
+    L.sw_sched_create.restype = ctypes.c_void_p
+    L.sw_sched_destroy.argtypes = [ctypes.c_void_p]
+    L.sw_sched_report.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_double, ctypes.c_double,
+                                  ctypes.c_double]
+    L.sw_sched_request.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_double,
+                                   P(ctypes.c_int32), ctypes.c_int32]
+    L.sw_sched_request.restype = ctypes.c_int32
+    L.sw_sched_complete.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_double]
+    L.sw_sched_complete.restype = ctypes.c_int32
+    L.sw_sched_abandon.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_double]
+    for name in ("sw_sched_is_finished", "sw_sched_state", "sw_sched_committed_by",
+                 "sw_sched_replicas"):
+        getattr(L, name).argtypes = [ctypes.c_void_p, ctypes.c_int32]
+        getattr(L, name).restype = ctypes.c_int32
+    L.sw_sched_phi.argtypes = [ctypes.c_void_p, ctypes.c_int32]
+    L.sw_sched_phi.restype = ctypes.c_int32
+    L.sw_sched_rate.argtypes = [ctypes.c_void_p, ctypes.c_int32]
+    L.sw_sched_rate.restype = ctypes.c_double
+    L.sw_sched_counter.argtypes = [ctypes.c_void_p, ctypes.c_int32]
+    L.sw_sched_counter.restype = ctypes.c_int64
+    L.sw_sched_log_json.argtypes = [ctypes.c_void_p]
+    L.sw_sched_log_json.restype = ctypes.c_char_p
+    _lib = L
+    return L
+
+
+def _check(rc):
+    if rc != SW_OK:
+        raise SwError(rc, lib().sw_last_error().decode(errors="replace"))
+
+
+def _seqset(s, keep):
+    off = np.ascontiguousarray(s.offsets, dtype=np.int64)
+    res = np.ascontiguousarray(s.residues, dtype=np.uint8)
+    keep += [off, res]
+    return sw_seqset(int(s.n), off.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)),
+                     res.ctypes.data if res.size else None, 0)
+
+
+@dataclass
+class SearchResult:
+    scores: object          # [nq, ndb] int32 (numpy, or torch on device), or None
+    hit_scores: object      # [nq, k]
+    hit_index: object       # [nq, k] (-1 = empty)
+    stats: dict
+
+
+def _stats_dict(st: sw_stats) -> dict:
+    d = {k: getattr(st, k) for k, _ in sw_stats._fields_ if k != "unit_log_json"}
+    d["unit_log"] = json.loads(st.unit_log_json.decode()) if st.unit_log_json else []
+    return d
+
+
+class Database:
+    """A packed database replicated on one or more GPUs (sw_db_create)."""
+
+    def __init__(self, db, devices=None):
+        keep = []
+        ss = _seqset(db, keep)
+        h = ctypes.c_void_p()
+        if devices:
+            arr = (ctypes.c_int * len(devices))(*devices)
+            _check(lib().sw_db_create(ctypes.byref(ss), arr, len(devices), ctypes.byref(h)))
+        else:
+            _check(lib().sw_db_create(ctypes.byref(ss), None, 0, ctypes.byref(h)))
+        self._h = h
+        self.n = db.n
+        self.devices = list(devices) if devices else [0]
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib().sw_db_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    @property
+    def residues(self) -> int:
+        return int(lib().sw_db_residues(self._h))
+
+    def search(self, queries, matrix=None, gap_open=10, gap_extend=2, top_k=10, want_scores=True,
+               policy="pss", workload_adjust=True, omega=4, streams=3, target_unit_cells=0,
+               long_threshold=0, outputs_on_device=False, straggler_mask=0, straggler_slowdown=6,
+               dist=None, out_scores=None, out_hits=None) -> SearchResult:
+        """sw_search.  Host outputs are numpy arrays (pinned buffers may be passed via
+        out_scores / out_hits); with outputs_on_device the outputs are torch CUDA tensors."""
+        keep = []
+        qs = _seqset(queries, keep)
+        nq, nd = int(queries.n), int(self.n)
+        o = sw_opts()
+        lib().sw_opts_default(ctypes.byref(o))
+        o.policy = SW_POLICY_SS if policy == "ss" else SW_POLICY_PSS
+        o.workload_adjust = int(bool(workload_adjust))
+        o.omega = omega
+        o.streams_per_device = streams
+        o.target_unit_cells = target_unit_cells
+        o.long_threshold = long_threshold
+        o.outputs_on_device = int(bool(outputs_on_device))
+        o.straggler_mask = straggler_mask
+        o.straggler_slowdown = straggler_slowdown
+        if dist is not None:
+            o.dist_rank, o.dist_world, o.dist_port = dist["rank"], dist["world"], dist["port"]
+            host = dist.get("host", "127.0.0.1").encode()
+            keep.append(host)
+            o.dist_host = host
+        mat = None
+        if matrix is not None:
+            mat = np.ascontiguousarray(np.asarray(matrix, dtype=np.int8).reshape(24, 24))
+            keep.append(mat)
+        if outputs_on_device:
+            import torch
+            dev = torch.device("cuda", self.devices[0])
+            scores = out_scores if out_scores is not None else (
+                torch.empty((nq, nd), dtype=torch.int32, device=dev) if want_scores else None)
+            hits = out_hits if out_hits is not None else (
+                torch.empty((nq, max(top_k, 0), 2), dtype=torch.int32, device=dev) if top_k > 0 else None)
+            sp = scores.data_ptr() if scores is not None else None
+            hp = hits.data_ptr() if hits is not None else None
+        else:
+            scores = out_scores if out_scores is not None else (
+                np.empty((nq, nd), dtype=np.int32) if want_scores else None)
+            hits = out_hits if out_hits is not None else (
+                np.empty((nq, max(top_k, 0), 2), dtype=np.int32) if top_k > 0 else None)
+            sp = _ptr(scores)
+            hp = _ptr(hits)
+        st = sw_stats()
+        rc = lib().sw_search(ctypes.byref(qs), self._h, mat.ctypes.data if mat is not None else None,
+                             gap_open, gap_extend, top_k, sp, hp, ctypes.byref(o), ctypes.byref(st))
+        _check(rc)
+        hs = hits[..., 0] if hits is not None else None
+        hi = hits[..., 1] if hits is not None else None
+        return SearchResult(scores, hs, hi, _stats_dict(st))
+
+    def topk_device(self, scores_dev, top_k):
+        """Top-k of a torch CUDA score matrix (entries < 0 ignored) -> (scores, index)."""
+        import torch
+        nq, nd = scores_dev.shape
+        hits = torch.empty((nq, top_k, 2), dtype=torch.int32, device=scores_dev.device)
+        _check(lib().sw_topk_device(self._h, scores_dev.data_ptr(), nq, nd, top_k, hits.data_ptr()))
+        return hits[..., 0], hits[..., 1]
+
+
+def _ptr(a):
+    if a is None:
+        return None
+    if isinstance(a, np.ndarray):
+        assert a.flags["C_CONTIGUOUS"]
+        return a.ctypes.data
+    return a.data_ptr()  # torch (pinned host) tensor
+
+
+class Scheduler:
+    """The master's task table (sw_sched_*), drivable with a simulated clock."""
+
+    def __init__(self, n_workers, unit_cells, policy="pss", wa=True, omega=4):
+        cells = np.ascontiguousarray(unit_cells, dtype=np.int64)
+        self._cells = cells
+        h = lib().sw_sched_create(n_workers, len(cells),
+                                  cells.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)),
+                                  SW_POLICY_SS if policy == "ss" else SW_POLICY_PSS, int(wa), omega)
+        if not h:
+            raise SwError(SW_EINVAL, "sw_sched_create failed")
+        self._h = h
+
+    def __del__(self):
+        if getattr(self, "_h", None):
+            lib().sw_sched_destroy(self._h)
+            self._h = None
+
+    def report(self, worker, now, cells, seconds):
+        lib().sw_sched_report(self._h, worker, now, float(cells), float(seconds))
+
+    def request(self, worker, now, cap=64):
+        buf = (ctypes.c_int32 * cap)()
+        n = lib().sw_sched_request(self._h, worker, now, buf, cap)
+        if n < 0:
+            return None  # every task finished
+        return [buf[i] for i in range(n)]
+
+    def complete(self, worker, unit, now) -> bool:
+        return bool(lib().sw_sched_complete(self._h, worker, unit, now))
+
+    def abandon(self, worker, unit, now):
+        lib().sw_sched_abandon(self._h, worker, unit, now)
+
+    def is_finished(self, unit) -> bool:
+        return bool(lib().sw_sched_is_finished(self._h, unit))
+
+    def state(self, unit):
+        return lib().sw_sched_state(self._h, unit)
+
+    def committed_by(self, unit):
+        return lib().sw_sched_committed_by(self._h, unit)
+
+    def replicas(self, unit):
+        return lib().sw_sched_replicas(self._h, unit)
+
+    def phi(self, worker):
+        return lib().sw_sched_phi(self._h, worker)
+
+    def rate(self, worker):
+        return lib().sw_sched_rate(self._h, worker)
+
+    def counter(self, which):
+        return lib().sw_sched_counter(self._h, which)
+
+    def log(self):
+        return json.loads(lib().sw_sched_log_json(self._h).decode())

@@ -1,0 +1,795 @@
+// api.cpp — libsw's C-ABI (include/sw.h): database creation, the search driver
+// (master + one worker thread per GPU, PSS/WA over the task table of sched.cpp), the
+// per-device runtime (streams, profiles, border slots, abort flags), result merge and
+// top-k.  Multi-process (torchrun) mode reaches a master in rank 0 over TCP (net.cpp).
+//
+// The paper's flow (P16 §IV, Fig. 4): register slaves -> acquire sequences -> convert
+// format -> allocate tasks (policy) -> execute tasks -> send results -> merge.
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <climits>
+#include <cmath>
+#include <condition_variable>
+#include <cstring>
+#include <deque>
+#include <memory>
+#include <mutex>
+#include <numeric>
+#include <sstream>
+#include <stdexcept>
+#include <string>
+#include <thread>
+#include <vector>
+#include <cuda_runtime.h>
+#include "sw_internal.h"
+#include "net.h"
+#include "../../include/sw.h"
+#include "../../include/sw_sched.h"
+
+namespace sw {
+
+// ---------------------------------------------------------------- errors
+static thread_local std::string g_err;
+#define CK(call)                                                                      \
+  do {                                                                                \
+    cudaError_t e_ = (call);                                                          \
+    if (e_ != cudaSuccess)                                                            \
+      throw Error(SW_ECUDA, std::string(#call) + ": " + cudaGetErrorString(e_));      \
+  } while (0)
+
+template <class F>
+static int guarded(F &&f) {
+  try {
+    g_err.clear();
+    f();
+    return SW_OK;
+  } catch (const Error &e) {
+    g_err = e.what();
+    return e.code;
+  } catch (const std::bad_alloc &) {
+    g_err = "out of host memory";
+    return SW_ENOMEM;
+  } catch (const std::exception &e) {
+    g_err = e.what();
+    return SW_EINVAL;
+  }
+}
+
+static double now_s() {
+  using namespace std::chrono;
+  return duration<double>(steady_clock::now().time_since_epoch()).count();
+}
+
+// ---------------------------------------------------------------- device buffers
+template <class T>
+struct DBuf {
+  T *p = nullptr;
+  size_t n = 0;
+  int dev = -1;
+  void alloc(int d, size_t count) {
+    free();
+    dev = d;
+    n = count;
+    if (count == 0) return;
+    cudaError_t e = cudaMalloc((void **)&p, sizeof(T) * count);
+    if (e != cudaSuccess) {
+      p = nullptr;
+      throw Error(SW_ENOMEM, std::string("cudaMalloc: ") + cudaGetErrorString(e));
+    }
+  }
+  void free() {
+    if (p) { cudaSetDevice(dev); cudaFree(p); }
+    p = nullptr; n = 0;
+  }
+  ~DBuf() { free(); }
+  DBuf() = default;
+  DBuf(const DBuf &) = delete;
+  DBuf &operator=(const DBuf &) = delete;
+};
+
+struct Device {
+  int id = 0;
+  int n_sm = 0;
+  DBuf<uint4> packed;
+  DBuf<GroupInfo> groups;
+  DBuf<int32_t> perm, sorted_len;
+  DBuf<uint2> k1_border;   // per-SM slots
+  DBuf<int32_t> slot_busy;
+  int32_t slots_per_sm = 0, slot_cols = 0, sm_slots = 0;
+  std::vector<cudaStream_t> streams;
+  ~Device() {
+    cudaSetDevice(id);
+    for (auto s : streams) cudaStreamDestroy(s);
+  }
+};
+
+}  // namespace sw
+
+struct sw_db {
+  sw::PackedDB host;
+  std::vector<std::unique_ptr<sw::Device>> devs;
+  std::atomic<int> busy{0};
+  std::string unit_log;
+};
+
+namespace sw {
+
+// ---------------------------------------------------------------- search plan
+struct Plan {
+  std::vector<QueryPair> pairs;
+  std::vector<uint8_t> qcodes;
+  std::vector<int64_t> qoff;
+  std::vector<Unit> units;
+  int64_t prof_total = 0;
+  int64_t cells = 0;
+  int32_t n_long_seqs = 0;   // sequences [0, n_long_seqs) in sorted order go to K3
+  int32_t first_short_group = 0;
+  int32_t max_k3_seqs = 0;   // largest K3 unit (sequences)
+  int32_t max_len = 0;
+};
+
+static void validate_seqset(const sw_seqset *s, const char *what) {
+  if (!s) throw Error(SW_EINVAL, std::string(what) + " is NULL");
+  if (s->n < 0) throw Error(SW_EINVAL, std::string(what) + ": n < 0");
+  if (s->n > 0 && !s->offsets) throw Error(SW_EINVAL, std::string(what) + ": offsets is NULL");
+  if (s->n > 0 && s->offsets[0] != 0) throw Error(SW_EINVAL, std::string(what) + ": offsets[0] != 0");
+  for (int32_t k = 0; k < s->n; k++)
+    if (s->offsets[k + 1] < s->offsets[k])
+      throw Error(SW_EINVAL, std::string(what) + ": offsets not monotone at " + std::to_string(k));
+  if (s->n > 0 && s->offsets[s->n] > 0 && !s->residues)
+    throw Error(SW_EINVAL, std::string(what) + ": residues is NULL");
+}
+
+static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, int n_workers) {
+  Plan P;
+  const int32_t nq = q->n;
+  P.qoff.resize(nq + 1);
+  P.qoff[0] = 0;
+  for (int32_t k = 0; k < nq; k++) {
+    const int64_t l = q->offsets[k + 1] - q->offsets[k];
+    if (l > 65535) throw Error(SW_EINVAL, "query " + std::to_string(k) + " longer than 65535");
+    P.qoff[k + 1] = P.qoff[k] + l;
+  }
+  P.qcodes.resize(P.qoff[nq]);
+  for (int32_t k = 0; k < nq; k++)
+    for (int64_t p = 0; p < P.qoff[k + 1] - P.qoff[k]; p++) {
+      const int c = encode_residue((unsigned char)q->residues[q->offsets[k] + p]);
+      if (c < 0)
+        throw Error(SW_ERESIDUE, "query " + std::to_string(k) + ": invalid residue '" +
+                                     std::string(1, q->residues[q->offsets[k] + p]) +
+                                     "' at position " + std::to_string(p));
+      P.qcodes[P.qoff[k] + p] = (uint8_t)c;
+    }
+  // query pairs: sort by length (descending), pair neighbours (two queries per s16x2 lane)
+  std::vector<int32_t> qo(nq);
+  std::iota(qo.begin(), qo.end(), 0);
+  std::stable_sort(qo.begin(), qo.end(), [&](int32_t a, int32_t b) {
+    return P.qoff[a + 1] - P.qoff[a] > P.qoff[b + 1] - P.qoff[b];
+  });
+  int64_t prof = 0;
+  for (int32_t k = 0; k < nq; k += 2) {
+    QueryPair qp;
+    qp.qa = qo[k];
+    qp.qb = (k + 1 < nq) ? qo[k + 1] : -1;
+    qp.la = (int32_t)(P.qoff[qp.qa + 1] - P.qoff[qp.qa]);
+    qp.lb = qp.qb >= 0 ? (int32_t)(P.qoff[qp.qb + 1] - P.qoff[qp.qb]) : 0;
+    const int32_t rows = std::max(qp.la, 1);
+    qp.rows_padded = (rows + kProfileRowAlign - 1) / kProfileRowAlign * kProfileRowAlign;
+    qp.prof_off = prof;
+    prof += (int64_t)kNCodes * qp.rows_padded;
+    P.pairs.push_back(qp);
+  }
+  P.prof_total = prof;
+  P.max_len = db.max_len;
+  // long sequences -> K3: whole groups whose longest member exceeds the threshold
+  int32_t thr = o.long_threshold == 0 ? 3072 : o.long_threshold;
+  const int32_t ng = (int32_t)db.groups.size();
+  int32_t gl = 0;
+  if (thr > 0)
+    while (gl < ng && db.sorted_len[db.groups[gl].first] > thr) gl++;
+  P.first_short_group = gl;
+  P.n_long_seqs = gl > 0 ? std::min(db.n, gl * kGroup) : 0;
+
+  // cells per pair and unit target
+  std::vector<int64_t> grp_res(ng, 0);
+  for (int32_t g = 0; g < ng; g++)
+    for (int32_t k = 0; k < db.groups[g].count; k++) grp_res[g] += db.sorted_len[db.groups[g].first + k];
+  int64_t total_cells = 0;
+  for (auto &qp : P.pairs) total_cells += (int64_t)(qp.la + qp.lb) * db.residues;
+  P.cells = total_cells;
+  int64_t target = o.target_unit_cells;
+  const int depth = std::max(1, o.streams_per_device);
+  if (target <= 0) {
+    target = total_cells / std::max(1, n_workers * depth * 8);
+    target = std::max<int64_t>(target, 1000000000LL);
+    target = std::min<int64_t>(target, 50000000000LL);
+  }
+  for (int32_t p = 0; p < (int32_t)P.pairs.size(); p++) {
+    const QueryPair &qp = P.pairs[p];
+    const int64_t rows_eff = (int64_t)qp.la + qp.lb;
+    // K3 units over the long sequences (multiples of kK3Warps)
+    for (int32_t s = 0; s < P.n_long_seqs;) {
+      int32_t e = s;
+      int64_t cells = 0, work = 0;
+      while (e < P.n_long_seqs && (cells < target || e == s || (e - s) % kK3Warps)) {
+        cells += rows_eff * db.sorted_len[e];
+        work += (int64_t)qp.rows_padded * db.sorted_len[e];
+        e++;
+      }
+      P.units.push_back({kUnitIntra, p, s, e, cells, work});
+      P.max_k3_seqs = std::max(P.max_k3_seqs, e - s);
+      s = e;
+    }
+    // K1 units over the short groups
+    const int64_t rows_k1 = (int64_t)(std::max(qp.la, 1) + kK1Band - 1) / kK1Band * kK1Band;
+    for (int32_t g = gl; g < ng;) {
+      int32_t e = g;
+      int64_t cells = 0, work = 0;
+      while (e < ng && (cells < target || e == g)) {
+        cells += rows_eff * grp_res[e];
+        work += rows_k1 * db.groups[e].ncols * kGroup;
+        e++;
+      }
+      P.units.push_back({kUnitInter, p, g, e, cells, work});
+      g = e;
+    }
+  }
+  // drop empty units (e.g. all-empty queries still produce valid zero scores: keep them
+  // so that every pair gets written, but they must have cells > 0 for the scheduler)
+  for (auto &u : P.units) u.cells = std::max<int64_t>(u.cells, 1);
+  // LPT: largest work first
+  std::stable_sort(P.units.begin(), P.units.end(),
+                   [](const Unit &a, const Unit &b) { return a.work > b.work; });
+  return P;
+}
+
+// ---------------------------------------------------------------- per-search device state
+struct DevSearch {
+  Device *D = nullptr;
+  DBuf<uint8_t> qcodes;
+  DBuf<int64_t> qoff;
+  DBuf<QueryPair> pairs;
+  DBuf<int8_t> matrix;
+  DBuf<int32_t> prof;
+  DBuf<int32_t> scores_own;
+  int32_t *scores = nullptr;
+  DBuf<int2> ovf;
+  DBuf<int32_t> ovf_count;
+  DBuf<uint2> k3_border;   // [streams][max_k3_seqs][max_len]
+  DBuf<int32_t> k2_border;
+  int32_t *abort_h = nullptr, *abort_d = nullptr;
+  cudaEvent_t ev_start = nullptr, ev_end = nullptr;
+  std::vector<cudaEvent_t> u_start, u_end;  // per stream
+  int launches = 0;
+  double k1_sec = 0, k3_sec = 0;
+  int64_t k1_cells = 0, k3_cells = 0;
+  int64_t dup_cells = 0;
+  double finish_wall = 0;
+  int32_t n_ovf = 0;
+  ~DevSearch() {
+    if (D) cudaSetDevice(D->id);
+    if (abort_h) cudaFreeHost(abort_h);
+    if (ev_start) cudaEventDestroy(ev_start);
+    if (ev_end) cudaEventDestroy(ev_end);
+    for (auto e : u_start) cudaEventDestroy(e);
+    for (auto e : u_end) cudaEventDestroy(e);
+  }
+};
+
+struct UnitLog {
+  int32_t unit, worker;
+  double t_grant, t_start, t_end;
+  int64_t cells;
+  int committed;
+};
+
+static const int kOvfCap = 1 << 20;
+
+static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const Unit &U, int uidx,
+                        int stream_idx, int32_t alpha, int32_t beta, int32_t thresh) {
+  Device &D = *S.D;
+  cudaStream_t st = D.streams[stream_idx];
+  const uint32_t na = ((uint32_t)(-alpha) & 0xffffu) * 0x10001u;
+  const uint32_t nbm = ((uint32_t)(-beta) & 0xffffu) * 0x10001u;
+  if (U.kind == kUnitInter) {
+    K1Args a;
+    a.packed = D.packed.p; a.groups = D.groups.p; a.perm = D.perm.p;
+    a.prof = S.prof.p; a.pairs = S.pairs.p;
+    a.pair = U.pair; a.g0 = U.b0;
+    a.scores = S.scores; a.ndb = db.n;
+    a.thresh = thresh;
+    a.ovf = S.ovf.p; a.ovf_count = S.ovf_count.p; a.ovf_cap = kOvfCap;
+    a.border = D.k1_border.p; a.border_slot_cols = D.slot_cols; a.slots_per_sm = D.slots_per_sm;
+    a.slot_busy = D.slot_busy.p;
+    a.abort_flag = S.abort_d + uidx;
+    a.na = na; a.nb = nbm;
+    launch_k1(a, U.b1 - U.b0, 0, P.pairs[U.pair].rows_padded, st, 0);
+  } else {
+    K3Args a;
+    a.packed = D.packed.p; a.groups = D.groups.p; a.perm = D.perm.p; a.sorted_len = D.sorted_len.p;
+    a.prof = S.prof.p; a.pairs = S.pairs.p;
+    a.pair = U.pair; a.l0 = U.b0; a.l1 = U.b1;
+    a.scores = S.scores; a.ndb = db.n;
+    a.thresh = thresh;
+    a.ovf = S.ovf.p; a.ovf_count = S.ovf_count.p; a.ovf_cap = kOvfCap;
+    const int64_t stride = std::max<int64_t>(P.max_len, 1);
+    a.border = S.k3_border.p + (size_t)stream_idx * P.max_k3_seqs * stride;
+    a.border_stride = stride;
+    a.abort_flag = S.abort_d + uidx;
+    a.na = na; a.nb = nbm;
+    launch_k3(a, P.pairs[U.pair].rows_padded, st);
+  }
+  S.launches++;
+}
+
+}  // namespace sw
+
+using namespace sw;
+
+extern "C" {
+
+const char *sw_last_error(void) { return g_err.c_str(); }
+const char *sw_version(void) { return "libsw 0.1 (sm_100a)"; }
+
+void sw_opts_default(sw_opts *o) {
+  if (!o) return;
+  std::memset(o, 0, sizeof(*o));
+  o->policy = SW_POLICY_PSS;
+  o->workload_adjust = 1;
+  o->omega = 4;
+  o->streams_per_device = 3;
+  o->target_unit_cells = 0;
+  o->long_threshold = 0;
+  o->straggler_slowdown = 6;
+}
+
+int sw_db_create(const sw_seqset *dbs, const int *devices, int n_devices, sw_db **out) {
+  return guarded([&] {
+    if (!out) throw Error(SW_EINVAL, "out is NULL");
+    *out = nullptr;
+    validate_seqset(dbs, "db");
+    int ndev_avail = 0;
+    if (cudaGetDeviceCount(&ndev_avail) != cudaSuccess || ndev_avail <= 0)
+      throw Error(SW_ECUDA, "no CUDA device available (libsw has no CPU fallback)");
+    std::vector<int> devs;
+    if (!devices || n_devices <= 0) devs.push_back(0);
+    else devs.assign(devices, devices + n_devices);
+    for (int d : devs)
+      if (d < 0 || d >= ndev_avail) throw Error(SW_EINVAL, "device " + std::to_string(d) + " not present");
+    auto db = std::make_unique<sw_db>();
+    std::string err;
+    int rc = pack_database(dbs->offsets, dbs->residues, dbs->n, db->host, err);
+    if (rc != SW_OK) throw Error(rc, err);
+    const PackedDB &H = db->host;
+    for (int d : devs) {
+      auto D = std::make_unique<Device>();
+      D->id = d;
+      CK(cudaSetDevice(d));
+      CK(cudaDeviceGetAttribute(&D->n_sm, cudaDevAttrMultiProcessorCount, d));
+      D->packed.alloc(d, std::max<size_t>(H.packed.size(), 1));
+      D->groups.alloc(d, std::max<size_t>(H.groups.size(), 1));
+      D->perm.alloc(d, std::max<size_t>(H.perm.size(), 1));
+      D->sorted_len.alloc(d, std::max<size_t>(H.sorted_len.size(), 1));
+      if (!H.packed.empty()) CK(cudaMemcpy(D->packed.p, H.packed.data(), sizeof(uint4) * H.packed.size(), cudaMemcpyHostToDevice));
+      if (!H.groups.empty()) CK(cudaMemcpy(D->groups.p, H.groups.data(), sizeof(GroupInfo) * H.groups.size(), cudaMemcpyHostToDevice));
+      if (!H.perm.empty()) CK(cudaMemcpy(D->perm.p, H.perm.data(), sizeof(int32_t) * H.perm.size(), cudaMemcpyHostToDevice));
+      if (!H.sorted_len.empty()) CK(cudaMemcpy(D->sorted_len.p, H.sorted_len.data(), sizeof(int32_t) * H.sorted_len.size(), cudaMemcpyHostToDevice));
+      db->devs.push_back(std::move(D));
+    }
+    *out = db.release();
+  });
+}
+
+void sw_db_destroy(sw_db *db) { delete db; }
+int64_t sw_db_residues(const sw_db *db) { return db ? db->host.residues : 0; }
+int32_t sw_db_size(const sw_db *db) { return db ? db->host.n : 0; }
+int32_t sw_db_devices(const sw_db *db) { return db ? (int32_t)db->devs.size() : 0; }
+
+int sw_topk_device(sw_db *db, const int32_t *scores_dev, int32_t nq, int32_t ndb, int32_t k,
+                   sw_hit *hits_dev) {
+  return guarded([&] {
+    if (!db || db->devs.empty()) throw Error(SW_EINVAL, "db is NULL");
+    if (k < 0 || k > 64) throw Error(SW_EINVAL, "top_k must be in [0, 64]");
+    if (nq <= 0 || k == 0) return;
+    CK(cudaSetDevice(db->devs[0]->id));
+    launch_topk(scores_dev, nq, ndb, k, reinterpret_cast<int2 *>(hits_dev), 0);
+    CK(cudaGetLastError());
+    CK(cudaDeviceSynchronize());
+  });
+}
+
+int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t gap_open,
+              int32_t gap_extend, int32_t top_k, int32_t *scores, sw_hit *hits,
+              const sw_opts *opts_in, sw_stats *stats) {
+  if (db && db->busy.exchange(1)) {
+    g_err = "a search is already running on this sw_db";
+    return SW_EBUSY;
+  }
+  int rc = guarded([&] {
+    if (!db) throw Error(SW_EINVAL, "db is NULL");
+    validate_seqset(queries, "queries");
+    if (gap_open < 0 || gap_extend < 0) throw Error(SW_EINVAL, "gap penalties must be >= 0");
+    if ((int64_t)gap_open + 2 * (int64_t)gap_extend > (1 << 20))
+      throw Error(SW_EINVAL, "gap_open + 2*gap_extend must be <= 2^20");
+    if (top_k < 0 || top_k > 64) throw Error(SW_EINVAL, "top_k must be in [0, 64]");
+    sw_opts o;
+    sw_opts_default(&o);
+    if (opts_in) o = *opts_in;
+    if (o.omega < 1) o.omega = 4;
+    if (o.streams_per_device <= 0) o.streams_per_device = 3;
+    if (o.policy != SW_POLICY_SS && o.policy != SW_POLICY_PSS) throw Error(SW_EINVAL, "bad policy");
+    const bool dist = o.dist_world > 1;
+    if (dist && (o.dist_rank < 0 || o.dist_rank >= o.dist_world || !o.dist_host || o.dist_port <= 0))
+      throw Error(SW_EINVAL, "bad multi-process options");
+    if (dist && db->devs.size() != 1) throw Error(SW_EINVAL, "multi-process mode needs one device per rank");
+    const int8_t *M = matrix ? matrix : blosum62();
+    int max_s = INT_MIN, min_s = INT_MAX;
+    for (int k = 0; k < 24 * 24; k++) { max_s = std::max(max_s, (int)M[k]); min_s = std::min(min_s, (int)M[k]); }
+    const int32_t alpha = gap_open + gap_extend, beta = gap_extend;
+    // precision routing: s16x2 only while alpha + beta <= 16384
+    const bool s16_ok = (int64_t)alpha + beta <= 16384;
+    // flag a lane half iff best~ + max(S) > 32767; if s16 is not usable
+    // every pair is flagged (thresh = INT_MIN) and re-scored by the int32 kernel
+    const int32_t thresh = s16_ok ? (max_s > 0 ? 32768 - max_s : 32768) : INT_MIN;
+
+    const PackedDB &H = db->host;
+    const int32_t nq = queries->n, nd = H.n;
+    const int nW = dist ? 1 : (int)db->devs.size();
+    Plan P = make_plan(queries, H, o, dist ? o.dist_world : nW);
+    const double wall0 = now_s();
+
+    std::vector<std::unique_ptr<DevSearch>> S(nW);
+    // ---------------- per device setup (not timed as device work)
+    for (int w = 0; w < nW; w++) {
+      S[w] = std::make_unique<DevSearch>();
+      DevSearch &X = *S[w];
+      X.D = db->devs[w].get();
+      Device &D = *X.D;
+      CK(cudaSetDevice(D.id));
+      const int depth = o.streams_per_device;
+      while ((int)D.streams.size() < depth) {
+        cudaStream_t st;
+        CK(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+        D.streams.push_back(st);
+      }
+      if (D.slots_per_sm == 0) {
+        D.slots_per_sm = k1_blocks_per_sm();
+        D.sm_slots = 256;  // %smid < 256
+        D.slot_cols = 0;
+      }
+      int32_t need_cols = 0;
+      for (int32_t g = P.first_short_group; g < (int32_t)H.groups.size(); g++)
+        need_cols = std::max(need_cols, H.groups[g].ncols);
+      if (need_cols > D.slot_cols) {
+        D.k1_border.alloc(D.id, (size_t)D.sm_slots * D.slots_per_sm * need_cols * 32);
+        D.slot_busy.alloc(D.id, (size_t)D.sm_slots * D.slots_per_sm);
+        CK(cudaMemset(D.slot_busy.p, 0, sizeof(int32_t) * D.slot_busy.n));
+        D.slot_cols = need_cols;
+      }
+      X.qcodes.alloc(D.id, std::max<size_t>(P.qcodes.size(), 1));
+      X.qoff.alloc(D.id, P.qoff.size());
+      X.pairs.alloc(D.id, std::max<size_t>(P.pairs.size(), 1));
+      X.matrix.alloc(D.id, 24 * 24);
+      X.prof.alloc(D.id, std::max<int64_t>(P.prof_total, 1));
+      if (!P.qcodes.empty()) CK(cudaMemcpy(X.qcodes.p, P.qcodes.data(), P.qcodes.size(), cudaMemcpyHostToDevice));
+      CK(cudaMemcpy(X.qoff.p, P.qoff.data(), sizeof(int64_t) * P.qoff.size(), cudaMemcpyHostToDevice));
+      if (!P.pairs.empty()) CK(cudaMemcpy(X.pairs.p, P.pairs.data(), sizeof(QueryPair) * P.pairs.size(), cudaMemcpyHostToDevice));
+      CK(cudaMemcpy(X.matrix.p, M, 24 * 24, cudaMemcpyHostToDevice));
+      const size_t nsc = (size_t)nq * nd;
+      if (w == 0 && o.outputs_on_device && scores && !dist) X.scores = scores;
+      else { X.scores_own.alloc(D.id, std::max<size_t>(nsc, 1)); X.scores = X.scores_own.p; }
+      X.ovf.alloc(D.id, kOvfCap);
+      X.ovf_count.alloc(D.id, 1);
+      const size_t k3b = (size_t)depth * std::max(P.max_k3_seqs, 1) * std::max<int64_t>(P.max_len, 1);
+      if (P.n_long_seqs > 0) X.k3_border.alloc(D.id, k3b);
+      CK(cudaHostAlloc((void **)&X.abort_h, sizeof(int32_t) * std::max<size_t>(P.units.size(), 1), cudaHostAllocMapped));
+      std::memset(X.abort_h, 0, sizeof(int32_t) * std::max<size_t>(P.units.size(), 1));
+      CK(cudaHostGetDevicePointer((void **)&X.abort_d, X.abort_h, 0));
+      CK(cudaEventCreate(&X.ev_start));
+      CK(cudaEventCreate(&X.ev_end));
+      X.u_start.resize(depth);
+      X.u_end.resize(depth);
+      for (int k = 0; k < depth; k++) {
+        CK(cudaEventCreate(&X.u_start[k]));
+        CK(cudaEventCreate(&X.u_end[k]));
+      }
+      CK(cudaDeviceSynchronize());
+    }
+
+    // ---------------- scheduler (in-process master, or TCP client of rank 0's master)
+    std::vector<int64_t> ucells(P.units.size());
+    for (size_t u = 0; u < P.units.size(); u++) ucells[u] = P.units[u].cells;
+    std::unique_ptr<MasterServer> server;
+    std::unique_ptr<SchedClient> client;
+    sw_sched *sched = nullptr;
+    if (dist) {
+      if (o.dist_rank == 0) {
+        server = std::make_unique<MasterServer>();
+        server->start(o.dist_port, o.dist_world, (int32_t)ucells.size(), ucells.data(), o.policy,
+                      o.workload_adjust, o.omega);
+      }
+      client = std::make_unique<SchedClient>();
+      client->connect(o.dist_host, o.dist_port, o.dist_rank, 30.0);
+    } else {
+      sched = sw_sched_create(nW, (int32_t)ucells.size(), ucells.data(), o.policy, o.workload_adjust, o.omega);
+      if (!sched && !ucells.empty()) throw Error(SW_EINVAL, "scheduler creation failed");
+    }
+    struct SchedGuard { sw_sched *s; ~SchedGuard() { if (s) sw_sched_destroy(s); } } sg{sched};
+    const int my_worker_base = dist ? o.dist_rank : 0;
+    auto sreq = [&](int w, double t, int32_t *out, int cap) -> int32_t {
+      if (client) return client->request(t, out, cap);
+      if (!sched) return -1;
+      return sw_sched_request(sched, w, t, out, cap);
+    };
+    auto srep = [&](int w, double t, double cells, double sec) {
+      if (client) client->report(t, cells, sec);
+      else if (sched) sw_sched_report(sched, w, t, cells, sec);
+    };
+    auto scomp = [&](int w, int u, double t) -> int {
+      if (client) return client->complete(u, t);
+      return sched ? sw_sched_complete(sched, w, u, t) : 1;
+    };
+    auto sfin = [&](int u) -> int {
+      if (client) return client->is_finished(u);
+      return sched ? sw_sched_is_finished(sched, u) : 0;
+    };
+    auto saband = [&](int w, int u, double t) {
+      if (client) client->abandon(u, t);
+      else if (sched) sw_sched_abandon(sched, w, u, t);
+    };
+
+    // ---------------- workers: one thread per device
+    std::vector<UnitLog> ulog;
+    std::mutex ulog_mu;
+    std::atomic<int> ready{0};
+    std::vector<std::string> werr(nW);
+    std::vector<int> wcode(nW, 0);
+    const double t0 = now_s();
+    auto worker = [&](int w) {
+      DevSearch &X = *S[w];
+      Device &D = *X.D;
+      const int wid = my_worker_base + w;
+      try {
+        CK(cudaSetDevice(D.id));
+        const int depth = o.streams_per_device;
+        cudaStream_t s0 = D.streams[0];
+        // barrier across workers, then the common device start
+        ready.fetch_add(1);
+        while (ready.load() < nW) std::this_thread::yield();
+        CK(cudaEventRecord(X.ev_start, s0));
+        launch_fill(X.scores, (int64_t)nq * nd, -1, s0);
+        CK(cudaMemsetAsync(X.ovf_count.p, 0, sizeof(int32_t), s0));
+        launch_profile(X.qcodes.p, X.qoff.p, X.pairs.p, (int)P.pairs.size(), X.matrix.p, X.prof.p,
+                       P.prof_total, s0);
+        X.launches += 2 + (P.pairs.empty() ? 0 : 1);
+        CK(cudaGetLastError());
+        cudaEvent_t setup_done;
+        CK(cudaEventCreateWithFlags(&setup_done, cudaEventDisableTiming));
+        CK(cudaEventRecord(setup_done, s0));
+        for (int k = 1; k < depth; k++) CK(cudaStreamWaitEvent(D.streams[k], setup_done, 0));
+        const bool straggler = (o.straggler_mask >> wid) & 1ull;
+        const double slow = std::max(1, o.straggler_slowdown);
+        std::deque<int32_t> pending;
+        std::vector<int32_t> inflight(depth, -1);
+        std::vector<double> t_grant(P.units.size(), 0), t_launch(depth, 0);
+        std::vector<double> hold_until(depth, 0);
+        std::vector<int> completed_wait(depth, 0);
+        bool done = false;
+        double last_report = now_s();
+        int32_t buf[64];
+        while (true) {
+          bool progressed = false;
+          const double tn = now_s();
+          // completions
+          for (int k = 0; k < depth; k++) {
+            if (inflight[k] < 0) continue;
+            if (!completed_wait[k]) {
+              cudaError_t q = cudaEventQuery(X.u_end[k]);
+              if (q == cudaErrorNotReady) continue;
+              CK(q);
+              completed_wait[k] = 1;
+              if (straggler) {  // emulate a PE `slow` times slower (SURVEY §8(d) WA experiment)
+                float ms = 0;
+                cudaEventElapsedTime(&ms, X.u_start[k], X.u_end[k]);
+                hold_until[k] = tn + (slow - 1.0) * ms * 1e-3;
+              } else {
+                hold_until[k] = tn;
+              }
+            }
+            if (tn < hold_until[k]) continue;
+            const int u = inflight[k];
+            const Unit &U = P.units[u];
+            float ms = 0;
+            cudaEventElapsedTime(&ms, X.u_start[k], X.u_end[k]);
+            const int committed = scomp(wid, u, tn);
+            srep(wid, tn, (double)U.cells, std::max(1e-6, tn - last_report));
+            last_report = tn;
+            if (U.kind == kUnitInter) { X.k1_sec += ms * 1e-3; X.k1_cells += U.cells; }
+            else { X.k3_sec += ms * 1e-3; X.k3_cells += U.cells; }
+            if (!committed) X.dup_cells += U.cells;
+            {
+              std::lock_guard<std::mutex> g(ulog_mu);
+              ulog.push_back({u, wid, t_grant[u] - t0, t_launch[k] - t0, tn - t0, U.cells, committed});
+            }
+            inflight[k] = -1;
+            completed_wait[k] = 0;
+            progressed = true;
+          }
+          // cancel in-flight replicas whose task finished elsewhere (WA loser)
+          for (int k = 0; k < depth; k++)
+            if (inflight[k] >= 0 && !X.abort_h[inflight[k]] && sfin(inflight[k]))
+              X.abort_h[inflight[k]] = 1;
+          // launch pending units on free streams
+          for (int k = 0; k < depth && !pending.empty(); k++) {
+            if (inflight[k] >= 0) continue;
+            const int u = pending.front();
+            pending.pop_front();
+            if (sfin(u)) { saband(wid, u, now_s()); progressed = true; k--; continue; }
+            CK(cudaEventRecord(X.u_start[k], D.streams[k]));
+            launch_unit(P, H, X, P.units[u], u, k, alpha, beta, thresh);
+            CK(cudaGetLastError());
+            CK(cudaEventRecord(X.u_end[k], D.streams[k]));
+            inflight[k] = u;
+            t_launch[k] = now_s();
+            progressed = true;
+          }
+          // ask the master for more when the local queue is empty and a stream is free
+          int n_inflight = 0;
+          for (int k = 0; k < depth; k++) n_inflight += inflight[k] >= 0;
+          if (!done && pending.empty() && n_inflight < depth) {
+            const int32_t r = sreq(wid, now_s(), buf, 64);
+            if (r < 0) done = true;
+            else {
+              for (int32_t i = 0; i < r; i++) { pending.push_back(buf[i]); t_grant[buf[i]] = now_s(); }
+              if (r > 0) progressed = true;
+            }
+          }
+          if (done && pending.empty() && n_inflight == 0) break;
+          if (!progressed) std::this_thread::sleep_for(std::chrono::microseconds(20));
+        }
+        // int32 re-run of saturated pairs (K2), on this device's own list
+        for (int k = 0; k < depth; k++) CK(cudaStreamSynchronize(D.streams[k]));
+        int32_t novf = 0;
+        CK(cudaMemcpy(&novf, X.ovf_count.p, sizeof(int32_t), cudaMemcpyDeviceToHost));
+        if (novf > kOvfCap) throw Error(SW_ENOMEM, "overflow list capacity exceeded");
+        X.n_ovf = novf;
+        if (novf > 0) {
+          const int blocks = std::min(1024, (novf + 3) / 4);
+          const int64_t stride = std::max<int64_t>(H.max_len, 1);
+          X.k2_border.alloc(D.id, (size_t)blocks * 4 * stride * 2);
+          K2Args a;
+          a.qcodes = X.qcodes.p; a.qoff = X.qoff.p;
+          a.packed = D.packed.p; a.groups = D.groups.p; a.sorted_len = D.sorted_len.p; a.perm = D.perm.p;
+          a.matrix = X.matrix.p; a.ovf = X.ovf.p; a.ovf_count = X.ovf_count.p;
+          a.scores = X.scores; a.ndb = nd; a.alpha = alpha; a.beta = beta;
+          a.border = X.k2_border.p; a.border_stride = stride; a.n_warps_total = blocks * 4;
+          launch_k2(a, blocks, s0);
+          X.launches++;
+          CK(cudaGetLastError());
+        }
+        CK(cudaEventRecord(X.ev_end, s0));
+        CK(cudaEventSynchronize(X.ev_end));
+        CK(cudaEventDestroy(setup_done));
+        X.finish_wall = now_s();
+      } catch (const Error &e) {
+        werr[w] = e.what();
+        wcode[w] = e.code;
+        ready.fetch_add(1 << 20);  // release the barrier
+      } catch (const std::exception &e) {
+        werr[w] = e.what();
+        wcode[w] = SW_ECUDA;
+        ready.fetch_add(1 << 20);
+      }
+    };
+    std::vector<std::thread> threads;
+    for (int w = 0; w < nW; w++) threads.emplace_back(worker, w);
+    for (auto &t : threads) t.join();
+    for (int w = 0; w < nW; w++)
+      if (wcode[w]) throw Error(wcode[w], "worker " + std::to_string(w) + ": " + werr[w]);
+    if (client) client->done();
+    if (server) server->stop();
+
+    // ---------------- merge (in-process multi-device: device 0 pulls the others over
+    // NVLink and takes the element-wise max; every pair was written by >= 1 device with
+    // identical values, the rest are -1), then top-k on device 0
+    DevSearch &X0 = *S[0];
+    CK(cudaSetDevice(X0.D->id));
+    cudaStream_t s0 = X0.D->streams[0];
+    cudaEvent_t m_start, m_end;
+    CK(cudaEventCreate(&m_start));
+    CK(cudaEventCreate(&m_end));
+    CK(cudaEventRecord(m_start, s0));
+    const int64_t nsc = (int64_t)nq * nd;
+    DBuf<int32_t> tmp;
+    if (nW > 1 && nsc > 0) {
+      tmp.alloc(X0.D->id, nsc);
+      for (int w = 1; w < nW; w++) {
+        CK(cudaMemcpyPeerAsync(tmp.p, X0.D->id, S[w]->scores, S[w]->D->id, sizeof(int32_t) * nsc, s0));
+        launch_max_merge(X0.scores, tmp.p, nsc, s0);
+        X0.launches++;
+      }
+    }
+    DBuf<int2> hits_dev;
+    int2 *hits_out = nullptr;
+    if (hits && top_k > 0 && nq > 0) {
+      if (o.outputs_on_device) hits_out = reinterpret_cast<int2 *>(hits);
+      else { hits_dev.alloc(X0.D->id, (size_t)nq * top_k); hits_out = hits_dev.p; }
+      launch_topk(X0.scores, nq, nd, top_k, hits_out, s0);
+      X0.launches++;
+    }
+    CK(cudaGetLastError());
+    CK(cudaEventRecord(m_end, s0));
+    CK(cudaEventSynchronize(m_end));
+    float merge_ms = 0;
+    cudaEventElapsedTime(&merge_ms, m_start, m_end);
+    cudaEventDestroy(m_start);
+    cudaEventDestroy(m_end);
+
+    // device time: max over devices of (end - start), device 0 extended by the merge
+    double dev_sec = 0;
+    for (int w = 0; w < nW; w++) {
+      float ms = 0;
+      CK(cudaEventElapsedTime(&ms, S[w]->ev_start, S[w]->ev_end));
+      double sec = ms * 1e-3 + (w == 0 ? merge_ms * 1e-3 : 0);
+      dev_sec = std::max(dev_sec, sec);
+    }
+    // outputs
+    if (scores && nsc > 0) {
+      if (o.outputs_on_device) {
+        if (X0.scores != scores) CK(cudaMemcpy(scores, X0.scores, sizeof(int32_t) * nsc, cudaMemcpyDeviceToDevice));
+      } else {
+        CK(cudaMemcpy(scores, X0.scores, sizeof(int32_t) * nsc, cudaMemcpyDeviceToHost));
+      }
+    }
+    if (hits && top_k > 0 && nq > 0 && !o.outputs_on_device)
+      CK(cudaMemcpy(hits, hits_dev.p, sizeof(int2) * nq * top_k, cudaMemcpyDeviceToHost));
+    const double wall = now_s() - wall0;
+
+    if (stats) {
+      std::memset(stats, 0, sizeof(*stats));
+      stats->cells = P.cells;
+      stats->seconds_device = dev_sec;
+      stats->seconds_wall = wall;
+      stats->gcups = dev_sec > 0 ? (double)P.cells / dev_sec / 1e9 : 0;
+      stats->n_units = (int32_t)P.units.size();
+      stats->n_devices = nW;
+      std::vector<double> fin;
+      for (int w = 0; w < nW; w++) {
+        stats->duplicated_cells += S[w]->dup_cells;
+        stats->n_overflow_pairs += S[w]->n_ovf;
+        stats->kernel_launches += S[w]->launches;
+        stats->kernel_seconds_k1 += S[w]->k1_sec;
+        stats->kernel_seconds_k3 += S[w]->k3_sec;
+        stats->cells_k1 += S[w]->k1_cells;
+        stats->cells_k3 += S[w]->k3_cells;
+        fin.push_back(S[w]->finish_wall - t0);
+      }
+      std::sort(fin.begin(), fin.end());
+      stats->tail_seconds = fin.empty() ? 0 : fin.back() - fin[fin.size() / 2];
+      if (sched) {
+        stats->n_wa_grants = (int32_t)sw_sched_counter(sched, 1);
+        stats->n_requests = (int32_t)sw_sched_counter(sched, 0);
+      } else if (client) {
+        stats->n_wa_grants = client->wa_grants();
+        stats->n_requests = client->requests();
+      }
+      std::ostringstream js;
+      js << "[";
+      for (size_t k = 0; k < ulog.size(); k++) {
+        const UnitLog &L = ulog[k];
+        const Unit &U = P.units[L.unit];
+        js << (k ? "," : "") << "{\"unit\":" << L.unit << ",\"kind\":" << U.kind << ",\"pair\":" << U.pair
+           << ",\"worker\":" << L.worker << ",\"t_grant\":" << L.t_grant << ",\"t_start\":" << L.t_start
+           << ",\"t_end\":" << L.t_end << ",\"cells\":" << L.cells << ",\"committed\":" << L.committed << "}";
+      }
+      js << "]";
+      db->unit_log = js.str();
+      stats->unit_log_json = db->unit_log.c_str();
+    }
+  });
+  if (db) db->busy.store(0);
+  return rc;
+}
+
+}  // extern "C"

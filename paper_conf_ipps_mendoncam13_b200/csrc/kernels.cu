@@ -1,0 +1,517 @@
+// kernels.cu — the sm_100a kernels of the hot path.
+//
+// All DP kernels compute the Gotoh/Smith-Waterman recurrence of PAPER.md P12 §II.A
+// (Eq. 1 with zero first row/column; affine gaps via "3 DP matrices: H, E and F"):
+//   E(i,j) = max(E(i,j-1) - beta, H(i,j-1) - alpha)
+//   F(i,j) = max(F(i-1,j) - beta, H(i-1,j) - alpha)
+//   H(i,j) = max(0, H(i-1,j-1) + S[q_i][d_j], E(i,j), F(i,j));   score = max H
+// with alpha = open + extend, beta = extend (gap of length L costs open + L*extend).
+//
+// s16x2 kernels (K1, K3) keep two queries per 32-bit lane word (query pair qa = low
+// half, qb = high half) and use the "offset representation" of DESIGN.md §6:
+//   every H, E, F is stored as value + kOff, E and F floored at 0 (exact for H, proof
+//   in DESIGN.md §6: flooring E/F at 0 never changes max(0, ., E, F));
+//   x  = Hdiag~ + V         one 32-bit IADD; V = S_b*65536 + S_a is the "signed-packed"
+//                           profile entry, exact because Hdiag~ >= kOff >= -min(S)
+//   h  = vimax3(x, E, F)    VIMNMX3.S16x2 (E, F >= kOff, so h >= kOff = H floor 0)
+//   t  = max(h - alpha, kOff)                 VIADDMNMX.S16x2
+//   E' = max(E - beta, t),  F' = max(F - beta, t)   VIADDMNMX.S16x2 (x2)
+// Saturation: no half can wrap while best~ + max(S) <= 32767;
+// a lane half whose best~ reaches 32768 - max(S) is flagged and re-scored in int32 (K2).
+#include <cuda_runtime.h>
+#include <cstdint>
+#include <cstdio>
+#include "sw_internal.h"
+
+namespace sw {
+
+__device__ __forceinline__ uint32_t pk2(int v) { return ((uint32_t)(v & 0xffff)) * 0x10001u; }
+__device__ __forceinline__ uint32_t smid() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
+  return r;
+}
+
+// ------------------------------------------------------------------------------------
+// K4: query-pair profiles.  prof[pair][c][row] = S_b*65536 + S_a (signed-packed int32),
+// S_a = S[qa_row][c] (kPadScore past the end of qa or for the pad code), same for qb.
+// ------------------------------------------------------------------------------------
+__global__ void profile_kernel(const uint8_t *__restrict__ qcodes, const int64_t *__restrict__ qoff,
+                               const QueryPair *__restrict__ pairs, const int8_t *__restrict__ M,
+                               int32_t *__restrict__ prof) {
+  const QueryPair P = pairs[blockIdx.y];
+  const int64_t n = (int64_t)kNCodes * P.rows_padded;
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < n;
+       k += (int64_t)gridDim.x * blockDim.x) {
+    const int c = (int)(k / P.rows_padded), row = (int)(k % P.rows_padded);
+    int sa = kPadScore, sb = kPadScore;
+    if (c < 24) {
+      if (row < P.la) sa = M[qcodes[qoff[P.qa] + row] * 24 + c];
+      if (P.qb >= 0 && row < P.lb) sb = M[qcodes[qoff[P.qb] + row] * 24 + c];
+    }
+    prof[P.prof_off + k] = sb * 65536 + sa;
+  }
+}
+
+void launch_profile(const uint8_t *qcodes, const int64_t *qoff, const QueryPair *pairs, int npairs,
+                    const int8_t *matrix, int32_t *prof, int64_t, cudaStream_t st) {
+  if (npairs == 0) return;
+  dim3 grid(64, npairs);
+  profile_kernel<<<grid, 256, 0, st>>>(qcodes, qoff, pairs, matrix, prof);
+}
+
+// ------------------------------------------------------------------------------------
+// Shared per-cell update of the s16x2 kernels (one query row, one DB column).
+// ------------------------------------------------------------------------------------
+struct Cell {
+  static __device__ __forceinline__ void row(uint32_t v, uint32_t &hd, uint32_t &Hi, uint32_t &Ei,
+                                             uint32_t &f, uint32_t &best, uint32_t na, uint32_t nb,
+                                             uint32_t koff) {
+    const uint32_t x = hd + v;                        // Hdiag~ + S  (exact 32-bit add)
+    const uint32_t h = __vimax3_s16x2(x, Ei, f);      // H~(i,j) (>= kOff)
+    const uint32_t t = __viaddmax_s16x2(h, na, koff); // max(H - alpha, 0) + kOff
+    Ei = __viaddmax_s16x2(Ei, nb, t);                 // E(i, j+1)
+    f = __viaddmax_s16x2(f, nb, t);                   // F(i+1, j)
+    hd = Hi;                                          // H(i, j-1): diagonal of row i+1
+    Hi = h;
+    best = __vmaxs2(best, h);
+  }
+};
+
+// ------------------------------------------------------------------------------------
+// K1: inter-task kernel.  Block = one packing group of 32 DB sequences (lane = sequence)
+// x W warps; warp w owns rows [w*K, (w+1)*K) of each band of W*K query rows.  Warps form
+// a pipeline over (band, column tile): at step s warp w works on element e = s - w; the
+// bottom row (H, F) of a tile goes to warp w+1 through shared memory (double-buffered)
+// and, for the last warp, to warp 0 of the next band through a global border row held
+// in a per-SM slot.  One __syncthreads per step.
+// ------------------------------------------------------------------------------------
+template <int K, int W, int T>
+__global__ void __launch_bounds__(W * 32, 3) k1_kernel(const K1Args a) {
+  constexpr int BAND = W * K;
+  constexpr int S = BAND + 1;  // odd stride: lanes reading one row with different codes hit
+                               // different banks
+  extern __shared__ __align__(16) uint32_t smem[];
+  uint32_t *prof_s = smem;                                       // [2][kNCodes][S]
+  uint2 *hand = reinterpret_cast<uint2 *>(smem + 2 * kNCodes * S);  // [W][2][T][32]
+  uint32_t *red = reinterpret_cast<uint32_t *>(hand + W * 2 * T * 32);  // [W][32]
+  __shared__ int slot_s;
+
+  if (a.abort_flag && *a.abort_flag) return;  // WA: this replica lost the race
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const GroupInfo G = a.groups[a.g0 + blockIdx.x];
+  const QueryPair P = a.pairs[a.pair];
+  const int rows = P.la > P.lb ? P.la : P.lb;
+  const int nb = (rows + BAND - 1) / BAND;
+  const int nt = G.ncols / T;
+  const int total = nb * nt;
+  const uint32_t koff = pk2(kOff), na = a.na, nbeta = a.nb;
+  const int32_t *gprof = a.prof + P.prof_off;
+
+  // border slot (only when there is more than one band)
+  uint2 *border = nullptr;
+  if (nb > 1) {
+    if (threadIdx.x == 0) {
+      const int base = (int)smid() * a.slots_per_sm;
+      int k = 0;
+      for (;; k = (k + 1) % a.slots_per_sm)
+        if (atomicCAS(&a.slot_busy[base + k], 0, 1) == 0) break;
+      slot_s = base + k;
+    }
+  }
+  auto load_band = [&](int b, int slot) {
+    uint32_t *dst = prof_s + slot * kNCodes * S;
+    for (int idx = threadIdx.x; idx < kNCodes * BAND; idx += W * 32) {
+      const int c = idx / BAND, r = idx - c * BAND;
+      dst[c * S + r] = (uint32_t)__ldg(gprof + (int64_t)c * P.rows_padded + b * BAND + r);
+    }
+  };
+  load_band(0, 0);
+  if (nb > 1) load_band(1, 1);
+  __syncthreads();
+  if (nb > 1) border = a.border + (size_t)slot_s * a.border_slot_cols * 32;
+
+  uint32_t H[K], E[K];
+  uint32_t best = koff, hprev_top = koff;
+  uint4 r4 = make_uint4(0, 0, 0, 0);
+  int band = 0, tile = 0;
+  const uint4 *wp = a.packed + G.word_off + lane;
+  const int steps = total + W - 1;
+  for (int s = 0; s < steps; s++) {
+    // band b+2 reuses the profile slot of band b once every warp has left band b
+    if (s >= W - 1 && (s - (W - 1)) % nt == 0) {
+      const int bl = (s - (W - 1)) / nt - 1;
+      if (bl >= 0 && bl + 2 < nb) {
+        load_band(bl + 2, bl & 1);
+        __syncthreads();
+      }
+    }
+    const int e = s - warp;
+    if (e >= 0 && e < total) {
+      if (tile == 0) {
+#pragma unroll
+        for (int i = 0; i < K; i++) { H[i] = koff; E[i] = koff; }
+        hprev_top = koff;
+      }
+      if ((tile & (kWordCols / T - 1)) == 0) r4 = wp[(size_t)(tile * T / kWordCols) * 32];
+      const uint32_t *pr_base = prof_s + (band & 1) * kNCodes * S + warp * K;
+      const uint32_t wsel = (tile * T / 4) & 3;  // which 32-bit word of r4 holds this tile
+      const uint32_t word = wsel == 0 ? r4.x : wsel == 1 ? r4.y : wsel == 2 ? r4.z : r4.w;
+#pragma unroll
+      for (int jj = 0; jj < T; jj++) {
+        const int col = tile * T + jj;
+        const int c = (word >> (8 * jj)) & 0xff;
+        uint32_t ht, ft;
+        if (warp == 0) {
+          if (band == 0) { ht = koff; ft = koff; }
+          else { const uint2 v = border[(size_t)col * 32 + lane]; ht = v.x; ft = v.y; }
+        } else {
+          const uint2 v = hand[(((warp - 1) * 2 + ((s - 1) & 1)) * T + jj) * 32 + lane];
+          ht = v.x; ft = v.y;
+        }
+        uint32_t hd = hprev_top, f = ft;
+        hprev_top = ht;
+        const uint32_t *pr = pr_base + c * S;
+#pragma unroll
+        for (int i = 0; i < K; i++) Cell::row(pr[i], hd, H[i], E[i], f, best, na, nbeta, koff);
+        const uint2 out = make_uint2(H[K - 1], f);
+        if (warp < W - 1) hand[((warp * 2 + (s & 1)) * T + jj) * 32 + lane] = out;
+        else if (band < nb - 1) border[(size_t)col * 32 + lane] = out;
+      }
+      if (++tile == nt) { tile = 0; band++; }
+    }
+    __syncthreads();
+  }
+  red[warp * 32 + lane] = best;
+  __syncthreads();
+  if (nb > 1 && threadIdx.x == 0) atomicExch(&a.slot_busy[slot_s], 0);
+  if (warp == 0) {
+    uint32_t m = red[lane];
+#pragma unroll
+    for (int w = 1; w < W; w++) m = __vmaxs2(m, red[w * 32 + lane]);
+    if (lane < G.count) {
+      const int ss = G.first + lane;
+      const int orig = a.perm[ss];
+      const int lo = (int)(int16_t)(m & 0xffff), hi = (int)(int16_t)(m >> 16);
+      if (lo >= a.thresh) {
+        const int k = atomicAdd(a.ovf_count, 1);
+        if (k < a.ovf_cap) a.ovf[k] = make_int2(P.qa, ss);
+      } else {
+        a.scores[(int64_t)P.qa * a.ndb + orig] = lo - kOff;
+      }
+      if (P.qb >= 0) {
+        if (hi >= a.thresh) {
+          const int k = atomicAdd(a.ovf_count, 1);
+          if (k < a.ovf_cap) a.ovf[k] = make_int2(P.qb, ss);
+        } else {
+          a.scores[(int64_t)P.qb * a.ndb + orig] = hi - kOff;
+        }
+      }
+    }
+  }
+}
+
+static size_t k1_smem() {
+  constexpr int S = kK1Band + 1;
+  return sizeof(uint32_t) * 2 * kNCodes * S + sizeof(uint2) * kK1Warps * 2 * kK1Tile * 32 +
+         sizeof(uint32_t) * kK1Warps * 32;
+}
+
+int k1_blocks_per_sm() {
+  static int v = -1;
+  if (v < 0) {
+    auto fn = k1_kernel<kK1Rows, kK1Warps, kK1Tile>;
+    cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem());
+    int n = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, kK1Warps * 32, k1_smem()) !=
+        cudaSuccess)
+      n = 8;
+    v = n > 0 ? n : 1;
+  }
+  return v;
+}
+
+void launch_k1(const K1Args &a, int n_groups, int, int, cudaStream_t st, int sm_cap) {
+  if (n_groups <= 0) return;
+  auto fn = k1_kernel<kK1Rows, kK1Warps, kK1Tile>;
+  (void)sm_cap;
+  fn<<<n_groups, kK1Warps * 32, k1_smem(), st>>>(a);
+}
+
+// ------------------------------------------------------------------------------------
+// K3: intra-task kernel for long DB sequences (P14 §II.B fine-grained approach, Fig. 3a:
+// "the calculations that can be done in parallel evolve as waves on diagonals").  One
+// warp per (query pair, long sequence); lane l owns rows [l*K, (l+1)*K) of each chunk of
+// 32*K rows; at step t lane l updates column t - l and receives the row above (H, F) and
+// the residue code from lane l-1 by __shfl_up_sync; lane 31 writes the chunk's bottom
+// row to a global border read by lane 0 in the next chunk.  Block = kK3Warps sequences
+// sharing the chunk profile in shared memory laid out [code][row-in-lane][lane] (bank =
+// lane: conflict-free with 32 different codes).
+// ------------------------------------------------------------------------------------
+template <int K>
+__global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
+  constexpr int CH = 32 * K;
+  extern __shared__ __align__(16) uint32_t smem[];  // [kNCodes][K][32]
+  if (a.abort_flag && *a.abort_flag) return;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const QueryPair P = a.pairs[a.pair];
+  const int rows = P.la > P.lb ? P.la : P.lb;
+  const int nch = (rows + CH - 1) / CH;
+  const int s = a.l0 + blockIdx.x * kK3Warps + warp;
+  const bool valid = s < a.l1;
+  const int len = valid ? a.sorted_len[s] : 0;
+  const GroupInfo G = a.groups[valid ? s / kGroup : 0];
+  const uint8_t *bytes = reinterpret_cast<const uint8_t *>(a.packed);
+  const int gl = s % kGroup;
+  uint2 *border = a.border + (size_t)(blockIdx.x * kK3Warps + warp) * a.border_stride;
+  const uint32_t koff = pk2(kOff), na = a.na, nbeta = a.nb;
+  const int32_t *gprof = a.prof + P.prof_off;
+  uint32_t best = koff;
+
+  for (int ch = 0; ch < nch; ch++) {
+    __syncthreads();
+    for (int idx = threadIdx.x; idx < kNCodes * CH; idx += kK3Warps * 32) {
+      const int c = idx / CH, r = idx - c * CH;     // r = l*K + i
+      const int l = r / K, i = r - l * K;
+      smem[(c * K + i) * 32 + l] = (uint32_t)__ldg(gprof + (int64_t)c * P.rows_padded + ch * CH + r);
+    }
+    __syncthreads();
+    if (!valid || len == 0) continue;
+    uint32_t H[K], E[K];
+#pragma unroll
+    for (int i = 0; i < K; i++) { H[i] = koff; E[i] = koff; }
+    uint32_t hprev_top = koff, out_h = koff, out_f = koff, out_c = kPadCode;
+    uint4 wcur = make_uint4(0, 0, 0, 0);
+    const int steps = len + 31;
+    for (int t = 0; t < steps; t++) {
+      uint32_t in_h = __shfl_up_sync(0xffffffffu, out_h, 1);
+      uint32_t in_f = __shfl_up_sync(0xffffffffu, out_f, 1);
+      uint32_t in_c = __shfl_up_sync(0xffffffffu, out_c, 1);
+      if (lane == 0) {
+        if (t < len) {
+          if ((t & 15) == 0)
+            wcur = *reinterpret_cast<const uint4 *>(bytes + (G.word_off + (int64_t)(t >> 4) * kGroup + gl) * 16);
+          const uint32_t wsel = (t >> 2) & 3;
+          const uint32_t word = wsel == 0 ? wcur.x : wsel == 1 ? wcur.y : wsel == 2 ? wcur.z : wcur.w;
+          in_c = (word >> (8 * (t & 3))) & 0xff;
+          if (ch == 0) { in_h = koff; in_f = koff; }
+          else { const uint2 v = border[t]; in_h = v.x; in_f = v.y; }
+        }
+      }
+      const int col = t - lane;
+      if (col >= 0 && col < len) {
+        uint32_t hd = hprev_top, f = in_f;
+        hprev_top = in_h;
+        const uint32_t *pr = smem + in_c * K * 32 + lane;
+#pragma unroll
+        for (int i = 0; i < K; i++) Cell::row(pr[i * 32], hd, H[i], E[i], f, best, na, nbeta, koff);
+        out_h = H[K - 1]; out_f = f; out_c = in_c;
+        if (lane == 31 && ch < nch - 1) border[col] = make_uint2(out_h, out_f);
+      }
+    }
+  }
+  // warp max of best, then the two halves
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) best = __vmaxs2(best, __shfl_xor_sync(0xffffffffu, best, o));
+  if (valid && lane == 0) {
+    const int orig = a.perm[s];
+    const int lo = (int)(int16_t)(best & 0xffff), hi = (int)(int16_t)(best >> 16);
+    if (lo >= a.thresh) {
+      const int k = atomicAdd(a.ovf_count, 1);
+      if (k < a.ovf_cap) a.ovf[k] = make_int2(P.qa, s);
+    } else {
+      a.scores[(int64_t)P.qa * a.ndb + orig] = lo - kOff;
+    }
+    if (P.qb >= 0) {
+      if (hi >= a.thresh) {
+        const int k = atomicAdd(a.ovf_count, 1);
+        if (k < a.ovf_cap) a.ovf[k] = make_int2(P.qb, s);
+      } else {
+        a.scores[(int64_t)P.qb * a.ndb + orig] = hi - kOff;
+      }
+    }
+  }
+}
+
+void launch_k3(const K3Args &a, int, cudaStream_t st) {
+  const int n = a.l1 - a.l0;
+  if (n <= 0) return;
+  const size_t smem = sizeof(uint32_t) * kNCodes * kK3Rows * 32;
+  auto fn = k3_kernel<kK3Rows>;
+  static bool attr = false;
+  if (!attr) { cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); attr = true; }
+  fn<<<(n + kK3Warps - 1) / kK3Warps, kK3Warps * 32, smem, st>>>(a);
+}
+
+// ------------------------------------------------------------------------------------
+// K2: int32 re-run of saturated (query, sequence) pairs.  Plain int32 Gotoh with the
+// zero floor, one warp per pair, lane l owning rows [l*K2R, (l+1)*K2R) of each chunk of
+// 32*K2R rows (same wavefront as K3); scores read from the 24x24 matrix in shared
+// memory.  Rare (only near-identical long pairs saturate int16), so kept simple.
+// ------------------------------------------------------------------------------------
+constexpr int K2R = 8;
+__global__ void __launch_bounds__(128) k2_kernel(const K2Args a) {
+  __shared__ int32_t Ms[kNCodes * 32];  // [query code][db code], pad row/col = kPadScore
+  for (int k = threadIdx.x; k < kNCodes * 32; k += blockDim.x) {
+    const int r = k / 32, c = k % 32;
+    Ms[k] = (r < 24 && c < 24) ? (int32_t)a.matrix[r * 24 + c] : kPadScore;
+  }
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int count = *a.ovf_count;
+  const uint8_t *bytes = reinterpret_cast<const uint8_t *>(a.packed);
+  constexpr int NEG = -(1 << 29);
+  for (int p = gw; p < count; p += a.n_warps_total) {
+    const int q = a.ovf[p].x, s = a.ovf[p].y;
+    const int m = (int)(a.qoff[q + 1] - a.qoff[q]);
+    const uint8_t *qc = a.qcodes + a.qoff[q];
+    const int len = a.sorted_len[s];
+    const GroupInfo G = a.groups[s / kGroup];
+    const int gl = s % kGroup;
+    int32_t *border = a.border + (size_t)gw * a.border_stride * 2;
+    int best = 0;
+    const int nch = (m + 32 * K2R - 1) / (32 * K2R);
+    for (int ch = 0; ch < nch; ch++) {
+      int qr[K2R];
+#pragma unroll
+      for (int i = 0; i < K2R; i++) {
+        const int row = ch * 32 * K2R + lane * K2R + i;
+        qr[i] = row < m ? qc[row] : kPadCode;
+      }
+      int H[K2R], E[K2R];
+#pragma unroll
+      for (int i = 0; i < K2R; i++) { H[i] = 0; E[i] = NEG; }
+      int hprev_top = 0, out_h = 0, out_f = NEG, out_c = kPadCode;
+      for (int t = 0; t < len + 31; t++) {
+        int in_h = __shfl_up_sync(0xffffffffu, out_h, 1);
+        int in_f = __shfl_up_sync(0xffffffffu, out_f, 1);
+        int in_c = __shfl_up_sync(0xffffffffu, out_c, 1);
+        if (lane == 0 && t < len) {
+          in_c = bytes[(G.word_off + (int64_t)(t >> 4) * kGroup + gl) * 16 + (t & 15)];
+          if (ch == 0) { in_h = 0; in_f = NEG; }
+          else { in_h = border[2 * t]; in_f = border[2 * t + 1]; }
+        }
+        const int col = t - lane;
+        if (col >= 0 && col < len) {
+          int hd = hprev_top, hup = in_h, f = in_f;
+          hprev_top = in_h;
+#pragma unroll
+          for (int i = 0; i < K2R; i++) {
+            const int e = max(E[i] - a.beta, H[i] - a.alpha);      // E(i,j)
+            f = max(f - a.beta, hup - a.alpha);                     // F(i,j)
+            int h = hd + Ms[qr[i] * 32 + in_c];                     // diagonal
+            h = max(max(h, e), max(f, 0));                          // H(i,j)
+            hd = H[i]; H[i] = h; E[i] = e; hup = h;
+            best = max(best, h);
+          }
+          out_h = H[K2R - 1]; out_f = f; out_c = in_c;
+          if (lane == 31 && ch < nch - 1) { border[2 * col] = out_h; border[2 * col + 1] = out_f; }
+        }
+      }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) best = max(best, __shfl_xor_sync(0xffffffffu, best, o));
+    if (lane == 0) a.scores[(int64_t)q * a.ndb + a.perm[s]] = best;
+  }
+}
+
+void launch_k2(const K2Args &a, int blocks, cudaStream_t st) {
+  k2_kernel<<<blocks, 128, 0, st>>>(a);
+}
+
+// ------------------------------------------------------------------------------------
+// helpers
+// ------------------------------------------------------------------------------------
+__global__ void fill_kernel(int32_t *p, int64_t n, int32_t v) {
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x)
+    p[k] = v;
+}
+void launch_fill(int32_t *p, int64_t n, int32_t v, cudaStream_t st) {
+  if (n > 0) fill_kernel<<<592, 256, 0, st>>>(p, n, v);
+}
+__global__ void max_merge_kernel(int32_t *dst, const int32_t *src, int64_t n) {
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x)
+    dst[k] = max(dst[k], src[k]);
+}
+void launch_max_merge(int32_t *dst, const int32_t *src, int64_t n, cudaStream_t st) {
+  if (n > 0) max_merge_kernel<<<592, 256, 0, st>>>(dst, src, n);
+}
+
+// ------------------------------------------------------------------------------------
+// K5: per-query top-k under (score desc, db_index asc); entries < 0 are ignored.
+// One block per query: each thread keeps its own sorted top-k of 64-bit keys
+// (score << 32 | ~index) over a strided slice, then warps and finally warp 0 merge the
+// lists k rounds at a time with shuffles.
+// ------------------------------------------------------------------------------------
+constexpr int kTopkMax = 64;
+__device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
+  uint32_t lo = __shfl_sync(0xffffffffu, (uint32_t)v, src);
+  uint32_t hi = __shfl_sync(0xffffffffu, (uint32_t)(v >> 32), src);
+  return ((uint64_t)hi << 32) | lo;
+}
+__device__ __forceinline__ uint64_t xor64(uint64_t v, int o) {
+  uint32_t lo = __shfl_xor_sync(0xffffffffu, (uint32_t)v, o);
+  uint32_t hi = __shfl_xor_sync(0xffffffffu, (uint32_t)(v >> 32), o);
+  return ((uint64_t)hi << 32) | lo;
+}
+// warp merge: each lane holds a descending list (len k, 0 = empty); returns in lane 0..
+// the merged top-k written to out[0..k)
+__device__ void warp_merge(const uint64_t *list, int k, uint64_t *out) {
+  const int lane = threadIdx.x & 31;
+  int head = 0;
+  for (int r = 0; r < k; r++) {
+    uint64_t mine = head < k ? list[head] : 0ull;
+    uint64_t m = mine;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) { uint64_t v = xor64(m, o); m = v > m ? v : m; }
+    // keys are unique (index in the low bits) except 0 = empty
+    if (m != 0ull && mine == m) head++;
+    if (lane == 0) out[r] = m;
+  }
+}
+
+__global__ void __launch_bounds__(1024) topk_kernel(const int32_t *__restrict__ scores, int64_t ndb,
+                                                    int k, int2 *__restrict__ hits) {
+  __shared__ uint64_t wl[32][kTopkMax];
+  const int q = blockIdx.x, lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int32_t *row = scores + (int64_t)q * ndb;
+  uint64_t list[kTopkMax];
+#pragma unroll
+  for (int i = 0; i < kTopkMax; i++) list[i] = 0ull;
+  uint64_t kth = 0ull;
+  for (int64_t d = threadIdx.x; d < ndb; d += blockDim.x) {
+    const int32_t sc = row[d];
+    if (sc < 0) continue;
+    const uint64_t key = ((uint64_t)(uint32_t)sc << 32) | (uint32_t)(~(uint32_t)d);
+    if (key <= kth) continue;
+    // insert into the descending list
+    int pos = k - 1;
+    while (pos > 0 && list[pos - 1] < key) { list[pos] = list[pos - 1]; pos--; }
+    list[pos] = key;
+    kth = list[k - 1];
+  }
+  uint64_t merged[kTopkMax];
+  warp_merge(list, k, merged);
+  if (lane == 0)
+    for (int i = 0; i < k; i++) wl[warp][i] = merged[i];
+  __syncthreads();
+  if (warp == 0) {
+    uint64_t l2[kTopkMax];
+    for (int i = 0; i < k; i++) l2[i] = wl[lane][i];
+    uint64_t fin[kTopkMax];
+    warp_merge(l2, k, fin);
+    if (lane == 0)
+      for (int i = 0; i < k; i++) {
+        const uint64_t v = fin[i];
+        hits[(int64_t)q * k + i] = v ? make_int2((int)(v >> 32), (int)(~(uint32_t)v)) : make_int2(0, -1);
+      }
+  }
+}
+
+void launch_topk(const int32_t *scores, int32_t nq, int64_t ndb, int32_t k, int2 *hits, cudaStream_t st) {
+  if (nq <= 0 || k <= 0) return;
+  topk_kernel<<<nq, 1024, 0, st>>>(scores, ndb, k, hits);
+}
+
+}  // namespace sw

@@ -1,0 +1,130 @@
+// sw_internal.h — internal declarations shared by libsw's host runtime and kernels.
+// (Nothing here is shared with oracle/: the product path has its own alphabet table,
+// BLOSUM62 transcription and arithmetic.)
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+#include <stdexcept>
+#include <string>
+#include <vector>
+
+namespace sw {
+
+// internal exception carrying an SW_E* code; converted to a return code at the C-ABI
+struct Error : std::runtime_error {
+  int code;
+  Error(int c, const std::string &m) : std::runtime_error(m), code(c) {}
+};
+
+// ---- alphabet / scoring constants -------------------------------------------------
+constexpr int kNCodes = 25;        // 24 NCBI letters ARNDCQEGHILKMFPSTWYVBZX* + pad
+constexpr int kPadCode = 24;       // packing pad (DB columns beyond a sequence's end)
+constexpr int kPadScore = -1;      // S[.][pad] and pad query rows: <= 0 (reading R9)
+constexpr int kOff = 128;          // offset representation bias of the s16x2 kernels
+                                   // (>= -min int8 score so 32-bit adds never borrow)
+constexpr int kWordCols = 16;      // residues per packed 128-bit word
+constexpr int kGroup = 32;         // DB sequences per packing group (one per lane)
+
+// K1 (inter-task) geometry: W warps per block split each band of W*K rows
+constexpr int kK1Rows = 16;        // K: rows per warp (registers H[K], E[K])
+constexpr int kK1Warps = 8;        // W
+constexpr int kK1Tile = 4;         // T: columns per pipeline step
+constexpr int kK1Band = kK1Rows * kK1Warps;
+// K3 (intra-task) geometry: one warp per (query pair, long DB sequence)
+constexpr int kK3Rows = 16;        // rows per lane
+constexpr int kK3Chunk = 32 * kK3Rows;   // rows per warp chunk
+constexpr int kK3Warps = 4;        // long sequences per block (share the chunk profile)
+constexpr int kProfileRowAlign = 512;    // lcm(kK1Band, kK3Chunk)
+
+// ---- packed database (device) -------------------------------------------------------
+struct GroupInfo {       // one packing group of up to 32 length-sorted sequences
+  int64_t word_off;      // offset (in uint4 words) of word 0, lane 0
+  int32_t ncols;         // padded columns (multiple of 16, >= kMinCols)
+  int32_t first;         // index of the group's first sequence in sorted order
+  int32_t count;         // real sequences in the group (<= 32)
+  int32_t pad_;
+};
+constexpr int kMinCols = 32;       // groups padded to >= (W-1)*T columns (K1 pipeline)
+
+// ---- a unit of work (one task of the paper's scheduler) -----------------------------
+enum UnitKind : int32_t { kUnitInter = 0, kUnitIntra = 1 };
+struct Unit {
+  int32_t kind;
+  int32_t pair;          // query pair index
+  int32_t b0, b1;        // group range [b0,b1) (inter) or long-seq range (intra)
+  int64_t cells;         // real cells (sum |q|*|d|), for GCUPS and PSS rates
+  int64_t work;          // padded lane-cells (balancing)
+};
+
+// ---- query pairs ----------------------------------------------------------------------
+struct QueryPair {
+  int32_t qa, qb;        // query indices (qb = -1 if absent)
+  int32_t la, lb;        // lengths
+  int32_t rows_padded;   // rows in the profile (multiple of kProfileRowAlign, >= 1 band)
+  int64_t prof_off;      // offset (in int32) of this pair's profile [kNCodes][rows_padded]
+};
+
+// ---- kernel launchers (kernels.cu) -------------------------------------------------------
+struct K1Args {
+  const uint4 *packed; const GroupInfo *groups; const int32_t *perm;
+  const int32_t *prof; const QueryPair *pairs;
+  int32_t pair; int32_t g0;          // unit: pair, first group (grid.x groups)
+  int32_t *scores; int64_t ndb;      // [nq][ndb]
+  int32_t thresh;                    // overflow threshold on best~ (offset repr)
+  int2 *ovf; int32_t *ovf_count; int32_t ovf_cap;
+  uint2 *border; int32_t border_slot_cols; int32_t slots_per_sm; int32_t *slot_busy;
+  const volatile int32_t *abort_flag;
+  uint32_t na, nb;                   // packed -alpha, -beta
+};
+struct K3Args {   // sequences [l0,l1) in sorted order (the long groups)
+  const uint4 *packed; const GroupInfo *groups; const int32_t *perm; const int32_t *sorted_len;
+  const int32_t *prof; const QueryPair *pairs;
+  int32_t pair; int32_t l0, l1;
+  int32_t *scores; int64_t ndb;
+  int32_t thresh;
+  int2 *ovf; int32_t *ovf_count; int32_t ovf_cap;
+  uint2 *border; int64_t border_stride;   // per-warp border (>= max long len)
+  const volatile int32_t *abort_flag;
+  uint32_t na, nb;
+};
+struct K2Args {   // int32 re-run of saturated pairs (warp per pair)
+  const uint8_t *qcodes; const int64_t *qoff;
+  const uint4 *packed; const GroupInfo *groups; const int32_t *sorted_len; const int32_t *perm;
+  const int8_t *matrix;                   // 24x24 (device)
+  const int2 *ovf; const int32_t *ovf_count;
+  int32_t *scores; int64_t ndb;
+  int32_t alpha, beta;
+  int32_t *border; int64_t border_stride; int32_t n_warps_total;
+};
+
+void launch_profile(const uint8_t *qcodes, const int64_t *qoff, const QueryPair *pairs, int npairs,
+                    const int8_t *matrix, int32_t *prof, int64_t prof_total, cudaStream_t st);
+void launch_k1(const K1Args &a, int n_groups, int max_cols, int rows_padded, cudaStream_t st,
+               int sm_cap);
+void launch_k3(const K3Args &a, int rows_padded, cudaStream_t st);
+void launch_k2(const K2Args &a, int blocks, cudaStream_t st);
+void launch_fill(int32_t *p, int64_t n, int32_t v, cudaStream_t st);
+void launch_max_merge(int32_t *dst, const int32_t *src, int64_t n, cudaStream_t st);
+void launch_topk(const int32_t *scores, int32_t nq, int64_t ndb, int32_t k, int2 *hits,
+                 cudaStream_t st);
+int k1_blocks_per_sm();
+
+// ---- host packing (pack.cpp) ----------------------------------------------------------------
+int encode_residue(int ascii);   // -1 if invalid
+const int8_t *blosum62();        // libsw's own transcription (24x24)
+
+struct PackedDB {
+  int32_t n = 0;
+  int64_t residues = 0;
+  std::vector<int32_t> perm;         // sorted order -> original index
+  std::vector<int32_t> sorted_len;   // lengths in sorted order (descending)
+  std::vector<GroupInfo> groups;     // groups of 32 consecutive sorted sequences
+  std::vector<uint4> packed;         // interleaved words
+  int32_t max_len = 0;
+};
+// Encode (strict alphabet), sort by length (descending, stable), group and interleave.
+// Returns 0 or an SW_E* code with the message in err.
+int pack_database(const int64_t *offsets, const char *residues, int32_t n, PackedDB &out,
+                  std::string &err);
+
+}  // namespace sw

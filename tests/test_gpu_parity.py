@@ -1,0 +1,234 @@
+"""Parity of the CUDA path (libsw through its C-ABI) with the oracle, bit-exact.
+
+Every score is an integer, so the bar is equality for every pair.
+Inputs are seeded (seqgen); expected values come only from oracle/.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import seqgen
+from paper_conf_ipps_mendoncam13_b200 import Database, SwError
+
+pytestmark = pytest.mark.gpu
+
+
+def _search(db, qs, **kw):
+    D = Database(db, devices=kw.pop("devices", None))
+    try:
+        return D.search(qs, **kw)
+    finally:
+        D.close()
+
+
+def _check_topk(res, scores_ref, k):
+    s, i = oracle.topk(scores_ref, k)
+    assert (np.asarray(res.hit_scores) == s).all()
+    assert (np.asarray(res.hit_index) == i).all()
+
+
+def test_c1_full_parity():
+    """C1 (BASELINE configs[0]): 1 x 100 aa vs 2,000 SwissProt-shaped sequences."""
+    w = seqgen.make_workload("C1")
+    ref = oracle.search(w.queries, w.db)
+    r = _search(w.db, w.queries, top_k=10)
+    assert (r.scores == ref).all()
+    _check_topk(r, ref, 10)
+    assert r.stats["cells"] == int(w.queries.total) * int(w.db.total)
+
+
+def _mixed_case(seed, nq=8, nd=700, max_len=3500):
+    qlens = [1, 15, 16, 17, 127, 129, 600, 1300][:nq]
+    qs = seqgen.SeqSet.from_list([seqgen.residues(seqgen.stream_seed(seed, f"q{k}"), 0, L).tobytes()
+                                  for k, L in enumerate(qlens)])
+    db = seqgen.random_seqset(seed, nd, 0, max_len)
+    # some lengths exactly at group/tile boundaries, and a planted copy of a query
+    extra = [b"", b"W", seqgen.residues(seed, 0, 16).tobytes(), seqgen.residues(seed, 0, 32).tobytes(),
+             qs.seq(nq - 2), qs.seq(nq - 1) + qs.seq(nq - 3)]
+    db = seqgen.SeqSet.from_list([db.seq(i) for i in range(db.n)] + extra)
+    return qs, db
+
+
+def test_mixed_lengths_k1_and_k3():
+    qs, db = _mixed_case(7)
+    ref = oracle.search(qs, db)
+    for thr in (0, 256, -1):   # auto (3072), many long sequences via K3, none via K3
+        r = _search(db, qs, top_k=12, long_threshold=thr)
+        bad = np.argwhere(r.scores != ref)
+        assert len(bad) == 0, (thr, bad[:10], r.scores[tuple(bad[0])], ref[tuple(bad[0])])
+        _check_topk(r, ref, 12)
+
+
+@pytest.mark.parametrize("go,ge", [(10, 2), (0, 2), (0, 0), (11, 1), (5, 0), (40, 7)])
+def test_gap_settings(go, ge):
+    qs, db = _mixed_case(11, nq=6, nd=300, max_len=1200)
+    ref = oracle.search(qs, db, gap_open=go, gap_extend=ge)
+    r = _search(db, qs, gap_open=go, gap_extend=ge, top_k=5, long_threshold=400)
+    assert (r.scores == ref).all()
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_random_matrices(seed):
+    M = seqgen.random_matrix(seed, lo=-12, hi=15)
+    M[3, 5] = 40    # asymmetric entry: query row vs db column must not be transposed
+    qs, db = _mixed_case(20 + seed, nq=5, nd=250, max_len=900)
+    ref = oracle.search(qs, db, matrix=M, gap_open=6, gap_extend=3)
+    r = _search(db, qs, matrix=M, gap_open=6, gap_extend=3, top_k=4, long_threshold=300)
+    assert (r.scores == ref).all()
+
+
+def test_overflow_rerun_int32():
+    """Saturation of the s16x2 lanes is detected and the pair re-scored in int32 (K2):
+    an all-W query of 3,200 aa vs a sequence containing it scores 11*3200 = 35,200."""
+    wq = "W" * 3200
+    qs = seqgen.SeqSet.from_list([wq, seqgen.residues(3, 0, 3100).tobytes(), "WWWW"])
+    base = seqgen.random_seqset(4, 120, 10, 4000)
+    seqs = [base.seq(i) for i in range(base.n)]
+    seqs[5] = b"ACD" + wq.encode() + b"KLM"
+    seqs[77] = wq.encode()[:1500]
+    db = seqgen.SeqSet.from_list(seqs)
+    ref = oracle.search(qs, db)
+    assert ref.max() > 32767
+    for thr in (0, 1000):
+        r = _search(db, qs, top_k=3, long_threshold=thr)
+        assert (r.scores == ref).all()
+        assert r.stats["n_overflow_pairs"] >= 1
+
+
+def test_big_matrix_forces_many_overflows():
+    M = np.full((24, 24), -20, np.int8)
+    np.fill_diagonal(M, 120)
+    qs = seqgen.SeqSet.from_list([b"A" * 400, b"C" * 300, seqgen.residues(9, 0, 500).tobytes()])
+    db = seqgen.SeqSet.from_list([b"A" * 350, b"C" * 280, b"AC" * 200, b"W" * 10] +
+                                 [seqgen.residues(10, k * 1000, 300 + k).tobytes() for k in range(60)])
+    ref = oracle.search(qs, db, matrix=M, gap_open=10, gap_extend=2)
+    r = _search(db, qs, matrix=M, top_k=5)
+    assert (r.scores == ref).all()
+    assert r.stats["n_overflow_pairs"] >= 2
+
+
+def test_precision_routing_large_gaps():
+    """alpha + beta > 16384: every pair goes to the int32 kernel."""
+    qs, db = _mixed_case(5, nq=4, nd=100, max_len=500)
+    ref = oracle.search(qs, db, gap_open=20000, gap_extend=1)
+    r = _search(db, qs, gap_open=20000, gap_extend=1, top_k=3)
+    assert (r.scores == ref).all()
+
+
+def test_edge_cases():
+    db = seqgen.SeqSet.from_list(["", "A", "ACDEFGHIK", ""])
+    qs = seqgen.SeqSet.from_list(["", "WWA", "k"])        # lower case accepted
+    ref = oracle.search(seqgen.SeqSet.from_list(["", "WWA", "K"]), db)
+    r = _search(db, qs, top_k=6)
+    assert (r.scores == ref).all()
+    assert (np.asarray(r.hit_index)[:, 4:] == -1).all()   # ndb < k: empty slots {0, -1}
+    assert (np.asarray(r.hit_scores)[:, 4:] == 0).all()
+    # no queries / no database sequences
+    r0 = _search(db, seqgen.SeqSet.from_list([]), top_k=3)
+    assert r0.scores.shape == (0, 4)
+    r1 = _search(seqgen.SeqSet.from_list([]), qs, top_k=3)
+    assert r1.scores.shape == (3, 0) and (np.asarray(r1.hit_index) == -1).all()
+
+
+def test_errors_are_reported():
+    db = seqgen.SeqSet.from_list(["ACD", "AJX"])
+    with pytest.raises(SwError) as e:
+        Database(db)
+    assert e.value.code == -2 and "sequence 1" in str(e.value)
+    D = Database(seqgen.SeqSet.from_list(["ACD"]))
+    with pytest.raises(SwError) as e:
+        D.search(seqgen.SeqSet.from_list(["AC1"]))
+    assert e.value.code == -2
+    with pytest.raises(SwError):
+        D.search(seqgen.SeqSet.from_list(["ACD"]), gap_open=-1)
+    D.close()
+
+
+def test_results_independent_of_schedule():
+    """Scores are identical for every policy, WA setting, unit size and stream count."""
+    qs, db = _mixed_case(31, nq=8, nd=600, max_len=2500)
+    ref = oracle.search(qs, db)
+    D = Database(db)
+    for kw in [dict(policy="ss"), dict(policy="pss", workload_adjust=False),
+               dict(target_unit_cells=2_000_000, streams=1),
+               dict(target_unit_cells=5_000_000, streams=4, long_threshold=200),
+               dict(target_unit_cells=2**62)]:
+        r = D.search(qs, top_k=7, **kw)
+        assert (r.scores == ref).all(), kw
+        _check_topk(r, ref, 7)
+    D.close()
+
+
+def test_two_workers_one_gpu_with_straggler():
+    """Two slave workers on one GPU (two replicas, separate streams); worker 1 emulates a
+    6x slower PE.  WA duplicates its late units; results stay bit-exact and every pair is
+    merged from the committing worker."""
+    qs, db = _mixed_case(41, nq=8, nd=800, max_len=2000)
+    ref = oracle.search(qs, db)
+    r = _search(db, qs, devices=[0, 0], top_k=5, target_unit_cells=3_000_000,
+                straggler_mask=0b10, straggler_slowdown=6)
+    assert (r.scores == ref).all()
+    _check_topk(r, ref, 5)
+    assert r.stats["n_devices"] == 2
+    log = r.stats["unit_log"]
+    assert {e["worker"] for e in log} == {0, 1}
+    assert sum(e["committed"] for e in log) == r.stats["n_units"]
+
+
+def test_outputs_on_device():
+    import torch
+    qs, db = _mixed_case(51, nq=4, nd=200, max_len=800)
+    ref = oracle.search(qs, db)
+    r = _search(db, qs, top_k=3, outputs_on_device=True)
+    assert r.scores.is_cuda
+    assert (r.scores.cpu().numpy() == ref).all()
+    s, i = oracle.topk(ref, 3)
+    assert (r.hit_index.cpu().numpy() == i).all() and (r.hit_scores.cpu().numpy() == s).all()
+
+
+def test_c5_long_sequences_small():
+    """C5 shape at reduced count: 8 x 5,000-aa queries (one W/C/Y-rich overflow query) vs
+    long sequences (10k-35k) on the intra-task kernel; full parity."""
+    w = seqgen.make_workload("C5", n_db=24)
+    ref = oracle.search(w.queries, w.db)
+    r = _search(w.db, w.queries, top_k=5)
+    assert (r.scores == ref).all()
+    assert r.stats["cells_k3"] > 0 and r.stats["n_overflow_pairs"] >= 1
+    _check_topk(r, ref, 5)
+
+
+def _sampled_parity(w, r, n_sample, seed):
+    rng = np.random.default_rng(seed)
+    qi = rng.integers(0, w.queries.n, n_sample).astype(np.int32)
+    di = rng.integers(0, w.db.n, n_sample).astype(np.int32)
+    # always include the longest DB sequences and every planted pair
+    longest = np.argsort(-w.db.lengths)[:8]
+    pq = [p["query"] for p in w.meta["planted"]]
+    pd = [p["slot"] for p in w.meta["planted"]]
+    qi = np.concatenate([qi, np.repeat(np.arange(w.queries.n), len(longest)), pq]).astype(np.int32)
+    di = np.concatenate([di, np.tile(longest, w.queries.n), pd]).astype(np.int32)
+    ref = oracle.pairs(w.queries, w.db, qi, di)
+    got = np.asarray(r.scores)[qi, di]
+    assert (got == ref).all(), np.argwhere(got != ref)[:5]
+    # self-hits (reading R16): each query's best hit is its own DB slot (or an equal score)
+    for p in w.meta["planted"]:
+        if p["kind"] == "self":
+            q = p["query"]
+            assert np.asarray(r.hit_scores)[q, 0] == np.asarray(r.scores)[q].max()
+            assert np.asarray(r.scores)[q, p["slot"]] == np.asarray(r.hit_scores)[q, 0]
+
+
+def test_c2_full_size_sampled():
+    w = seqgen.make_workload("C2")
+    r = _search(w.db, w.queries, top_k=10)
+    _sampled_parity(w, r, 1500, 2)
+    # every pair's score is a valid non-negative integer
+    assert (np.asarray(r.scores) >= 0).all()
+
+
+@pytest.mark.slow
+def test_c4_full_size_sampled():
+    w = seqgen.make_workload("C4")
+    r = _search(w.db, w.queries, top_k=10)
+    _sampled_parity(w, r, 1000, 4)
+    assert (np.asarray(r.scores) >= 0).all()

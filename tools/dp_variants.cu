@@ -1,0 +1,229 @@
+// Microbenchmark of Gotoh inner-loop formulations on sm_100a (s16x2, two queries per lane).
+// Each thread: one synthetic DB sequence (n columns) against a strip of K query rows held in
+// registers; profile in shared memory (conflict-free stride).  Prints cells/clk/SM per
+// variant and checks every variant returns the same per-thread best.
+#include <cstdio>
+#include <cstdint>
+#include <vector>
+#include <cstring>
+
+#define NCOL 1024
+#define NC 32           // profile codes (padded)
+#define KOFF 256        // offset representation bias (per half)
+
+__device__ __forceinline__ uint32_t pk(int v) { return ((uint32_t)(v & 0xffff)) * 0x10001u; }
+
+// profile entries: P[c][i] s16x2 (natural), Pa = S + alpha (s16x2), V = signed-packed int32 S
+template <int K, int VAR>
+__global__ void __launch_bounds__(256) dp(const uint4 *__restrict__ db, const uint32_t *__restrict__ gprof,
+                                          int alpha, int beta, uint32_t *out, int reps) {
+  __shared__ uint32_t P[NC * (K + 1)];
+  for (int k = threadIdx.x; k < NC * (K + 1); k += blockDim.x) P[k] = gprof[k];
+  __syncthreads();
+  const uint32_t na = pk(-alpha), nb = pk(-beta), A32 = (uint32_t)(alpha * 65537),
+                 B32 = (uint32_t)(beta * 65537), Kp = pk(KOFF), zero = 0;
+  const int tid = blockIdx.x * blockDim.x + threadIdx.x;
+  uint32_t best = (VAR >= 2) ? Kp : 0;
+  for (int rep = 0; rep < reps; rep++) {
+    uint32_t H[K], E[K];
+#pragma unroll
+    for (int i = 0; i < K; i++) {
+      if (VAR == 0) { H[i] = na; E[i] = 0; }            // T-state: T = H - alpha
+      else if (VAR == 1) { H[i] = 0; E[i] = pk(alpha); }// E~ = E + alpha; E(i,0)=0
+      else { H[i] = Kp; E[i] = Kp; }                    // offset repr, floored E
+    }
+    const uint4 *p = db + tid;
+    for (int w = 0; w < NCOL / 16; w++) {
+      uint4 r4 = p[(size_t)w * gridDim.x * blockDim.x];
+      uint32_t rw[4] = {r4.x, r4.y, r4.z, r4.w};
+#pragma unroll
+      for (int b = 0; b < 16; b++) {
+        const int c = (rw[b >> 2] >> ((b & 3) * 8)) & 31;
+        const uint32_t *pr = P + c * (K + 1);
+        if (VAR == 0) {
+          uint32_t tdiag = na, tup = na, f = 0;   // row 0: H = 0 -> T = -alpha; F = 0
+#pragma unroll
+          for (int i = 0; i < K; i++) {
+            uint32_t sa = pr[i];                    // S + alpha
+            uint32_t e = __viaddmax_s16x2(E[i], nb, H[i]);
+            f = __viaddmax_s16x2(f, nb, tup);
+            uint32_t h = __vimax3_s16x2_relu(__vadd2(tdiag, sa), e, f);
+            tdiag = H[i];
+            uint32_t t = __vadd2(h, na);
+            H[i] = t; E[i] = e; tup = t;
+            best = __vmaxs2(best, h);
+          }
+        } else if (VAR == 1) {
+          uint32_t hd = 0, hup = 0, f = pk(alpha);
+#pragma unroll
+          for (int i = 0; i < K; i++) {
+            uint32_t sa = pr[i];                    // S + alpha
+            uint32_t e = __viaddmax_s16x2(E[i], nb, H[i]);
+            f = __viaddmax_s16x2(f, nb, hup);
+            uint32_t m = __vmaxs2(e, f);
+            uint32_t x = __viaddmax_s16x2(hd, sa, m);
+            uint32_t h = __viaddmax_s16x2_relu(x, na, zero);
+            hd = H[i]; H[i] = h; E[i] = e; hup = h;
+            best = __vmaxs2(best, x);
+          }
+        } else if (VAR == 2) {   // offset: x by IADD, eager E, floored t'
+          uint32_t hd = Kp, f = Kp;
+#pragma unroll
+          for (int i = 0; i < K; i++) {
+            uint32_t v = pr[i];                     // signed-packed S
+            uint32_t x = hd + v;
+            uint32_t h = __vimax3_s16x2(x, E[i], f);
+            uint32_t t = __viaddmax_s16x2(h, na, Kp);
+            E[i] = __viaddmax_s16x2(E[i], nb, t);
+            f = __viaddmax_s16x2(f, nb, t);
+            hd = H[i]; H[i] = h;
+            best = __vmaxs2(best, h);
+          }
+        } else if (VAR == 4) {   // VAR2 with E/F as IADD + 2-input max
+          uint32_t hd = Kp, f = Kp;
+#pragma unroll
+          for (int i = 0; i < K; i++) {
+            uint32_t v = pr[i];
+            uint32_t x = hd + v;
+            uint32_t h = __vimax3_s16x2(x, E[i], f);
+            uint32_t t = __viaddmax_s16x2(h, na, Kp);
+            E[i] = __vmaxs2(E[i] - B32, t);
+            f = __vmaxs2(f - B32, t);
+            hd = H[i]; H[i] = h;
+            best = __vmaxs2(best, h);
+          }
+        } else if (VAR == 5) {   // VAR2 with best merged every 2 rows (vimax3)
+          uint32_t hd = Kp, f = Kp;
+#pragma unroll
+          for (int i = 0; i < K; i += 2) {
+            uint32_t v = pr[i];
+            uint32_t x = hd + v;
+            uint32_t h = __vimax3_s16x2(x, E[i], f);
+            uint32_t t = __viaddmax_s16x2(h, na, Kp);
+            E[i] = __viaddmax_s16x2(E[i], nb, t);
+            f = __viaddmax_s16x2(f, nb, t);
+            hd = H[i]; H[i] = h;
+            uint32_t v2 = pr[i + 1];
+            uint32_t x2 = hd + v2;
+            uint32_t h2 = __vimax3_s16x2(x2, E[i + 1], f);
+            uint32_t t2 = __viaddmax_s16x2(h2, na, Kp);
+            E[i + 1] = __viaddmax_s16x2(E[i + 1], nb, t2);
+            f = __viaddmax_s16x2(f, nb, t2);
+            hd = H[i + 1]; H[i + 1] = h2;
+            best = __vimax3_s16x2(best, h, h2);
+          }
+        } else if (VAR == 6) {   // VAR2 with x by packed vadd2 (profile s16x2 natural S)
+          uint32_t hd = Kp, f = Kp;
+#pragma unroll
+          for (int i = 0; i < K; i++) {
+            uint32_t v = pr[i];
+            uint32_t x = __vadd2(hd, v);
+            uint32_t h = __vimax3_s16x2(x, E[i], f);
+            uint32_t t = __viaddmax_s16x2(h, na, Kp);
+            E[i] = __viaddmax_s16x2(E[i], nb, t);
+            f = __viaddmax_s16x2(f, nb, t);
+            hd = H[i]; H[i] = h;
+            best = __vmaxs2(best, h);
+          }
+        } else {                 // all full-rate: IADD + 2-input max
+          uint32_t hd = Kp, f = Kp;
+#pragma unroll
+          for (int i = 0; i < K; i++) {
+            uint32_t v = pr[i];
+            uint32_t x = hd + v;
+            uint32_t h = __vmaxs2(__vmaxs2(x, E[i]), f);
+            uint32_t t = __vmaxs2(h - A32, Kp);
+            E[i] = __vmaxs2(E[i] - B32, t);
+            f = __vmaxs2(f - B32, t);
+            hd = H[i]; H[i] = h;
+            best = __vmaxs2(best, h);
+          }
+        }
+      }
+    }
+  }
+  if (VAR == 1) {  // best tracked on x = H + alpha (unfloored)
+    uint32_t lo = (uint32_t)max(0, (int)(int16_t)(best & 0xffff) - alpha);
+    uint32_t hi = (uint32_t)max(0, (int)(int16_t)(best >> 16) - alpha);
+    best = lo | (hi << 16);
+  } else if (VAR >= 2) {
+    best = __vsub2(best, Kp);
+  }
+  out[tid] = best;
+}
+
+static int blosum_like(int a, int b) { return a == b ? 4 + (a % 8) : ((a * 7 + b * 3) % 7) - 4; }
+
+template <int K, int VAR>
+double run(int nthreads, const uint4 *ddb, int alpha, int beta, uint32_t *dout, std::vector<uint32_t> &hout,
+           int reps, double clk_ghz, int nsm) {
+  // profile for this variant
+  std::vector<uint32_t> prof(NC * (K + 1), 0);
+  for (int c = 0; c < NC; c++)
+    for (int i = 0; i < K; i++) {
+      int qa = (i * 5 + 1) % 20, qb = (i * 11 + 3) % 20;
+      int sa = c < 20 ? blosum_like(qa, c) : -1, sb = c < 20 ? blosum_like(qb, c) : -1;
+      uint32_t v;
+      if (VAR == 0 || VAR == 1) v = (uint32_t)((sa + alpha) & 0xffff) | ((uint32_t)((sb + alpha) & 0xffff) << 16);
+      else if (VAR == 6) v = (uint32_t)(sa & 0xffff) | ((uint32_t)(sb & 0xffff) << 16);
+      else v = (uint32_t)(sb * 65536 + sa);
+      prof[c * (K + 1) + i] = v;
+    }
+  uint32_t *dprof; cudaMalloc(&dprof, prof.size() * 4);
+  cudaMemcpy(dprof, prof.data(), prof.size() * 4, cudaMemcpyHostToDevice);
+  int blocks = nthreads / 256;
+  dp<K, VAR><<<blocks, 256>>>(ddb, dprof, alpha, beta, dout, 1);
+  cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+  cudaEventRecord(e0);
+  dp<K, VAR><<<blocks, 256>>>(ddb, dprof, alpha, beta, dout, reps);
+  cudaEventRecord(e1); cudaEventSynchronize(e1);
+  float ms; cudaEventElapsedTime(&ms, e0, e1);
+  cudaError_t err = cudaGetLastError();
+  hout.resize(nthreads);
+  cudaMemcpy(hout.data(), dout, nthreads * 4, cudaMemcpyDeviceToHost);
+  double cells = (double)nthreads * NCOL * K * 2 * reps;
+  double gcups = cells / (ms * 1e6);
+  cudaFuncAttributes fa; cudaFuncGetAttributes(&fa, dp<K, VAR>);
+  printf("K=%2d VAR=%d regs=%3d  %8.1f GCUPS  %6.2f cells/clk/SM (at %.3f GHz)  err=%s\n", K, VAR, fa.numRegs, gcups,
+         cells / (ms * 1e-3) / (clk_ghz * 1e9) / nsm, clk_ghz, cudaGetErrorString(err));
+  cudaFree(dprof);
+  return gcups;
+}
+
+int main() {
+  cudaDeviceProp p; cudaGetDeviceProperties(&p, 0);
+  int nsm = p.multiProcessorCount;
+  int nthreads = nsm * 256 * 8;
+  std::vector<uint8_t> res((size_t)nthreads * NCOL);
+  uint64_t s = 12345;
+  for (auto &r : res) { s = s * 6364136223846793005ULL + 1442695040888963407ULL; r = (uint8_t)((s >> 33) % 20); }
+  // interleave: word w of thread t at [w * nthreads + t]
+  std::vector<uint4> packed((size_t)nthreads * NCOL / 16);
+  for (int t = 0; t < nthreads; t++)
+    for (int w = 0; w < NCOL / 16; w++) {
+      uint8_t b[16];
+      for (int k = 0; k < 16; k++) b[k] = res[(size_t)t * NCOL + w * 16 + k];
+      memcpy(&packed[(size_t)w * nthreads + t], b, 16);
+    }
+  uint4 *ddb; cudaMalloc(&ddb, packed.size() * 16);
+  cudaMemcpy(ddb, packed.data(), packed.size() * 16, cudaMemcpyHostToDevice);
+  uint32_t *dout; cudaMalloc(&dout, nthreads * 4);
+  double ghz = 1.965;  // nominal max; actual printed by nvidia-smi sampling
+  std::vector<uint32_t> r0, r1, r2, r3;
+  int reps = 2;
+  std::vector<uint32_t> r4, r5, r6;
+  for (int pass = 0; pass < 2; pass++) {
+    run<16, 0>(nthreads, ddb, 12, 2, dout, r0, reps, ghz, nsm);
+    run<16, 2>(nthreads, ddb, 12, 2, dout, r2, reps, ghz, nsm);
+    run<16, 4>(nthreads, ddb, 12, 2, dout, r4, reps, ghz, nsm);
+    run<16, 5>(nthreads, ddb, 12, 2, dout, r5, reps, ghz, nsm);
+    run<16, 6>(nthreads, ddb, 12, 2, dout, r6, reps, ghz, nsm);
+    printf("agree16: %d %d %d %d\n", r0 == r2, r0 == r4, r0 == r5, r0 == r6);
+    run<24, 2>(nthreads, ddb, 12, 2, dout, r2, reps, ghz, nsm);
+    run<24, 5>(nthreads, ddb, 12, 2, dout, r5, reps, ghz, nsm);
+    run<32, 5>(nthreads, ddb, 12, 2, dout, r5, reps, ghz, nsm);
+    run<12, 5>(nthreads, ddb, 12, 2, dout, r5, reps, ghz, nsm);
+    run<8, 5>(nthreads, ddb, 12, 2, dout, r5, reps, ghz, nsm);
+  }
+  return 0;
+}
