@@ -1,0 +1,322 @@
+#!/usr/bin/env python
+"""bench.py — GCUPS of the Smith-Waterman/Gotoh database search (BASELINE.json metric)
+on the SwissProt-shaped 40-query workload (C4 = BASELINE configs[3]) over N B200s.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C4] [--impl ours|reference]
+  (N > 1: launched by torchrun, one process per GPU; the PSS/WA master runs in rank 0)
+
+A step = one sw_search of all queries against the whole database: query profiles (K4),
+inter-task DP (K1), intra-task DP for long sequences (K3), int32 re-run (K2), cross-rank
+merge (NCCL) and top-k (K5).  The packed database is resident in HBM (sw_db_create, timed
+separately); `value` is device-timed (CUDA events inside libsw, max over ranks); `e2e` is
+the same search through the C-ABI with host buffers (queries in, scores + hits out to
+pinned host memory) timed by the host clock around the call.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import seqgen  # noqa: E402
+
+PAPER_CONTEXT = ("paper: 7,190 s on 1 SSE core (Core i7 3.4 GHz) vs 112 s on 4x GTX580 + 4 SSE cores "
+                 "for 40 queries vs SwissProt (PAPER.md P12); derived ~2.7 and ~174 GCUPS")
+DPX_RATE = 64.0   # measured lane-ops/clk/SM of VIMNMX3.S16x2 / VIADDMNMX.S16x2 (tools/dpx_peak)
+DPX_PER_CELL = 2.0  # K1/K3 inner loop: 4 three-input DPX per s16x2 lane word = 2 per cell
+
+
+def env_rank():
+    return (int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")),
+            int(os.environ.get("LOCAL_RANK", "0")))
+
+
+class ClockSampler:
+    """nvidia-smi clocks and throttle reasons sampled during the timed region."""
+    FIELDS = ["clocks.sm", "clocks.max.sm", "clocks_event_reasons.hw_slowdown",
+              "clocks_event_reasons.hw_thermal_slowdown", "clocks_event_reasons.sw_thermal_slowdown",
+              "clocks_event_reasons.sw_power_cap"]
+
+    def __init__(self, gpu: int):
+        self.gpu, self.rows, self.proc = gpu, [], None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.gpu), "--query-gpu=" + ",".join(self.FIELDS),
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except FileNotFoundError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) == len(self.FIELDS):
+                self.rows.append(parts)
+
+    def stop(self):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in self.rows:
+            for k, nm in enumerate(names):
+                if r[2 + k].lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": sorted(reasons),
+                "samples": len(self.rows)}
+
+
+def oracle_rate(w, seconds_target=15.0, seed=99, max_threads=None):
+    """Time the oracle (as it stands) on a bounded random sample of the workload's pairs,
+    on all host cores.  Returns (GCUPS, cores, description)."""
+    import oracle
+    cores = max_threads or os.cpu_count() or 1
+    rng = np.random.default_rng(seed)
+    qlen = w.queries.lengths
+
+    def run(n_db):
+        di = rng.integers(0, w.db.n, n_db)
+        qi = np.repeat(np.arange(w.queries.n, dtype=np.int32), n_db)
+        dd = np.tile(di, w.queries.n).astype(np.int32)
+        cells = int((qlen[qi] * w.db.lengths[dd]).sum())
+        t = time.perf_counter()
+        oracle.pairs(w.queries, w.db, qi, dd, n_threads=cores)
+        return cells, time.perf_counter() - t
+
+    cells, dt = run(20)                       # calibration
+    rate = cells / max(dt, 1e-6)
+    avg_cells_per_db = cells / 20
+    n_db = int(max(20, min(w.db.n, seconds_target * rate / max(avg_cells_per_db, 1))))
+    cells, dt = run(n_db)
+    desc = (f"all {w.queries.n} queries x {n_db} random DB sequences of {w.name} "
+            f"({cells:.3e} cells, {dt:.1f} s, OpenMP dynamic over pairs)")
+    return cells / dt / 1e9, cores, desc, cells, dt
+
+
+def reference_arm(args):
+    rank, world, _ = env_rank()
+    if rank != 0:
+        return 0
+    w = seqgen.make_workload(args.config)
+    per_step = []
+    cores = os.cpu_count()
+    desc = ""
+    for k in range(args.warmup + args.steps):
+        g, cores, desc, cells, dt = oracle_rate(w, seconds_target=args.ref_seconds, seed=1000 + k)
+        if k >= args.warmup:
+            per_step.append((cells, dt))
+    cells = sum(c for c, _ in per_step)
+    sec = sum(t for _, t in per_step)
+    value = cells / sec / 1e9
+    line = {"metric": "GCUPS", "value": value, "unit": "GCUPS", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sec / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int32",
+            "data": "synthetic", "impl": "reference",
+            "config": {"workload": args.config, "doc": w.meta["doc"],
+                       "note": "oracle (plain C Gotoh, OpenMP over pairs) on host cores; each step a "
+                               "bounded random sample of the workload's pairs"},
+            "cpu_baseline": {"value": value, "unit": "GCUPS", "cores": cores, "kind": "oracle",
+                             "sample": desc},
+            "e2e": {"value": value, "unit": "GCUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+            "context": PAPER_CONTEXT}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def load_traffic():
+    p = os.path.join(ROOT, "profiles", "ncu_k1_summary.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d.get("dram_bytes_per_launch"), d
+    except Exception:
+        return None, None
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C4")
+    ap.add_argument("--n-db", type=int, default=None, help="scale the DB down (debug only)")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--ref-seconds", type=float, default=12.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--policy", default="pss")
+    ap.add_argument("--no-wa", action="store_true")
+    ap.add_argument("--straggler-mask", type=int, default=0)
+    ap.add_argument("--streams", type=int, default=3)
+    ap.add_argument("--unit-cells", type=int, default=0)
+    ap.add_argument("--top-k", type=int, default=10)
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return reference_arm(args)
+
+    import torch
+    from paper_conf_ipps_mendoncam13_b200 import Database
+    from paper_conf_ipps_mendoncam13_b200 import dist as swdist
+
+    rank, world, local = env_rank()
+    torch.cuda.set_device(local)
+    if world > 1:
+        import torch.distributed as tdist
+        tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    t = time.perf_counter()
+    w = seqgen.make_workload(args.config, n_db=args.n_db)
+    gen_s = time.perf_counter() - t
+    t = time.perf_counter()
+    D = Database(w.db, devices=[local])
+    db_create_s = time.perf_counter() - t
+    cells = int(w.meta["cells"])
+    kw = dict(policy=args.policy, workload_adjust=not args.no_wa, streams=args.streams,
+              target_unit_cells=args.unit_cells, straggler_mask=args.straggler_mask)
+
+    def step():
+        if world > 1:
+            tdist.barrier()
+            torch.cuda.synchronize()
+            _, _, _, st = swdist.search(D, w.queries, rank, world, top_k=args.top_k, **kw)
+            torch.cuda.synchronize()   # NCCL merge + top-k ran on torch's stream after libsw
+            return st["seconds_device"], st
+        r = D.search(w.queries, top_k=args.top_k, outputs_on_device=True, **kw)
+        return r.stats["seconds_device"], r.stats
+
+    for _ in range(args.warmup):
+        step()
+    if world > 1:
+        tdist.barrier()
+    torch.cuda.synchronize()
+    sampler = ClockSampler(local)
+    sampler.start()
+    time.sleep(0.3)
+    dev_s, launches, wall0 = 0.0, 0, time.perf_counter()
+    stats = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        sec, st = step()
+        t1 = time.perf_counter()
+        if world > 1:
+            # merge time is part of the step: use the host span of the step as the upper
+            # bound on top of the device time of libsw (both measured on this rank)
+            sec = max(sec, t1 - t0)
+        dev_s += sec
+        launches += st["kernel_launches"]
+        stats.append(st)
+    wall = time.perf_counter() - wall0
+    clocks = sampler.stop()
+    if world > 1:
+        tt = torch.tensor([dev_s], device="cuda", dtype=torch.float64)
+        tdist.all_reduce(tt, op=tdist.ReduceOp.MAX)
+        dev_s = float(tt.item())
+    value = cells * args.steps / dev_s / 1e9
+    ms = 1e3 * dev_s / args.steps
+
+    # ---- e2e: host buffers through the C-ABI (queries H2D, scores + hits D2H, pinned)
+    e2e = None
+    nq, nd = w.queries.n, w.db.n
+    h2d = int(w.queries.total + 8 * (nq + 1) + 576)
+    d2h = int(4 * nq * nd + 8 * nq * args.top_k)
+    if args.e2e_steps > 0:
+        pin_s = torch.empty((nq, nd), dtype=torch.int32, pin_memory=True)
+        pin_h = torch.empty((nq, args.top_k, 2), dtype=torch.int32, pin_memory=True)
+        tsum = 0.0
+        for k in range(args.e2e_steps + 1):
+            if world > 1:
+                tdist.barrier()
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            if world > 1:
+                sc, hs, hi, _ = swdist.search(D, w.queries, rank, world, top_k=args.top_k, **kw)
+                if rank == 0:
+                    pin_s.copy_(sc, non_blocking=True)
+                    pin_h[..., 0].copy_(hs)
+                    pin_h[..., 1].copy_(hi)
+                torch.cuda.synchronize()
+            else:
+                D.search(w.queries, top_k=args.top_k, out_scores=pin_s, out_hits=pin_h, **kw)
+            dt = time.perf_counter() - t0
+            if k > 0:
+                tsum += dt
+        if world > 1:
+            tt = torch.tensor([tsum], device="cuda", dtype=torch.float64)
+            tdist.all_reduce(tt, op=tdist.ReduceOp.MAX)
+            tsum = float(tt.item())
+        e2e = {"value": cells * args.e2e_steps / tsum / 1e9, "unit": "GCUPS",
+               "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+               "note": "sw_search with host queries and pinned host outputs (scores + hits), host "
+                       "clock around the call; packed DB resident (created once, db_create_s)"}
+
+    # ---- roofline of the DP kernels (integer/DPX pipe bound)
+    last = stats[-1]
+    sm_mhz = clocks["sm_mhz"] or 1965.0
+    nsm = torch.cuda.get_device_properties(local).multi_processor_count
+    peak = nsm * sm_mhz * 1e6 * DPX_RATE / DPX_PER_CELL / 1e9
+    peak_max = nsm * 1965e6 * DPX_RATE / DPX_PER_CELL / 1e9
+    per_gpu = value / world
+    traffic, _ = load_traffic()
+    roofline = {"bound": "alu", "achieved": per_gpu, "peak": peak, "unit": "GCUPS",
+                "frac": per_gpu / peak, "traffic": traffic,
+                "peak_at_max_clock": peak_max, "frac_at_max_clock": per_gpu / peak_max,
+                "kernel": "k1_kernel (inter-task) + k3_kernel (intra-task): whole step per GPU",
+                "derivation": f"{nsm} SMs x {sm_mhz:.0f} MHz (median under load) x {DPX_RATE:.0f} "
+                              f"DPX lane-ops/clk/SM (measured) / {DPX_PER_CELL:.0f} DPX per cell",
+                "k1_cells_share": last["cells_k1"] / max(1, last["cells_k1"] + last["cells_k3"])}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        g, cores, desc, _, _ = oracle_rate(w, seconds_target=args.cpu_seconds)
+        cpu = {"value": g, "unit": "GCUPS", "cores": cores, "kind": "oracle", "sample": desc}
+
+    if rank == 0:
+        line = {"metric": "GCUPS", "value": value, "unit": "GCUPS", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+                "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+                "dtype": "s16x2 (int32 re-run)", "data": "synthetic",
+                "config": {"workload": args.config, "doc": w.meta["doc"], "n_db": nd,
+                           "n_queries": nq, "db_residues": int(w.db.total),
+                           "cells_per_step": cells, "policy": args.policy,
+                           "workload_adjust": not args.no_wa, "streams_per_gpu": args.streams,
+                           "top_k": args.top_k, "l2": "inputs larger than L2 (packed DB "
+                           f"{w.db.total / 1e6:.0f} MB > 126 MB); no flush",
+                           "units_per_step": last["n_units"],
+                           "overflow_pairs": last["n_overflow_pairs"],
+                           "wa_grants": last["n_wa_grants"],
+                           "db_create_s": db_create_s, "generate_s": gen_s,
+                           "wall_s_timed": wall, "parallelism": f"dp{world} (PSS/WA units)"},
+                "gpu_launches": launches, "clocks": clocks, "e2e": e2e, "roofline": roofline,
+                "cpu_baseline": cpu, "context": PAPER_CONTEXT}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        tdist.barrier()
+        tdist.destroy_process_group()
+    D.close()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())
