@@ -258,7 +258,11 @@ struct DevSearch {
   DBuf<int32_t> ovf_count;
   DBuf<uint2> k3_border;   // [streams][max_k3_seqs][max_len]
   DBuf<int32_t> k2_border;
-  int32_t *abort_h = nullptr, *abort_d = nullptr;
+  DBuf<int32_t> abort_dev;      // per-unit WA cancellation flags (device memory)
+  int32_t *abort_d = nullptr;
+  int32_t *one_h = nullptr;      // pinned constant 1, source of the cancellation copies
+  cudaStream_t cancel_st = nullptr;
+  std::vector<char> cancelled;
   cudaEvent_t ev_start = nullptr, ev_end = nullptr;
   std::vector<cudaEvent_t> u_start, u_end;  // per stream
   int launches = 0;
@@ -269,7 +273,8 @@ struct DevSearch {
   int32_t n_ovf = 0;
   ~DevSearch() {
     if (D) cudaSetDevice(D->id);
-    if (abort_h) cudaFreeHost(abort_h);
+    if (one_h) cudaFreeHost(one_h);
+    if (cancel_st) cudaStreamDestroy(cancel_st);
     if (ev_start) cudaEventDestroy(ev_start);
     if (ev_end) cudaEventDestroy(ev_end);
     for (auto e : u_start) cudaEventDestroy(e);
@@ -483,9 +488,14 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       X.ovf_count.alloc(D.id, 1);
       const size_t k3b = (size_t)depth * std::max(P.max_k3_seqs, 1) * std::max<int64_t>(P.max_len, 1);
       if (P.n_long_seqs > 0) X.k3_border.alloc(D.id, k3b);
-      CK(cudaHostAlloc((void **)&X.abort_h, sizeof(int32_t) * std::max<size_t>(P.units.size(), 1), cudaHostAllocMapped));
-      std::memset(X.abort_h, 0, sizeof(int32_t) * std::max<size_t>(P.units.size(), 1));
-      CK(cudaHostGetDevicePointer((void **)&X.abort_d, X.abort_h, 0));
+      const size_t nu = std::max<size_t>(P.units.size(), 1);
+      X.abort_dev.alloc(D.id, nu);
+      CK(cudaMemset(X.abort_dev.p, 0, sizeof(int32_t) * nu));
+      X.abort_d = X.abort_dev.p;
+      X.cancelled.assign(nu, 0);
+      CK(cudaHostAlloc((void **)&X.one_h, sizeof(int32_t), cudaHostAllocDefault));
+      *X.one_h = 1;
+      CK(cudaStreamCreateWithFlags(&X.cancel_st, cudaStreamNonBlocking));
       CK(cudaEventCreate(&X.ev_start));
       CK(cudaEventCreate(&X.ev_end));
       X.u_start.resize(depth);
@@ -618,8 +628,11 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
           }
           // cancel in-flight replicas whose task finished elsewhere (WA loser)
           for (int k = 0; k < depth; k++)
-            if (inflight[k] >= 0 && !X.abort_h[inflight[k]] && sfin(inflight[k]))
-              X.abort_h[inflight[k]] = 1;
+            if (inflight[k] >= 0 && !X.cancelled[inflight[k]] && sfin(inflight[k])) {
+              X.cancelled[inflight[k]] = 1;
+              CK(cudaMemcpyAsync(X.abort_d + inflight[k], X.one_h, sizeof(int32_t),
+                                 cudaMemcpyHostToDevice, X.cancel_st));
+            }
           // launch pending units on free streams
           for (int k = 0; k < depth && !pending.empty(); k++) {
             if (inflight[k] >= 0) continue;

@@ -21,11 +21,27 @@
 #include <cuda_runtime.h>
 #include <cstdint>
 #include <cstdio>
+#include <cstdlib>
 #include "sw_internal.h"
 
 namespace sw {
 
 __device__ __forceinline__ uint32_t pk2(int v) { return ((uint32_t)(v & 0xffff)) * 0x10001u; }
+__device__ __forceinline__ void cp_async8(void *smem_dst, const void *gsrc) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(smem_dst);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(d), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit_wait() {
+  asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+}
+// WA cancellation flag (device memory, set by the host with an async copy): read once by
+// thread 0 and broadcast, so a block start costs one L2 read
+__device__ __forceinline__ bool block_aborted(const volatile int32_t *flag) {
+  __shared__ int ab;
+  if (threadIdx.x == 0) ab = flag ? *flag : 0;
+  __syncthreads();
+  return ab != 0;
+}
 __device__ __forceinline__ uint32_t smid() {
   uint32_t r;
   asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
@@ -86,8 +102,8 @@ struct Cell {
 // and, for the last warp, to warp 0 of the next band through a global border row held
 // in a per-SM slot.  One __syncthreads per step.
 // ------------------------------------------------------------------------------------
-template <int K, int W, int T>
-__global__ void __launch_bounds__(W * 32, 3) k1_kernel(const K1Args a) {
+template <int K, int W, int T, int MINB>
+__global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   constexpr int BAND = W * K;
   constexpr int S = BAND + 1;  // odd stride: lanes reading one row with different codes hit
                                // different banks
@@ -95,9 +111,10 @@ __global__ void __launch_bounds__(W * 32, 3) k1_kernel(const K1Args a) {
   uint32_t *prof_s = smem;                                       // [2][kNCodes][S]
   uint2 *hand = reinterpret_cast<uint2 *>(smem + 2 * kNCodes * S);  // [W][2][T][32]
   uint32_t *red = reinterpret_cast<uint32_t *>(hand + W * 2 * T * 32);  // [W][32]
+  uint2 *bsm = reinterpret_cast<uint2 *>(red + W * 32);                  // [2][T][32]
   __shared__ int slot_s;
 
-  if (a.abort_flag && *a.abort_flag) return;  // WA: this replica lost the race
+  if (block_aborted(a.abort_flag)) return;  // WA: this replica lost the race
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const GroupInfo G = a.groups[a.g0 + blockIdx.x];
   const QueryPair P = a.pairs[a.pair];
@@ -133,9 +150,13 @@ __global__ void __launch_bounds__(W * 32, 3) k1_kernel(const K1Args a) {
 
   uint32_t H[K], E[K];
   uint32_t best = koff, hprev_top = koff;
-  uint4 r4 = make_uint4(0, 0, 0, 0);
   int band = 0, tile = 0;
   const uint4 *wp = a.packed + G.word_off + lane;
+  const int nwords = G.ncols / kWordCols;
+  // residue words: current and the next one (prefetched a word ahead)
+  uint4 r4 = wp[0];
+  uint4 r4n = wp[(size_t)(nwords > 1 ? 1 : 0) * 32];
+  int wnext = nwords > 1 ? 1 : 0;
   const int steps = total + W - 1;
   for (int s = 0; s < steps; s++) {
     // band b+2 reuses the profile slot of band b once every warp has left band b
@@ -153,7 +174,27 @@ __global__ void __launch_bounds__(W * 32, 3) k1_kernel(const K1Args a) {
         for (int i = 0; i < K; i++) { H[i] = koff; E[i] = koff; }
         hprev_top = koff;
       }
-      if ((tile & (kWordCols / T - 1)) == 0) r4 = wp[(size_t)(tile * T / kWordCols) * 32];
+      if (tile != 0 && (tile & (kWordCols / T - 1)) == 0) {
+        r4 = r4n;
+        wnext = (wnext + 1 == nwords) ? 0 : wnext + 1;
+        r4n = wp[(size_t)wnext * 32];
+      } else if (tile == 0 && band > 0) {
+        // new band: restart at word 0 (prefetched at the end of the previous band)
+        r4 = r4n;
+        wnext = nwords > 1 ? 1 : 0;
+        r4n = wp[(size_t)wnext * 32];
+      }
+      // warp 0: copy the border row of its next element (band2, tile2) into shared memory
+      // with cp.async, one step ahead (warp W-1 wrote it >= 1 step earlier: nt >= W+1)
+      if (warp == 0) {
+        const int tile2 = tile + 1 == nt ? 0 : tile + 1;
+        const int band2 = tile + 1 == nt ? band + 1 : band;
+        if (band2 >= 1 && band2 < nb) {
+#pragma unroll
+          for (int jj = 0; jj < T; jj++)
+            cp_async8(&bsm[(((s + 1) & 1) * T + jj) * 32 + lane], &border[(size_t)(tile2 * T + jj) * 32 + lane]);
+        }
+      }
       const uint32_t *pr_base = prof_s + (band & 1) * kNCodes * S + warp * K;
       const uint32_t wsel = (tile * T / 4) & 3;  // which 32-bit word of r4 holds this tile
       const uint32_t word = wsel == 0 ? r4.x : wsel == 1 ? r4.y : wsel == 2 ? r4.z : r4.w;
@@ -164,7 +205,7 @@ __global__ void __launch_bounds__(W * 32, 3) k1_kernel(const K1Args a) {
         uint32_t ht, ft;
         if (warp == 0) {
           if (band == 0) { ht = koff; ft = koff; }
-          else { const uint2 v = border[(size_t)col * 32 + lane]; ht = v.x; ft = v.y; }
+          else { const uint2 v = bsm[((s & 1) * T + jj) * 32 + lane]; ht = v.x; ft = v.y; }
         } else {
           const uint2 v = hand[(((warp - 1) * 2 + ((s - 1) & 1)) * T + jj) * 32 + lane];
           ht = v.x; ft = v.y;
@@ -179,6 +220,7 @@ __global__ void __launch_bounds__(W * 32, 3) k1_kernel(const K1Args a) {
         else if (band < nb - 1) border[(size_t)col * 32 + lane] = out;
       }
       if (++tile == nt) { tile = 0; band++; }
+      if (warp == 0) cp_async_commit_wait();
     }
     __syncthreads();
   }
@@ -214,45 +256,60 @@ __global__ void __launch_bounds__(W * 32, 3) k1_kernel(const K1Args a) {
 static size_t k1_smem() {
   constexpr int S = kK1Band + 1;
   return sizeof(uint32_t) * 2 * kNCodes * S + sizeof(uint2) * kK1Warps * 2 * kK1Tile * 32 +
-         sizeof(uint32_t) * kK1Warps * 32;
+         sizeof(uint32_t) * kK1Warps * 32 + sizeof(uint2) * 2 * kK1Tile * 32;
 }
 
-int k1_blocks_per_sm() {
+// K1 occupancy variant: 3 blocks/SM (<= 85 registers) or 2 blocks/SM (<= 128 registers);
+// SW_K1_MINB overrides the default (tuning)
+static int k1_minb() {
   static int v = -1;
   if (v < 0) {
-    auto fn = k1_kernel<kK1Rows, kK1Warps, kK1Tile>;
-    cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem());
-    int n = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, kK1Warps * 32, k1_smem()) !=
-        cudaSuccess)
-      n = 8;
-    v = n > 0 ? n : 1;
+    const char *e = getenv("SW_K1_MINB");
+    v = (e && atoi(e) == 2) ? 2 : 3;
   }
   return v;
 }
+template <int MINB>
+static int k1_occ() {
+  auto fn = k1_kernel<kK1Rows, kK1Warps, kK1Tile, MINB>;
+  cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem());
+  int n = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, kK1Warps * 32, k1_smem()) != cudaSuccess) n = 8;
+  return n > 0 ? n : 1;
+}
+int k1_blocks_per_sm() {
+  static int v = -1;
+  if (v < 0) v = k1_minb() == 2 ? k1_occ<2>() : k1_occ<3>();
+  return v;
+}
 
-void launch_k1(const K1Args &a, int n_groups, int, int, cudaStream_t st, int sm_cap) {
+void launch_k1(const K1Args &a, int n_groups, int, int, cudaStream_t st, int) {
   if (n_groups <= 0) return;
-  auto fn = k1_kernel<kK1Rows, kK1Warps, kK1Tile>;
-  (void)sm_cap;
-  fn<<<n_groups, kK1Warps * 32, k1_smem(), st>>>(a);
+  k1_blocks_per_sm();  // sets the smem attribute once
+  if (k1_minb() == 2)
+    k1_kernel<kK1Rows, kK1Warps, kK1Tile, 2><<<n_groups, kK1Warps * 32, k1_smem(), st>>>(a);
+  else
+    k1_kernel<kK1Rows, kK1Warps, kK1Tile, 3><<<n_groups, kK1Warps * 32, k1_smem(), st>>>(a);
 }
 
 // ------------------------------------------------------------------------------------
 // K3: intra-task kernel for long DB sequences (P14 §II.B fine-grained approach, Fig. 3a:
 // "the calculations that can be done in parallel evolve as waves on diagonals").  One
 // warp per (query pair, long sequence); lane l owns rows [l*K, (l+1)*K) of each chunk of
-// 32*K rows; at step t lane l updates column t - l and receives the row above (H, F) and
-// the residue code from lane l-1 by __shfl_up_sync; lane 31 writes the chunk's bottom
-// row to a global border read by lane 0 in the next chunk.  Block = kK3Warps sequences
-// sharing the chunk profile in shared memory laid out [code][row-in-lane][lane] (bank =
-// lane: conflict-free with 32 different codes).
+// 32*K query rows.  At step t lane l updates the T-column tile t - l (T columns give the
+// lane T independent dependency chains); it receives the bottom row (H, F) of that tile
+// and its 4 residue codes from lane l-1 by __shfl_up_sync, lane 0 takes them from the
+// previous chunk's border row (prefetched one step ahead) and the packed database, and
+// lane 31 writes the chunk's bottom row to the border.  Block = kK3Warps sequences that
+// share the chunk profile in shared memory laid out [code][row-in-lane][lane] (bank =
+// lane: conflict-free although every lane reads a different code).
 // ------------------------------------------------------------------------------------
-template <int K>
+template <int K, int T>
 __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
+  static_assert(T == 4, "one 32-bit word of packed residues per tile");
   constexpr int CH = 32 * K;
   extern __shared__ __align__(16) uint32_t smem[];  // [kNCodes][K][32]
-  if (a.abort_flag && *a.abort_flag) return;
+  if (block_aborted(a.abort_flag)) return;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const QueryPair P = a.pairs[a.pair];
   const int rows = P.la > P.lb ? P.la : P.lb;
@@ -261,11 +318,13 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
   const bool valid = s < a.l1;
   const int len = valid ? a.sorted_len[s] : 0;
   const GroupInfo G = a.groups[valid ? s / kGroup : 0];
-  const uint8_t *bytes = reinterpret_cast<const uint8_t *>(a.packed);
   const int gl = s % kGroup;
+  const uint4 *wp = a.packed + G.word_off + gl;
   uint2 *border = a.border + (size_t)(blockIdx.x * kK3Warps + warp) * a.border_stride;
   const uint32_t koff = pk2(kOff), na = a.na, nbeta = a.nb;
+  const uint32_t padw = 0x01010101u * kPadCode;
   const int32_t *gprof = a.prof + P.prof_off;
+  const int ntile = (len + T - 1) / T;   // columns up to ntile*T <= G.ncols carry pad codes
   uint32_t best = koff;
 
   for (int ch = 0; ch < nch; ch++) {
@@ -280,33 +339,65 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
     uint32_t H[K], E[K];
 #pragma unroll
     for (int i = 0; i < K; i++) { H[i] = koff; E[i] = koff; }
-    uint32_t hprev_top = koff, out_h = koff, out_f = koff, out_c = kPadCode;
-    uint4 wcur = make_uint4(0, 0, 0, 0);
-    const int steps = len + 31;
+    uint32_t hprev_top = koff, out_c = padw;
+    uint32_t out_h[T], out_f[T];
+    uint2 bn[T];
+#pragma unroll
+    for (int jj = 0; jj < T; jj++) { out_h[jj] = koff; out_f[jj] = koff; bn[jj] = make_uint2(koff, koff); }
+    // lane 0's residue words (current, next) and border prefetch for tile 0
+    uint4 wcur = make_uint4(padw, padw, padw, padw), wnx = wcur;
+    if (lane == 0) {
+      wcur = wp[0];
+      if (ntile > 4) wnx = wp[kGroup];
+      if (ch > 0)
+#pragma unroll
+        for (int jj = 0; jj < T; jj++) bn[jj] = border[jj];
+    }
+    const int steps = ntile + 31;
     for (int t = 0; t < steps; t++) {
-      uint32_t in_h = __shfl_up_sync(0xffffffffu, out_h, 1);
-      uint32_t in_f = __shfl_up_sync(0xffffffffu, out_f, 1);
+      uint32_t in_h[T], in_f[T];
+#pragma unroll
+      for (int jj = 0; jj < T; jj++) {
+        in_h[jj] = __shfl_up_sync(0xffffffffu, out_h[jj], 1);
+        in_f[jj] = __shfl_up_sync(0xffffffffu, out_f[jj], 1);
+      }
       uint32_t in_c = __shfl_up_sync(0xffffffffu, out_c, 1);
-      if (lane == 0) {
-        if (t < len) {
-          if ((t & 15) == 0)
-            wcur = *reinterpret_cast<const uint4 *>(bytes + (G.word_off + (int64_t)(t >> 4) * kGroup + gl) * 16);
-          const uint32_t wsel = (t >> 2) & 3;
-          const uint32_t word = wsel == 0 ? wcur.x : wsel == 1 ? wcur.y : wsel == 2 ? wcur.z : wcur.w;
-          in_c = (word >> (8 * (t & 3))) & 0xff;
-          if (ch == 0) { in_h = koff; in_f = koff; }
-          else { const uint2 v = border[t]; in_h = v.x; in_f = v.y; }
+      if (lane == 0 && t < ntile) {
+        const int q = t & 3;
+        in_c = q == 0 ? wcur.x : q == 1 ? wcur.y : q == 2 ? wcur.z : wcur.w;
+        if (ch == 0) {
+#pragma unroll
+          for (int jj = 0; jj < T; jj++) { in_h[jj] = koff; in_f[jj] = koff; }
+        } else {
+#pragma unroll
+          for (int jj = 0; jj < T; jj++) { in_h[jj] = bn[jj].x; in_f[jj] = bn[jj].y; }
+          if (t + 1 < ntile)
+#pragma unroll
+            for (int jj = 0; jj < T; jj++) bn[jj] = border[(t + 1) * T + jj];
+        }
+        if (q == 3) {   // move to the next 16-column word, prefetch the one after
+          wcur = wnx;
+          const int nw = (t >> 2) + 2;
+          if (nw * 4 < ntile) wnx = wp[(size_t)nw * kGroup];
         }
       }
-      const int col = t - lane;
-      if (col >= 0 && col < len) {
-        uint32_t hd = hprev_top, f = in_f;
-        hprev_top = in_h;
-        const uint32_t *pr = smem + in_c * K * 32 + lane;
+      const int tile = t - lane;
+      if (tile >= 0 && tile < ntile) {
 #pragma unroll
-        for (int i = 0; i < K; i++) Cell::row(pr[i * 32], hd, H[i], E[i], f, best, na, nbeta, koff);
-        out_h = H[K - 1]; out_f = f; out_c = in_c;
-        if (lane == 31 && ch < nch - 1) border[col] = make_uint2(out_h, out_f);
+        for (int jj = 0; jj < T; jj++) {
+          const uint32_t c = (in_c >> (8 * jj)) & 0xffu;
+          uint32_t hd = hprev_top, f = in_f[jj];
+          hprev_top = in_h[jj];
+          const uint32_t *pr = smem + c * K * 32 + lane;
+#pragma unroll
+          for (int i = 0; i < K; i++) Cell::row(pr[i * 32], hd, H[i], E[i], f, best, na, nbeta, koff);
+          out_h[jj] = H[K - 1];
+          out_f[jj] = f;
+        }
+        out_c = in_c;
+        if (lane == 31 && ch < nch - 1)
+#pragma unroll
+          for (int jj = 0; jj < T; jj++) border[tile * T + jj] = make_uint2(out_h[jj], out_f[jj]);
       }
     }
   }
@@ -337,7 +428,7 @@ void launch_k3(const K3Args &a, int, cudaStream_t st) {
   const int n = a.l1 - a.l0;
   if (n <= 0) return;
   const size_t smem = sizeof(uint32_t) * kNCodes * kK3Rows * 32;
-  auto fn = k3_kernel<kK3Rows>;
+  auto fn = k3_kernel<kK3Rows, 4>;
   static bool attr = false;
   if (!attr) { cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); attr = true; }
   fn<<<(n + kK3Warps - 1) / kK3Warps, kK3Warps * 32, smem, st>>>(a);

@@ -44,7 +44,8 @@ struct GroupInfo {       // one packing group of up to 32 length-sorted sequence
   int32_t count;         // real sequences in the group (<= 32)
   int32_t pad_;
 };
-constexpr int kMinCols = 32;       // groups padded to >= (W-1)*T columns (K1 pipeline)
+constexpr int kMinCols = 48;       // groups padded to >= (W+1)*T columns: the K1 pipeline
+                                   // prefetches warp 0's border one step ahead
 
 // ---- a unit of work (one task of the paper's scheduler) -----------------------------
 enum UnitKind : int32_t { kUnitInter = 0, kUnitIntra = 1 };

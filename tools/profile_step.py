@@ -1,0 +1,30 @@
+"""One (or more) sw_search steps on a config, for ncu launch lists / captures.
+  python tools/profile_step.py --config C4 [--steps 1] [--n-db N]"""
+import argparse
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import seqgen  # noqa: E402
+from paper_conf_ipps_mendoncam13_b200 import Database  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--config", default="C4")
+ap.add_argument("--steps", type=int, default=1)
+ap.add_argument("--n-db", type=int, default=None)
+ap.add_argument("--n-queries", type=int, default=None)
+ap.add_argument("--streams", type=int, default=3)
+ap.add_argument("--long-threshold", type=int, default=0)
+args = ap.parse_args()
+w = seqgen.make_workload(args.config, n_db=args.n_db, n_queries=args.n_queries)
+D = Database(w.db)
+for s in range(args.steps):
+    t = time.perf_counter()
+    r = D.search(w.queries, top_k=10, outputs_on_device=True, streams=args.streams,
+                 long_threshold=args.long_threshold)
+    st = r.stats
+    print(f"step {s}: {st['gcups']:.1f} GCUPS dev {st['seconds_device']:.3f}s wall {time.perf_counter()-t:.3f}s "
+          f"k1 {st['kernel_seconds_k1']:.3f}s/{st['cells_k1']:.3e} k3 {st['kernel_seconds_k3']:.3f}s/{st['cells_k3']:.3e} "
+          f"units {st['n_units']} launches {st['kernel_launches']}", flush=True)
