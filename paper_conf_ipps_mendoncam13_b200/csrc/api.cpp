@@ -212,7 +212,7 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
     for (int32_t s = 0; s < P.n_long_seqs;) {
       int32_t e = s;
       int64_t cells = 0, work = 0;
-      while (e < P.n_long_seqs && (cells < target || e == s || (e - s) % kK3Warps)) {
+      while (e < P.n_long_seqs && (cells < 4 * target || e == s || (e - s) % kK3Warps)) {
         cells += rows_eff * db.sorted_len[e];
         work += (int64_t)qp.rows_padded * db.sorted_len[e];
         e++;
@@ -238,9 +238,12 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
   // drop empty units (e.g. all-empty queries still produce valid zero scores: keep them
   // so that every pair gets written, but they must have cells > 0 for the scheduler)
   for (auto &u : P.units) u.cells = std::max<int64_t>(u.cells, 1);
-  // LPT: largest work first
-  std::stable_sort(P.units.begin(), P.units.end(),
-                   [](const Unit &a, const Unit &b) { return a.work > b.work; });
+  // LPT by expected duration: intra-task (long-sequence) units first -- each warp walks a
+  // whole long pair, so they have the longest latency -- then inter-task units by work
+  std::stable_sort(P.units.begin(), P.units.end(), [](const Unit &a, const Unit &b) {
+    if (a.kind != b.kind) return a.kind == kUnitIntra;
+    return a.work > b.work;
+  });
   return P;
 }
 

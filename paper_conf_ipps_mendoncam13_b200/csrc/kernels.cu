@@ -112,6 +112,7 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   uint2 *hand = reinterpret_cast<uint2 *>(smem + 2 * kNCodes * S);  // [W][2][T][32]
   uint32_t *red = reinterpret_cast<uint32_t *>(hand + W * 2 * T * 32);  // [W][32]
   uint2 *bsm = reinterpret_cast<uint2 *>(red + W * 32);                  // [2][T][32]
+  uint2 *kin = bsm + 2 * T * 32;                                         // [T][32] = (kOff, kOff)
   __shared__ int slot_s;
 
   if (block_aborted(a.abort_flag)) return;  // WA: this replica lost the race
@@ -145,6 +146,7 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   };
   load_band(0, 0);
   if (nb > 1) load_band(1, 1);
+  for (int k = threadIdx.x; k < T * 32; k += W * 32) kin[k] = make_uint2(koff, koff);
   __syncthreads();
   if (nb > 1) border = a.border + (size_t)slot_s * a.border_slot_cols * 32;
 
@@ -153,6 +155,7 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   int band = 0, tile = 0;
   const uint4 *wp = a.packed + G.word_off + lane;
   const int nwords = G.ncols / kWordCols;
+  constexpr int TPW = kWordCols / T;   // tiles per 16-column residue word
   // residue words: current and the next one (prefetched a word ahead)
   uint4 r4 = wp[0];
   uint4 r4n = wp[(size_t)(nwords > 1 ? 1 : 0) * 32];
@@ -174,7 +177,7 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
         for (int i = 0; i < K; i++) { H[i] = koff; E[i] = koff; }
         hprev_top = koff;
       }
-      if (tile != 0 && (tile & (kWordCols / T - 1)) == 0) {
+      if (tile != 0 && (tile % TPW) == 0) {
         r4 = r4n;
         wnext = (wnext + 1 == nwords) ? 0 : wnext + 1;
         r4n = wp[(size_t)wnext * 32];
@@ -195,29 +198,33 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
             cp_async8(&bsm[(((s + 1) & 1) * T + jj) * 32 + lane], &border[(size_t)(tile2 * T + jj) * 32 + lane]);
         }
       }
+      // top input of this tile (all in shared memory, so the column loop is branch-free):
+      // warp 0 <- constant row (band 0) or the cp.async'd border; warp w <- warp w-1
+      const uint2 *inp = warp == 0 ? (band == 0 ? kin : bsm + (s & 1) * T * 32)
+                                   : hand + ((warp - 1) * 2 + ((s - 1) & 1)) * T * 32;
+      uint2 *outp = hand + (warp * 2 + (s & 1)) * T * 32;
       const uint32_t *pr_base = prof_s + (band & 1) * kNCodes * S + warp * K;
-      const uint32_t wsel = (tile * T / 4) & 3;  // which 32-bit word of r4 holds this tile
-      const uint32_t word = wsel == 0 ? r4.x : wsel == 1 ? r4.y : wsel == 2 ? r4.z : r4.w;
+      const int wq = (tile % TPW) * (T / 4);   // first 32-bit word of r4 used by this tile
+      uint32_t wds[T / 4];
+#pragma unroll
+      for (int q = 0; q < T / 4; q++) {
+        const int k = wq + q;
+        wds[q] = k == 0 ? r4.x : k == 1 ? r4.y : k == 2 ? r4.z : r4.w;
+      }
 #pragma unroll
       for (int jj = 0; jj < T; jj++) {
-        const int col = tile * T + jj;
-        const int c = (word >> (8 * jj)) & 0xff;
-        uint32_t ht, ft;
-        if (warp == 0) {
-          if (band == 0) { ht = koff; ft = koff; }
-          else { const uint2 v = bsm[((s & 1) * T + jj) * 32 + lane]; ht = v.x; ft = v.y; }
-        } else {
-          const uint2 v = hand[(((warp - 1) * 2 + ((s - 1) & 1)) * T + jj) * 32 + lane];
-          ht = v.x; ft = v.y;
-        }
-        uint32_t hd = hprev_top, f = ft;
-        hprev_top = ht;
+        const int c = (wds[jj / 4] >> (8 * (jj % 4))) & 0xff;
+        const uint2 v = inp[jj * 32 + lane];
+        uint32_t hd = hprev_top, f = v.y;
+        hprev_top = v.x;
         const uint32_t *pr = pr_base + c * S;
 #pragma unroll
         for (int i = 0; i < K; i++) Cell::row(pr[i], hd, H[i], E[i], f, best, na, nbeta, koff);
-        const uint2 out = make_uint2(H[K - 1], f);
-        if (warp < W - 1) hand[((warp * 2 + (s & 1)) * T + jj) * 32 + lane] = out;
-        else if (band < nb - 1) border[(size_t)col * 32 + lane] = out;
+        outp[jj * 32 + lane] = make_uint2(H[K - 1], f);
+      }
+      if (warp == W - 1 && band < nb - 1) {
+#pragma unroll
+        for (int jj = 0; jj < T; jj++) border[(size_t)(tile * T + jj) * 32 + lane] = outp[jj * 32 + lane];
       }
       if (++tile == nt) { tile = 0; band++; }
       if (warp == 0) cp_async_commit_wait();
@@ -256,16 +263,16 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
 static size_t k1_smem() {
   constexpr int S = kK1Band + 1;
   return sizeof(uint32_t) * 2 * kNCodes * S + sizeof(uint2) * kK1Warps * 2 * kK1Tile * 32 +
-         sizeof(uint32_t) * kK1Warps * 32 + sizeof(uint2) * 2 * kK1Tile * 32;
+         sizeof(uint32_t) * kK1Warps * 32 + sizeof(uint2) * 3 * kK1Tile * 32;
 }
 
-// K1 occupancy variant: 3 blocks/SM (<= 85 registers) or 2 blocks/SM (<= 128 registers);
+// K1 occupancy variant: 2 blocks/SM (<= 128 registers, default) or 3 (<= 85, spills at T=8);
 // SW_K1_MINB overrides the default (tuning)
 static int k1_minb() {
   static int v = -1;
   if (v < 0) {
     const char *e = getenv("SW_K1_MINB");
-    v = (e && atoi(e) == 2) ? 2 : 3;
+    v = (e && atoi(e) == 3) ? 3 : 2;
   }
   return v;
 }

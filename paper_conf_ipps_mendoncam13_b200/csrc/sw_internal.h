@@ -28,7 +28,7 @@ constexpr int kGroup = 32;         // DB sequences per packing group (one per la
 // K1 (inter-task) geometry: W warps per block split each band of W*K rows
 constexpr int kK1Rows = 16;        // K: rows per warp (registers H[K], E[K])
 constexpr int kK1Warps = 8;        // W
-constexpr int kK1Tile = 4;         // T: columns per pipeline step
+constexpr int kK1Tile = 8;         // T: columns per pipeline step
 constexpr int kK1Band = kK1Rows * kK1Warps;
 // K3 (intra-task) geometry: one warp per (query pair, long DB sequence)
 constexpr int kK3Rows = 16;        // rows per lane
@@ -44,7 +44,7 @@ struct GroupInfo {       // one packing group of up to 32 length-sorted sequence
   int32_t count;         // real sequences in the group (<= 32)
   int32_t pad_;
 };
-constexpr int kMinCols = 48;       // groups padded to >= (W+1)*T columns: the K1 pipeline
+constexpr int kMinCols = 80;       // groups padded to >= (W+1)*T columns (rounded to 16): the K1 pipeline
                                    // prefetches warp 0's border one step ahead
 
 // ---- a unit of work (one task of the paper's scheduler) -----------------------------
