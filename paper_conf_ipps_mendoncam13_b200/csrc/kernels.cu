@@ -102,8 +102,9 @@ struct Cell {
 // and, for the last warp, to warp 0 of the next band through a global border row held
 // in a per-SM slot.  One __syncthreads per step.
 // ------------------------------------------------------------------------------------
-template <int K, int W, int T, int MINB>
+template <int K, int W, int T, int MINB, int UQ>
 __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
+  static_assert(T == 4 || T == 8, "tile = one or two 32-bit words of residues");
   constexpr int BAND = W * K;
   constexpr int S = BAND + 1;  // odd stride: lanes reading one row with different codes hit
                                // different banks
@@ -211,16 +212,24 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
         const int k = wq + q;
         wds[q] = k == 0 ? r4.x : k == 1 ? r4.y : k == 2 ? r4.z : r4.w;
       }
+      // rows of the last band past the longer query are padding: skip them (nobody reads
+      // their output; the last band writes no border)
+      const bool live = band < nb - 1 || warp * K < rows - (nb - 1) * BAND;
+#pragma unroll UQ
+      for (int q = 0; q < T / 4 && live; q++) {
+        const uint32_t word = (T == 4 || q == 0) ? wds[0] : wds[T / 4 - 1];
 #pragma unroll
-      for (int jj = 0; jj < T; jj++) {
-        const int c = (wds[jj / 4] >> (8 * (jj % 4))) & 0xff;
-        const uint2 v = inp[jj * 32 + lane];
-        uint32_t hd = hprev_top, f = v.y;
-        hprev_top = v.x;
-        const uint32_t *pr = pr_base + c * S;
+        for (int j4 = 0; j4 < 4; j4++) {
+          const int jj = q * 4 + j4;
+          const int c = (word >> (8 * j4)) & 0xff;
+          const uint2 v = inp[jj * 32 + lane];
+          uint32_t hd = hprev_top, f = v.y;
+          hprev_top = v.x;
+          const uint32_t *pr = pr_base + c * S;
 #pragma unroll
-        for (int i = 0; i < K; i++) Cell::row(pr[i], hd, H[i], E[i], f, best, na, nbeta, koff);
-        outp[jj * 32 + lane] = make_uint2(H[K - 1], f);
+          for (int i = 0; i < K; i++) Cell::row(pr[i], hd, H[i], E[i], f, best, na, nbeta, koff);
+          outp[jj * 32 + lane] = make_uint2(H[K - 1], f);
+        }
       }
       if (warp == W - 1 && band < nb - 1) {
 #pragma unroll
@@ -260,43 +269,50 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   }
 }
 
+template <int T>
 static size_t k1_smem() {
   constexpr int S = kK1Band + 1;
-  return sizeof(uint32_t) * 2 * kNCodes * S + sizeof(uint2) * kK1Warps * 2 * kK1Tile * 32 +
-         sizeof(uint32_t) * kK1Warps * 32 + sizeof(uint2) * 3 * kK1Tile * 32;
+  return sizeof(uint32_t) * 2 * kNCodes * S + sizeof(uint2) * kK1Warps * 2 * T * 32 +
+         sizeof(uint32_t) * kK1Warps * 32 + sizeof(uint2) * 3 * T * 32;
 }
 
-// K1 occupancy variant: 2 blocks/SM (<= 128 registers, default) or 3 (<= 85, spills at T=8);
-// SW_K1_MINB overrides the default (tuning)
-static int k1_minb() {
+// K1 variants (tuning; SW_K1_VARIANT): 0 = T8 / 2 blocks per SM, 1 = T4 / 3 blocks per SM,
+// 2 = T8 / 3 blocks per SM, 3 = T8 / 3 blocks / one 4-column word unrolled at a time (default)
+static int k1_variant() {
   static int v = -1;
   if (v < 0) {
-    const char *e = getenv("SW_K1_MINB");
-    v = (e && atoi(e) == 3) ? 3 : 2;
+    const char *e = getenv("SW_K1_VARIANT");
+    v = e ? atoi(e) : 3;
+    if (v < 0 || v > 3) v = 3;
   }
   return v;
 }
-template <int MINB>
+template <int T, int MINB, int UQ>
 static int k1_occ() {
-  auto fn = k1_kernel<kK1Rows, kK1Warps, kK1Tile, MINB>;
-  cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem());
+  auto fn = k1_kernel<kK1Rows, kK1Warps, T, MINB, UQ>;
+  cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem<T>());
   int n = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, kK1Warps * 32, k1_smem()) != cudaSuccess) n = 8;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, kK1Warps * 32, k1_smem<T>()) != cudaSuccess) n = 8;
   return n > 0 ? n : 1;
 }
 int k1_blocks_per_sm() {
   static int v = -1;
-  if (v < 0) v = k1_minb() == 2 ? k1_occ<2>() : k1_occ<3>();
+  if (v < 0) {
+    const int k = k1_variant();
+    v = k == 1 ? k1_occ<4, 3, 1>() : k == 2 ? k1_occ<8, 3, 2>() : k == 3 ? k1_occ<8, 3, 1>() : k1_occ<8, 2, 2>();
+  }
   return v;
 }
 
 void launch_k1(const K1Args &a, int n_groups, int, int, cudaStream_t st, int) {
   if (n_groups <= 0) return;
   k1_blocks_per_sm();  // sets the smem attribute once
-  if (k1_minb() == 2)
-    k1_kernel<kK1Rows, kK1Warps, kK1Tile, 2><<<n_groups, kK1Warps * 32, k1_smem(), st>>>(a);
-  else
-    k1_kernel<kK1Rows, kK1Warps, kK1Tile, 3><<<n_groups, kK1Warps * 32, k1_smem(), st>>>(a);
+  const int k = k1_variant();
+  const dim3 g(n_groups), b(kK1Warps * 32);
+  if (k == 1) k1_kernel<kK1Rows, kK1Warps, 4, 3, 1><<<g, b, k1_smem<4>(), st>>>(a);
+  else if (k == 2) k1_kernel<kK1Rows, kK1Warps, 8, 3, 2><<<g, b, k1_smem<8>(), st>>>(a);
+  else if (k == 3) k1_kernel<kK1Rows, kK1Warps, 8, 3, 1><<<g, b, k1_smem<8>(), st>>>(a);
+  else k1_kernel<kK1Rows, kK1Warps, 8, 2, 2><<<g, b, k1_smem<8>(), st>>>(a);
 }
 
 // ------------------------------------------------------------------------------------
