@@ -2,7 +2,7 @@
 Mendonca & Melo (IPDPSW 2013).  The compute path is libsw (csrc/, C-ABI in include/sw.h);
 this package is its thin Python binding plus the multi-process (torchrun) glue.
 """
-from .binding import (Database, Scheduler, SearchResult, SwError, lib, EXPORTS,  # noqa: F401
+from .binding import (Database, Scheduler, SearchResult, SwError, lib, EXPORTS, Master, Slave,  # noqa: F401
                       SW_TASK_READY, SW_TASK_EXECUTING, SW_TASK_FINISHED)
 from . import _build  # noqa: F401
 

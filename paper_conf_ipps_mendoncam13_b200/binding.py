@@ -61,7 +61,9 @@ EXPORTS = ["sw_opts_default", "sw_db_create", "sw_db_destroy", "sw_db_residues",
            "sw_sched_create", "sw_sched_destroy", "sw_sched_report", "sw_sched_request",
            "sw_sched_complete", "sw_sched_abandon", "sw_sched_is_finished", "sw_sched_state",
            "sw_sched_committed_by", "sw_sched_replicas", "sw_sched_phi", "sw_sched_rate",
-           "sw_sched_counter", "sw_sched_log_json"]
+           "sw_sched_counter", "sw_sched_log_json", "sw_master_start", "sw_master_stop",
+           "sw_slave_connect", "sw_slave_request", "sw_slave_report", "sw_slave_complete",
+           "sw_slave_abandon", "sw_slave_is_finished", "sw_slave_done"]
 
 
 def lib():
@@ -123,6 +125,21 @@ def lib():
     L.sw_sched_counter.restype = ctypes.c_int64
     L.sw_sched_log_json.argtypes = [ctypes.c_void_p]
     L.sw_sched_log_json.restype = ctypes.c_char_p
+    L.sw_master_start.argtypes = [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, P(ctypes.c_int64),
+                                  ctypes.c_int32, ctypes.c_int32, ctypes.c_int32]
+    L.sw_master_start.restype = ctypes.c_void_p
+    L.sw_master_stop.argtypes = [ctypes.c_void_p]
+    L.sw_slave_connect.argtypes = [ctypes.c_char_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_double]
+    L.sw_slave_connect.restype = ctypes.c_void_p
+    L.sw_slave_request.argtypes = [ctypes.c_void_p, P(ctypes.c_int32), ctypes.c_int32]
+    L.sw_slave_request.restype = ctypes.c_int32
+    L.sw_slave_report.argtypes = [ctypes.c_void_p, ctypes.c_double, ctypes.c_double]
+    L.sw_slave_complete.argtypes = [ctypes.c_void_p, ctypes.c_int32]
+    L.sw_slave_complete.restype = ctypes.c_int32
+    L.sw_slave_abandon.argtypes = [ctypes.c_void_p, ctypes.c_int32]
+    L.sw_slave_is_finished.argtypes = [ctypes.c_void_p, ctypes.c_int32]
+    L.sw_slave_is_finished.restype = ctypes.c_int32
+    L.sw_slave_done.argtypes = [ctypes.c_void_p]
     _lib = L
     return L
 
@@ -313,3 +330,55 @@ class Scheduler:
 
     def log(self):
         return json.loads(lib().sw_sched_log_json(self._h).decode())
+
+
+class Master:
+    """The multi-process master (sw_master_start): serves `world` slaves over TCP."""
+
+    def __init__(self, port, world, unit_cells, policy="pss", wa=True, omega=4):
+        cells = np.ascontiguousarray(unit_cells, dtype=np.int64)
+        h = lib().sw_master_start(port, world, len(cells),
+                                  cells.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)),
+                                  SW_POLICY_SS if policy == "ss" else SW_POLICY_PSS, int(wa), omega)
+        if not h:
+            raise SwError(SW_ENET, lib().sw_last_error().decode())
+        self._h = h
+
+    def stop(self):
+        if self._h:
+            lib().sw_master_stop(self._h)
+            self._h = None
+
+
+class Slave:
+    """A slave's connection to the master (sw_slave_*)."""
+
+    def __init__(self, host, port, rank, timeout=30.0):
+        h = lib().sw_slave_connect(host.encode(), port, rank, timeout)
+        if not h:
+            raise SwError(SW_ENET, lib().sw_last_error().decode())
+        self._h = h
+
+    def request(self, cap=64):
+        buf = (ctypes.c_int32 * cap)()
+        n = lib().sw_slave_request(self._h, buf, cap)
+        if n == -2:
+            raise SwError(SW_ENET, lib().sw_last_error().decode())
+        return None if n < 0 else [buf[i] for i in range(n)]
+
+    def report(self, cells, seconds):
+        lib().sw_slave_report(self._h, float(cells), float(seconds))
+
+    def complete(self, unit) -> bool:
+        return lib().sw_slave_complete(self._h, unit) == 1
+
+    def abandon(self, unit):
+        lib().sw_slave_abandon(self._h, unit)
+
+    def is_finished(self, unit) -> bool:
+        return lib().sw_slave_is_finished(self._h, unit) == 1
+
+    def done(self):
+        if self._h:
+            lib().sw_slave_done(self._h)
+            self._h = None

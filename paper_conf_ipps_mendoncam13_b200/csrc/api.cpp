@@ -31,6 +31,7 @@ namespace sw {
 
 // ---------------------------------------------------------------- errors
 static thread_local std::string g_err;
+void set_last_error(const std::string &m) { g_err = m; }
 #define CK(call)                                                                      \
   do {                                                                                \
     cudaError_t e_ = (call);                                                          \

@@ -213,3 +213,66 @@ void SchedClient::done() {
 }
 
 }  // namespace sw
+
+// ---- C-ABI wrappers (include/sw_sched.h) --------------------------------------------------
+struct sw_master { sw::MasterServer s; };
+struct sw_slave { sw::SchedClient c; };
+
+namespace sw { void set_last_error(const std::string &m); }
+
+extern "C" {
+
+sw_master *sw_master_start(int32_t port, int32_t world, int32_t n_units, const int64_t *unit_cells,
+                           int32_t policy, int32_t wa, int32_t omega) {
+  auto *m = new sw_master();
+  try {
+    m->s.start(port, world, n_units, unit_cells, policy, wa, omega);
+    return m;
+  } catch (const std::exception &e) {
+    sw::set_last_error(e.what());
+    delete m;
+    return nullptr;
+  }
+}
+void sw_master_stop(sw_master *m) {
+  if (!m) return;
+  m->s.stop();
+  delete m;
+}
+sw_slave *sw_slave_connect(const char *host, int32_t port, int32_t rank, double timeout_s) {
+  auto *c = new sw_slave();
+  try {
+    c->c.connect(host, port, rank, timeout_s);
+    return c;
+  } catch (const std::exception &e) {
+    sw::set_last_error(e.what());
+    delete c;
+    return nullptr;
+  }
+}
+static double clk() {
+  using namespace std::chrono;
+  return duration<double>(steady_clock::now().time_since_epoch()).count();
+}
+int32_t sw_slave_request(sw_slave *c, int32_t *out, int32_t cap) {
+  try { return c->c.request(clk(), out, cap); } catch (const std::exception &e) { sw::set_last_error(e.what()); return -2; }
+}
+void sw_slave_report(sw_slave *c, double cells, double seconds) {
+  try { c->c.report(clk(), cells, seconds); } catch (const std::exception &e) { sw::set_last_error(e.what()); }
+}
+int32_t sw_slave_complete(sw_slave *c, int32_t unit) {
+  try { return c->c.complete(unit, clk()); } catch (const std::exception &e) { sw::set_last_error(e.what()); return -2; }
+}
+void sw_slave_abandon(sw_slave *c, int32_t unit) {
+  try { c->c.abandon(unit, clk()); } catch (const std::exception &e) { sw::set_last_error(e.what()); }
+}
+int32_t sw_slave_is_finished(sw_slave *c, int32_t unit) {
+  try { return c->c.is_finished(unit); } catch (const std::exception &e) { sw::set_last_error(e.what()); return -2; }
+}
+void sw_slave_done(sw_slave *c) {
+  if (!c) return;
+  try { c->c.done(); } catch (const std::exception &e) { sw::set_last_error(e.what()); }
+  delete c;
+}
+
+}  // extern "C"
