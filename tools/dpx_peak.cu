@@ -2,6 +2,7 @@
 // instructions the Gotoh recurrence uses on sm_100a. Prints lane-ops per SM-clock.
 // Used to derive the ALU roofline peak in DESIGN.md (R in GCUPS_peak = N_SM f R / I_cell).
 #include <cstdio>
+#include <cuda_fp16.h>
 #include <cstdint>
 #include <vector>
 #include <algorithm>
@@ -22,6 +23,10 @@ __device__ __forceinline__ uint32_t op(uint32_t a, uint32_t b, uint32_t c) {
   if (OP == 8) return (uint32_t)max((int)a, (int)b);  // VIMNMX
   if (OP == 9) return __viaddmax_s16x2_relu(a, b, c);
   if (OP == 10) return __vimax_s16x2_relu(a, b);
+  if (OP == 11) { __half2 x = *reinterpret_cast<__half2*>(&a), y = *reinterpret_cast<__half2*>(&b);
+                  __half2 r = __hmax2(x, y); return *reinterpret_cast<uint32_t*>(&r); }
+  if (OP == 12) return __viaddmax_s16x2(a, b, c) ^ 0;   // placeholder, mixed below
+  if (OP == 13) return (uint32_t)__float_as_uint(fmaxf(__uint_as_float(a), __uint_as_float(b)));
   return a;
 }
 
@@ -49,6 +54,48 @@ __global__ void bench(uint32_t *out, unsigned long long *t, uint32_t seed) {
     unsigned smid; asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
     t[3 * blockIdx.x] = smid; t[3 * blockIdx.x + 1] = t0; t[3 * blockIdx.x + 2] = t1;
   }
+}
+
+__global__ void mixk(uint32_t *out, unsigned long long *t, uint32_t seed, int mode) {
+  uint32_t v[CHAINS], w[CHAINS];
+#pragma unroll
+  for (int c = 0; c < CHAINS; c++) { v[c] = seed * (threadIdx.x + c + 1); w[c] = 0x3c003c00u + c; }
+  uint32_t b = seed ^ 0x00030003u, cc = seed ^ 0x00050005u;
+  __syncthreads();
+  unsigned long long t0 = clock64();
+#pragma unroll 4
+  for (int i = 0; i < ITERS; i++) {
+#pragma unroll
+    for (int c = 0; c < CHAINS; c++) {
+      v[c] = __viaddmax_s16x2(v[c], b, cc);
+      if (mode == 1) { __half2 x = *reinterpret_cast<__half2*>(&w[c]), y = *reinterpret_cast<__half2*>(&v[c]);
+                       __half2 r = __hmax2(x, y); w[c] = *reinterpret_cast<uint32_t*>(&r); }
+      if (mode == 2) w[c] = __vmaxs2(w[c], v[c]);
+      if (mode == 3) w[c] = w[c] + v[c];
+    }
+    b += 0x00010001u;
+  }
+  __syncthreads();
+  unsigned long long t1 = clock64();
+  uint32_t r = 0;
+#pragma unroll
+  for (int c = 0; c < CHAINS; c++) r ^= v[c] ^ w[c];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = r;
+  if (threadIdx.x == 0) { t[2 * blockIdx.x] = t0; t[2 * blockIdx.x + 1] = t1; }
+}
+void runmix(const char *name, int nsm, int mode) {
+  int threads = 256, blocks = nsm * 8;
+  uint32_t *out; unsigned long long *t;
+  cudaMalloc(&out, 4 * blocks * threads); cudaMalloc(&t, 16 * blocks);
+  mixk<<<blocks, threads>>>(out, t, 7, mode);
+  cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+  cudaEventRecord(e0);
+  mixk<<<blocks, threads>>>(out, t, 7, mode);
+  cudaEventRecord(e1); cudaEventSynchronize(e1);
+  float ms; cudaEventElapsedTime(&ms, e0, e1);
+  double dpx = (double)blocks * threads * ITERS * CHAINS;
+  printf("%-26s DPX lane-ops/s = %.1f G  (ms %.3f)\n", name, dpx / (ms * 1e6), ms);
+  cudaFree(out); cudaFree(t);
 }
 
 template <int OP>
@@ -102,5 +149,11 @@ int main() {
   run<8>("imax_s32", nsm);
   run<9>("viaddmax_s16x2_relu", nsm);
   run<10>("vimax_s16x2_relu", nsm);
+  run<11>("hmax2", nsm);
+  run<13>("fmaxf", nsm);
+  runmix("mix dpx only", nsm, 0);
+  runmix("mix dpx + hmax2", nsm, 1);
+  runmix("mix dpx + vmaxs2", nsm, 2);
+  runmix("mix dpx + iadd", nsm, 3);
   return 0;
 }
