@@ -94,6 +94,29 @@ struct Cell {
   }
 };
 
+// G consecutive columns of one lane's K rows, skewed by one row per column so the G
+// dependency chains (row i of column g needs row i of column g-1 and row i-1 of column g)
+// are interleaved explicitly: at step k column g updates row k - g.  Column g starts with
+// diagonal hdc[g] and top F fc[g]; on return out_h[g] / fc[g] hold its bottom-row H and
+// the F passed down.  PS = profile stride between consecutive rows.
+template <int K, int G, int PS>
+__device__ __forceinline__ void dp_tile(const uint32_t *const (&prc)[G], uint32_t (&H)[K],
+                                        uint32_t (&E)[K], uint32_t (&hdc)[G], uint32_t (&fc)[G],
+                                        uint32_t (&out_h)[G], uint32_t &best, uint32_t na, uint32_t nb,
+                                        uint32_t koff) {
+#pragma unroll
+  for (int k = 0; k < K + G - 1; k++) {
+#pragma unroll
+    for (int g = 0; g < G; g++) {
+      const int i = k - g;
+      if (i >= 0 && i < K) {
+        Cell::row(prc[g][i * PS], hdc[g], H[i], E[i], fc[g], best, na, nb, koff);
+        if (i == K - 1) out_h[g] = H[K - 1];
+      }
+    }
+  }
+}
+
 // ------------------------------------------------------------------------------------
 // K1: inter-task kernel.  Block = one packing group of 32 DB sequences (lane = sequence)
 // x W warps; warp w owns rows [w*K, (w+1)*K) of each band of W*K query rows.  Warps form
@@ -102,6 +125,7 @@ struct Cell {
 // and, for the last warp, to warp 0 of the next band through a global border row held
 // in a per-SM slot.  One __syncthreads per step.
 // ------------------------------------------------------------------------------------
+// UQ: 8 = one skewed tile over all 8 columns of a step, otherwise tiles of 4 columns
 template <int K, int W, int T, int MINB, int UQ>
 __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   static_assert(T == 4 || T == 8, "tile = one or two 32-bit words of residues");
@@ -215,21 +239,25 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
       // rows of the last band past the longer query are padding: skip them (nobody reads
       // their output; the last band writes no border)
       const bool live = band < nb - 1 || warp * K < rows - (nb - 1) * BAND;
-#pragma unroll UQ
-      for (int q = 0; q < T / 4 && live; q++) {
-        const uint32_t word = (T == 4 || q == 0) ? wds[0] : wds[T / 4 - 1];
+      constexpr int G = (UQ == 8) ? 8 : 4;   // columns interleaved in one skewed tile
 #pragma unroll
-        for (int j4 = 0; j4 < 4; j4++) {
-          const int jj = q * 4 + j4;
-          const int c = (word >> (8 * j4)) & 0xff;
+      for (int q = 0; q < T / G && live; q++) {
+        const uint32_t *prc[G];
+        uint32_t hdc[G], fc[G], oh[G];
+#pragma unroll
+        for (int j = 0; j < G; j++) {
+          const int jj = q * G + j;
+          const uint32_t word = wds[jj / 4];
+          const int c = (word >> (8 * (jj % 4))) & 0xff;
           const uint2 v = inp[jj * 32 + lane];
-          uint32_t hd = hprev_top, f = v.y;
+          prc[j] = pr_base + c * S;
+          hdc[j] = hprev_top;   // H(row above, previous column)
+          fc[j] = v.y;
           hprev_top = v.x;
-          const uint32_t *pr = pr_base + c * S;
-#pragma unroll
-          for (int i = 0; i < K; i++) Cell::row(pr[i], hd, H[i], E[i], f, best, na, nbeta, koff);
-          outp[jj * 32 + lane] = make_uint2(H[K - 1], f);
         }
+        dp_tile<K, G, 1>(prc, H, E, hdc, fc, oh, best, na, nbeta, koff);
+#pragma unroll
+        for (int j = 0; j < G; j++) outp[(q * G + j) * 32 + lane] = make_uint2(oh[j], fc[j]);
       }
       if (warp == W - 1 && band < nb - 1) {
 #pragma unroll
@@ -276,8 +304,8 @@ static size_t k1_smem() {
          sizeof(uint32_t) * kK1Warps * 32 + sizeof(uint2) * 3 * T * 32;
 }
 
-// K1 variants (tuning; SW_K1_VARIANT): 0 = T8 / 2 blocks per SM, 1 = T4 / 3 blocks per SM,
-// 2 = T8 / 3 blocks per SM, 3 = T8 / 3 blocks / one 4-column word unrolled at a time (default)
+// K1 variants (tuning; SW_K1_VARIANT): 0 = T8 / 2 blocks per SM / 4-column skewed tiles,
+// 1 = T4 / 3 blocks, 2 = T8 / 3 blocks, 3 = T8 / 2 blocks / one 8-column tile (default)
 static int k1_variant() {
   static int v = -1;
   if (v < 0) {
@@ -299,7 +327,7 @@ int k1_blocks_per_sm() {
   static int v = -1;
   if (v < 0) {
     const int k = k1_variant();
-    v = k == 1 ? k1_occ<4, 3, 1>() : k == 2 ? k1_occ<8, 3, 2>() : k == 3 ? k1_occ<8, 3, 1>() : k1_occ<8, 2, 2>();
+    v = k == 1 ? k1_occ<4, 3, 4>() : k == 2 ? k1_occ<8, 3, 4>() : k == 3 ? k1_occ<8, 2, 8>() : k1_occ<8, 2, 4>();
   }
   return v;
 }
@@ -309,10 +337,10 @@ void launch_k1(const K1Args &a, int n_groups, int, int, cudaStream_t st, int) {
   k1_blocks_per_sm();  // sets the smem attribute once
   const int k = k1_variant();
   const dim3 g(n_groups), b(kK1Warps * 32);
-  if (k == 1) k1_kernel<kK1Rows, kK1Warps, 4, 3, 1><<<g, b, k1_smem<4>(), st>>>(a);
-  else if (k == 2) k1_kernel<kK1Rows, kK1Warps, 8, 3, 2><<<g, b, k1_smem<8>(), st>>>(a);
-  else if (k == 3) k1_kernel<kK1Rows, kK1Warps, 8, 3, 1><<<g, b, k1_smem<8>(), st>>>(a);
-  else k1_kernel<kK1Rows, kK1Warps, 8, 2, 2><<<g, b, k1_smem<8>(), st>>>(a);
+  if (k == 1) k1_kernel<kK1Rows, kK1Warps, 4, 3, 4><<<g, b, k1_smem<4>(), st>>>(a);
+  else if (k == 2) k1_kernel<kK1Rows, kK1Warps, 8, 3, 4><<<g, b, k1_smem<8>(), st>>>(a);
+  else if (k == 3) k1_kernel<kK1Rows, kK1Warps, 8, 2, 8><<<g, b, k1_smem<8>(), st>>>(a);
+  else k1_kernel<kK1Rows, kK1Warps, 8, 2, 4><<<g, b, k1_smem<8>(), st>>>(a);
 }
 
 // ------------------------------------------------------------------------------------
@@ -406,17 +434,17 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
       }
       const int tile = t - lane;
       if (tile >= 0 && tile < ntile) {
+        const uint32_t *prc[T];
+        uint32_t hdc[T];
 #pragma unroll
         for (int jj = 0; jj < T; jj++) {
           const uint32_t c = (in_c >> (8 * jj)) & 0xffu;
-          uint32_t hd = hprev_top, f = in_f[jj];
+          prc[jj] = smem + c * K * 32 + lane;
+          hdc[jj] = hprev_top;
+          out_f[jj] = in_f[jj];
           hprev_top = in_h[jj];
-          const uint32_t *pr = smem + c * K * 32 + lane;
-#pragma unroll
-          for (int i = 0; i < K; i++) Cell::row(pr[i * 32], hd, H[i], E[i], f, best, na, nbeta, koff);
-          out_h[jj] = H[K - 1];
-          out_f[jj] = f;
         }
+        dp_tile<K, T, 32>(prc, H, E, hdc, out_f, out_h, best, na, nbeta, koff);
         out_c = in_c;
         if (lane == 31 && ch < nch - 1)
 #pragma unroll

@@ -164,6 +164,19 @@ __global__ void __launch_bounds__(256) dp(const uint4 *__restrict__ db, const ui
             hd = H[i]; H[i] = h;
             best = __vmaxs2(best, h);
           }
+        } else if (VAR == 10) {  // t by 32-bit add (no floor); E, F floored by 3-input max
+          uint32_t hd = Kp, f = Kp;
+#pragma unroll
+          for (int i = 0; i < K; i++) {
+            uint32_t v = pr[i];
+            uint32_t x = hd + v;
+            uint32_t h = __vimax3_s16x2(x, E[i], f);
+            uint32_t t = h - A32;
+            E[i] = __vimax3_s16x2(E[i] - B32, t, Kp);
+            f = __vimax3_s16x2(f - B32, t, Kp);
+            hd = H[i]; H[i] = h;
+            best = __vmaxs2(best, h);
+          }
         } else {                 // all full-rate: IADD + 2-input max
           uint32_t hd = Kp, f = Kp;
 #pragma unroll
@@ -250,14 +263,12 @@ int main() {
   double ghz = 1.965;  // nominal max; actual printed by nvidia-smi sampling
   std::vector<uint32_t> r0, r1, r2, r3;
   int reps = 2;
-  std::vector<uint32_t> r4, r5, r6, r7, r8, r9;
+  std::vector<uint32_t> r4, r10;
   for (int pass = 0; pass < 2; pass++) {
     run<16, 2>(nthreads, ddb, 12, 2, dout, r2, reps, ghz, nsm);
-    run<16, 7>(nthreads, ddb, 12, 2, dout, r7, reps, ghz, nsm);
-    run<16, 8>(nthreads, ddb, 12, 2, dout, r8, reps, ghz, nsm);
-    run<16, 9>(nthreads, ddb, 12, 2, dout, r9, reps, ghz, nsm);
-    run<16, 4>(nthreads, ddb, 12, 2, dout, r4, reps, ghz, nsm);
-    printf("agree16: %d %d %d %d\n", r2 == r7, r2 == r8, r2 == r9, r2 == r4);
+    run<16, 10>(nthreads, ddb, 12, 2, dout, r10, reps, ghz, nsm);
+    run<16, 5>(nthreads, ddb, 12, 2, dout, r4, reps, ghz, nsm);
+    printf("agree16: %d %d\n", r2 == r10, r2 == r4);
   }
   return 0;
 }
