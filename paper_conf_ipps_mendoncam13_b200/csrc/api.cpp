@@ -83,10 +83,51 @@ struct DBuf {
     if (p) { cudaSetDevice(dev); cudaFree(p); }
     p = nullptr; n = 0;
   }
+  // grow-only: keep the allocation across searches when it is large enough
+  void ensure(int d, size_t count) {
+    if (p && dev == d && count <= n) return;
+    alloc(d, std::max<size_t>(count, 1));
+  }
   ~DBuf() { free(); }
   DBuf() = default;
   DBuf(const DBuf &) = delete;
   DBuf &operator=(const DBuf &) = delete;
+};
+
+struct Device;
+// per-device search resources, cached in the sw_db across searches (grow-only buffers,
+// events and the cancellation stream are created once)
+struct DevSearch {
+  Device *D = nullptr;
+  DBuf<uint8_t> qcodes;
+  DBuf<int64_t> qoff;
+  DBuf<QueryPair> pairs;
+  DBuf<int8_t> matrix;
+  DBuf<int32_t> prof;
+  DBuf<int32_t> scores_own;
+  int32_t *scores = nullptr;
+  DBuf<int2> ovf;
+  DBuf<int32_t> ovf_count;
+  DBuf<uint2> k3_border;   // [streams][max_k3_seqs][max_len]
+  DBuf<int32_t> k2_border;
+  DBuf<int32_t> abort_dev;      // per-unit WA cancellation flags (device memory)
+  int32_t *abort_d = nullptr;
+  int32_t *one_h = nullptr;      // pinned constant 1, source of the cancellation copies
+  cudaStream_t cancel_st = nullptr;
+  std::vector<char> cancelled;
+  cudaEvent_t ev_start = nullptr, ev_end = nullptr;
+  std::vector<cudaEvent_t> u_start, u_end;  // per stream
+  int launches = 0;
+  double k1_sec = 0, k3_sec = 0;
+  int64_t k1_cells = 0, k3_cells = 0;
+  int64_t dup_cells = 0;
+  double finish_wall = 0;
+  int32_t n_ovf = 0;
+  void reset_counters() {
+    launches = 0; k1_sec = k3_sec = 0; k1_cells = k3_cells = 0; dup_cells = 0;
+    finish_wall = 0; n_ovf = 0; scores = nullptr;
+  }
+  ~DevSearch();
 };
 
 struct Device {
@@ -99,11 +140,22 @@ struct Device {
   DBuf<int32_t> slot_busy;
   int32_t slots_per_sm = 0, slot_cols = 0, sm_slots = 0;
   std::vector<cudaStream_t> streams;
+  std::unique_ptr<DevSearch> ws;   // cached search resources
   ~Device() {
     cudaSetDevice(id);
+    ws.reset();
     for (auto s : streams) cudaStreamDestroy(s);
   }
 };
+inline DevSearch::~DevSearch() {
+  if (one_h) cudaFreeHost(one_h);
+  if (cancel_st) cudaStreamDestroy(cancel_st);
+  if (ev_start) cudaEventDestroy(ev_start);
+  if (ev_end) cudaEventDestroy(ev_end);
+  for (auto e : u_start) cudaEventDestroy(e);
+  for (auto e : u_end) cudaEventDestroy(e);
+}
+
 
 }  // namespace sw
 
@@ -249,43 +301,6 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
 }
 
 // ---------------------------------------------------------------- per-search device state
-struct DevSearch {
-  Device *D = nullptr;
-  DBuf<uint8_t> qcodes;
-  DBuf<int64_t> qoff;
-  DBuf<QueryPair> pairs;
-  DBuf<int8_t> matrix;
-  DBuf<int32_t> prof;
-  DBuf<int32_t> scores_own;
-  int32_t *scores = nullptr;
-  DBuf<int2> ovf;
-  DBuf<int32_t> ovf_count;
-  DBuf<uint2> k3_border;   // [streams][max_k3_seqs][max_len]
-  DBuf<int32_t> k2_border;
-  DBuf<int32_t> abort_dev;      // per-unit WA cancellation flags (device memory)
-  int32_t *abort_d = nullptr;
-  int32_t *one_h = nullptr;      // pinned constant 1, source of the cancellation copies
-  cudaStream_t cancel_st = nullptr;
-  std::vector<char> cancelled;
-  cudaEvent_t ev_start = nullptr, ev_end = nullptr;
-  std::vector<cudaEvent_t> u_start, u_end;  // per stream
-  int launches = 0;
-  double k1_sec = 0, k3_sec = 0;
-  int64_t k1_cells = 0, k3_cells = 0;
-  int64_t dup_cells = 0;
-  double finish_wall = 0;
-  int32_t n_ovf = 0;
-  ~DevSearch() {
-    if (D) cudaSetDevice(D->id);
-    if (one_h) cudaFreeHost(one_h);
-    if (cancel_st) cudaStreamDestroy(cancel_st);
-    if (ev_start) cudaEventDestroy(ev_start);
-    if (ev_end) cudaEventDestroy(ev_end);
-    for (auto e : u_start) cudaEventDestroy(e);
-    for (auto e : u_end) cudaEventDestroy(e);
-  }
-};
-
 struct UnitLog {
   int32_t unit, worker;
   double t_grant, t_start, t_end;
@@ -448,14 +463,16 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
     Plan P = make_plan(queries, H, o, dist ? o.dist_world : nW);
     const double wall0 = now_s();
 
-    std::vector<std::unique_ptr<DevSearch>> S(nW);
-    // ---------------- per device setup (not timed as device work)
+    std::vector<DevSearch *> S(nW);
+    // ---------------- per device setup (cached, grow-only resources; not device-timed)
     for (int w = 0; w < nW; w++) {
-      S[w] = std::make_unique<DevSearch>();
-      DevSearch &X = *S[w];
-      X.D = db->devs[w].get();
-      Device &D = *X.D;
+      Device &D = *db->devs[w];
       CK(cudaSetDevice(D.id));
+      if (!D.ws) D.ws = std::make_unique<DevSearch>();
+      S[w] = D.ws.get();
+      DevSearch &X = *S[w];
+      X.D = &D;
+      X.reset_counters();
       const int depth = o.streams_per_device;
       while ((int)D.streams.size() < depth) {
         cudaStream_t st;
@@ -476,37 +493,40 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         CK(cudaMemset(D.slot_busy.p, 0, sizeof(int32_t) * D.slot_busy.n));
         D.slot_cols = need_cols;
       }
-      X.qcodes.alloc(D.id, std::max<size_t>(P.qcodes.size(), 1));
-      X.qoff.alloc(D.id, P.qoff.size());
-      X.pairs.alloc(D.id, std::max<size_t>(P.pairs.size(), 1));
-      X.matrix.alloc(D.id, 24 * 24);
-      X.prof.alloc(D.id, std::max<int64_t>(P.prof_total, 1));
+      X.qcodes.ensure(D.id, P.qcodes.size());
+      X.qoff.ensure(D.id, P.qoff.size());
+      X.pairs.ensure(D.id, P.pairs.size());
+      X.matrix.ensure(D.id, 24 * 24);
+      X.prof.ensure(D.id, (size_t)P.prof_total);
       if (!P.qcodes.empty()) CK(cudaMemcpy(X.qcodes.p, P.qcodes.data(), P.qcodes.size(), cudaMemcpyHostToDevice));
       CK(cudaMemcpy(X.qoff.p, P.qoff.data(), sizeof(int64_t) * P.qoff.size(), cudaMemcpyHostToDevice));
       if (!P.pairs.empty()) CK(cudaMemcpy(X.pairs.p, P.pairs.data(), sizeof(QueryPair) * P.pairs.size(), cudaMemcpyHostToDevice));
       CK(cudaMemcpy(X.matrix.p, M, 24 * 24, cudaMemcpyHostToDevice));
       const size_t nsc = (size_t)nq * nd;
       if (w == 0 && o.outputs_on_device && scores && !dist) X.scores = scores;
-      else { X.scores_own.alloc(D.id, std::max<size_t>(nsc, 1)); X.scores = X.scores_own.p; }
-      X.ovf.alloc(D.id, kOvfCap);
-      X.ovf_count.alloc(D.id, 1);
+      else { X.scores_own.ensure(D.id, nsc); X.scores = X.scores_own.p; }
+      X.ovf.ensure(D.id, kOvfCap);
+      X.ovf_count.ensure(D.id, 1);
       const size_t k3b = (size_t)depth * std::max(P.max_k3_seqs, 1) * std::max<int64_t>(P.max_len, 1);
-      if (P.n_long_seqs > 0) X.k3_border.alloc(D.id, k3b);
+      if (P.n_long_seqs > 0) X.k3_border.ensure(D.id, k3b);
       const size_t nu = std::max<size_t>(P.units.size(), 1);
-      X.abort_dev.alloc(D.id, nu);
+      X.abort_dev.ensure(D.id, nu);
       CK(cudaMemset(X.abort_dev.p, 0, sizeof(int32_t) * nu));
       X.abort_d = X.abort_dev.p;
       X.cancelled.assign(nu, 0);
-      CK(cudaHostAlloc((void **)&X.one_h, sizeof(int32_t), cudaHostAllocDefault));
-      *X.one_h = 1;
-      CK(cudaStreamCreateWithFlags(&X.cancel_st, cudaStreamNonBlocking));
-      CK(cudaEventCreate(&X.ev_start));
-      CK(cudaEventCreate(&X.ev_end));
-      X.u_start.resize(depth);
-      X.u_end.resize(depth);
-      for (int k = 0; k < depth; k++) {
-        CK(cudaEventCreate(&X.u_start[k]));
-        CK(cudaEventCreate(&X.u_end[k]));
+      if (!X.one_h) {
+        CK(cudaHostAlloc((void **)&X.one_h, sizeof(int32_t), cudaHostAllocDefault));
+        *X.one_h = 1;
+      }
+      if (!X.cancel_st) CK(cudaStreamCreateWithFlags(&X.cancel_st, cudaStreamNonBlocking));
+      if (!X.ev_start) CK(cudaEventCreate(&X.ev_start));
+      if (!X.ev_end) CK(cudaEventCreate(&X.ev_end));
+      while ((int)X.u_start.size() < depth) {
+        cudaEvent_t a, b;
+        CK(cudaEventCreate(&a));
+        CK(cudaEventCreate(&b));
+        X.u_start.push_back(a);
+        X.u_end.push_back(b);
       }
       CK(cudaDeviceSynchronize());
     }
@@ -674,7 +694,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         if (novf > 0) {
           const int blocks = std::min(1024, (novf + 3) / 4);
           const int64_t stride = std::max<int64_t>(H.max_len, 1);
-          X.k2_border.alloc(D.id, (size_t)blocks * 4 * stride * 2);
+          X.k2_border.ensure(D.id, (size_t)blocks * 4 * stride * 2);
           K2Args a;
           a.qcodes = X.qcodes.p; a.qoff = X.qoff.p;
           a.packed = D.packed.p; a.groups = D.groups.p; a.sorted_len = D.sorted_len.p; a.perm = D.perm.p;

@@ -179,7 +179,7 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   uint32_t best = koff, hprev_top = koff;
   int band = 0, tile = 0;
   const uint4 *wp = a.packed + G.word_off + lane;
-  const int nwords = G.ncols / kWordCols;
+  const int nwords = (G.ncols + kWordCols - 1) / kWordCols;
   constexpr int TPW = kWordCols / T;   // tiles per 16-column residue word
   // residue words: current and the next one (prefetched a word ahead)
   uint4 r4 = wp[0];

@@ -96,8 +96,11 @@ void MasterServer::serve(int fd) {
     buf.clear();
     const double t = now_s();  // the master's clock
     switch (m.op) {
-      case kHello: worker = m.worker; break;
+      case kHello: worker = m.worker; registered_.fetch_add(1); break;
       case kRequest: {
+        // "the master process starts the execution and waits for the slaves to register"
+        // (P16 §IV): no task is handed out before every slave has registered
+        if (registered_.load() < world_) { h.rc = 0; break; }
         buf.resize(std::max(1, m.cap));
         h.rc = sched_ ? sw_sched_request(sched_, worker, t, buf.data(), m.cap) : -1;
         buf.resize(h.rc > 0 ? h.rc : 0);

@@ -31,6 +31,7 @@ class MasterServer {
   std::vector<std::thread> conns_;
   std::mutex mu_;
   std::atomic<int> done_{0};
+  std::atomic<int> registered_{0};
   std::atomic<bool> stopping_{false};
 };
 

@@ -8,7 +8,8 @@
 //    residues become 5-bit codes in NCBI order.
 // a2 "Length sort + interleaved packing" (north_star): stable sort by length
 //    (descending), groups of 32 sequences (one per lane of a K1 block), each group
-//    padded to its longest member rounded up to 16 columns, interleaved so word w of
+//    padded to its longest member rounded up to 8 columns (one K1 tile; the last
+//    16-column word may be half used), interleaved so word w of
 //    lane l is packed[word_off + w*32 + l] (a warp load = 512 contiguous bytes).
 #include <algorithm>
 #include <cstring>
@@ -133,17 +134,17 @@ int pack_database(const int64_t *offsets, const char *residues, int32_t n, Packe
     G.first = g * kGroup;
     G.count = std::min(kGroup, n - G.first);
     int32_t l = out.sorted_len[G.first];
-    int32_t cols = (l + kWordCols - 1) / kWordCols * kWordCols;
+    int32_t cols = (l + kColAlign - 1) / kColAlign * kColAlign;
     G.ncols = std::max(cols, kMinCols);
     G.word_off = words;
     G.pad_ = 0;
-    words += (int64_t)(G.ncols / kWordCols) * kGroup;
+    words += (int64_t)((G.ncols + kWordCols - 1) / kWordCols) * kGroup;
   }
   out.packed.assign(words, make_uint4(0, 0, 0, 0));
   uint8_t *bytes = reinterpret_cast<uint8_t *>(out.packed.data());
   for (int32_t g = 0; g < ng; g++) {
     const GroupInfo &G = out.groups[g];
-    const int32_t nw = G.ncols / kWordCols;
+    const int32_t nw = (G.ncols + kWordCols - 1) / kWordCols;
     for (int32_t lane = 0; lane < kGroup; lane++) {
       const int32_t s = G.first + lane;
       const bool real = lane < G.count;

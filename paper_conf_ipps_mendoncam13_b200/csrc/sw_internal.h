@@ -39,11 +39,12 @@ constexpr int kProfileRowAlign = 512;    // lcm(kK1Band, kK3Chunk)
 // ---- packed database (device) -------------------------------------------------------
 struct GroupInfo {       // one packing group of up to 32 length-sorted sequences
   int64_t word_off;      // offset (in uint4 words) of word 0, lane 0
-  int32_t ncols;         // padded columns (multiple of 16, >= kMinCols)
+  int32_t ncols;         // padded columns (multiple of kColAlign, >= kMinCols)
   int32_t first;         // index of the group's first sequence in sorted order
   int32_t count;         // real sequences in the group (<= 32)
   int32_t pad_;
 };
+constexpr int kColAlign = 8;       // group columns rounded to one K1 tile
 constexpr int kMinCols = 80;       // groups padded to >= (W+1)*T columns (rounded to 16): the K1 pipeline
                                    // prefetches warp 0's border one step ahead
 
