@@ -169,7 +169,7 @@ def main():
     ap.add_argument("--policy", default="pss")
     ap.add_argument("--no-wa", action="store_true")
     ap.add_argument("--straggler-mask", type=int, default=0)
-    ap.add_argument("--streams", type=int, default=3)
+    ap.add_argument("--streams", type=int, default=4)
     ap.add_argument("--unit-cells", type=int, default=0)
     ap.add_argument("--top-k", type=int, default=10)
     args = ap.parse_args()

@@ -78,7 +78,7 @@ typedef struct {
   int32_t policy;            /* SW_POLICY_SS | SW_POLICY_PSS (default PSS) */
   int32_t workload_adjust;   /* 1 = WA on (default, P20 "always activated"), 0 = off */
   int32_t omega;             /* PSS history length (Omega, P18 §IV.A.2); default 4 (reading R10) */
-  int32_t streams_per_device;/* units in flight per GPU (default 3) */
+  int32_t streams_per_device;/* units in flight per GPU (default 4) */
   int64_t target_unit_cells; /* cells per work unit; 0 = auto; INT64_MAX = one unit per
                                 query pair and kernel kind (the paper's very coarse
                                 "comparison of one query sequence to one genomic database",
@@ -87,15 +87,19 @@ typedef struct {
                                 (warp wavefront) kernel; 0 = auto (3072), <0 = never */
   int32_t outputs_on_device; /* 1: `scores` / `hits` are device pointers on the first
                                 device of the sw_db (inputs-resident timing mode) */
-  uint64_t straggler_mask;   /* bench/tests: worker w is throttled if bit w is set */
-  int32_t straggler_slowdown;/* throttle factor (grid capped to 1/slowdown of the SMs) */
+  uint64_t straggler_mask;   /* experiments: worker w emulates a slower PE if bit w is set:
+                                each completion is held back by (slowdown-1) x the unit's
+                                device time (SURVEY §8(d) WA experiment, P24 §V.C) */
+  int32_t straggler_slowdown;/* slowdown factor (default 6, Fig. 5's GPU:SSE ratio) */
   /* multi-process mode (one process per GPU, torchrun): world > 1 makes every rank a
      worker of one master, run as a thread of rank 0 and reached over TCP */
   int32_t dist_rank;
   int32_t dist_world;        /* 0/1 = single process (in-process master) */
   int32_t dist_port;         /* TCP port of the master (on dist_host) */
   const char *dist_host;     /* master address, e.g. "127.0.0.1" */
-  int32_t reserved[8];
+  int32_t straggler_after_ms;/* the straggler slows down only after this many ms (local
+                                load introduced mid-run, P24 §V.C); 0 = from the start */
+  int32_t reserved[7];
 } sw_opts;
 
 typedef struct {

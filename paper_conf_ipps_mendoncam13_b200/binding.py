@@ -40,7 +40,8 @@ class sw_opts(ctypes.Structure):
                 ("outputs_on_device", ctypes.c_int32), ("straggler_mask", ctypes.c_uint64),
                 ("straggler_slowdown", ctypes.c_int32), ("dist_rank", ctypes.c_int32),
                 ("dist_world", ctypes.c_int32), ("dist_port", ctypes.c_int32),
-                ("dist_host", ctypes.c_char_p), ("reserved", ctypes.c_int32 * 8)]
+                ("dist_host", ctypes.c_char_p), ("straggler_after_ms", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 7)]
 
 
 class sw_stats(ctypes.Structure):
@@ -203,9 +204,9 @@ class Database:
         return int(lib().sw_db_residues(self._h))
 
     def search(self, queries, matrix=None, gap_open=10, gap_extend=2, top_k=10, want_scores=True,
-               policy="pss", workload_adjust=True, omega=4, streams=3, target_unit_cells=0,
+               policy="pss", workload_adjust=True, omega=4, streams=4, target_unit_cells=0,
                long_threshold=0, outputs_on_device=False, straggler_mask=0, straggler_slowdown=6,
-               dist=None, out_scores=None, out_hits=None) -> SearchResult:
+               straggler_after_ms=0, dist=None, out_scores=None, out_hits=None) -> SearchResult:
         """sw_search.  Host outputs are numpy arrays (pinned buffers may be passed via
         out_scores / out_hits); with outputs_on_device the outputs are torch CUDA tensors."""
         keep = []
@@ -222,6 +223,7 @@ class Database:
         o.outputs_on_device = int(bool(outputs_on_device))
         o.straggler_mask = straggler_mask
         o.straggler_slowdown = straggler_slowdown
+        o.straggler_after_ms = straggler_after_ms
         if dist is not None:
             o.dist_rank, o.dist_world, o.dist_port = dist["rank"], dist["world"], dist["port"]
             host = dist.get("host", "127.0.0.1").encode()

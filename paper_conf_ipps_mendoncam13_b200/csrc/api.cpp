@@ -275,7 +275,8 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
       s = e;
     }
     // K1 units over the short groups
-    const int64_t rows_k1 = (int64_t)(std::max(qp.la, 1) + kK1Band - 1) / kK1Band * kK1Band;
+    const int64_t band = k1_band_rows();
+    const int64_t rows_k1 = (int64_t)(std::max(qp.la, 1) + band - 1) / band * band;
     for (int32_t g = gl; g < ng;) {
       int32_t e = g;
       int64_t cells = 0, work = 0;
@@ -362,7 +363,7 @@ void sw_opts_default(sw_opts *o) {
   o->policy = SW_POLICY_PSS;
   o->workload_adjust = 1;
   o->omega = 4;
-  o->streams_per_device = 3;
+  o->streams_per_device = 4;
   o->target_unit_cells = 0;
   o->long_threshold = 0;
   o->straggler_slowdown = 6;
@@ -441,7 +442,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
     sw_opts_default(&o);
     if (opts_in) o = *opts_in;
     if (o.omega < 1) o.omega = 4;
-    if (o.streams_per_device <= 0) o.streams_per_device = 3;
+    if (o.streams_per_device <= 0) o.streams_per_device = 4;
     if (o.policy != SW_POLICY_SS && o.policy != SW_POLICY_PSS) throw Error(SW_EINVAL, "bad policy");
     const bool dist = o.dist_world > 1;
     if (dist && (o.dist_rank < 0 || o.dist_rank >= o.dist_world || !o.dist_host || o.dist_port <= 0))
@@ -623,7 +624,8 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
               if (q == cudaErrorNotReady) continue;
               CK(q);
               completed_wait[k] = 1;
-              if (straggler) {  // emulate a PE `slow` times slower (SURVEY §8(d) WA experiment)
+              if (straggler && tn - t0 >= 1e-3 * o.straggler_after_ms) {
+                // emulate a PE `slow` times slower (SURVEY §8(d) WA experiment; P24 §V.C)
                 float ms = 0;
                 cudaEventElapsedTime(&ms, X.u_start[k], X.u_end[k]);
                 hold_until[k] = tn + (slow - 1.0) * ms * 1e-3;

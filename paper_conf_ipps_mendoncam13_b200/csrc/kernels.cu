@@ -297,50 +297,59 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   }
 }
 
-template <int T>
+template <int W, int T>
 static size_t k1_smem() {
-  constexpr int S = kK1Band + 1;
-  return sizeof(uint32_t) * 2 * kNCodes * S + sizeof(uint2) * kK1Warps * 2 * T * 32 +
-         sizeof(uint32_t) * kK1Warps * 32 + sizeof(uint2) * 3 * T * 32;
+  constexpr int S = kK1Rows * W + 1;
+  return sizeof(uint32_t) * 2 * kNCodes * S + sizeof(uint2) * W * 2 * T * 32 +
+         sizeof(uint32_t) * W * 32 + sizeof(uint2) * 3 * T * 32;
 }
 
-// K1 variants (tuning; SW_K1_VARIANT): 0 = T8 / 2 blocks per SM / 4-column skewed tiles,
-// 1 = T4 / 3 blocks, 2 = T8 / 3 blocks, 3 = T8 / 2 blocks / one 8-column tile (default)
+// K1 variants (tuning; SW_K1_VARIANT), (warps per block W, tile T, min blocks/SM, skew G):
+// 0 = (8, 8, 2, 4), 1 = (8, 4, 3, 4), 2 = (8, 8, 3, 4), 3 = (8, 8, 2, 8) (default),
+// 4 = (4, 8, 4, 8)
 static int k1_variant() {
   static int v = -1;
   if (v < 0) {
     const char *e = getenv("SW_K1_VARIANT");
     v = e ? atoi(e) : 3;
-    if (v < 0 || v > 3) v = 3;
+    if (v < 0 || v > 4) v = 3;
   }
   return v;
 }
-template <int T, int MINB, int UQ>
+template <int W, int T, int MINB, int UQ>
 static int k1_occ() {
-  auto fn = k1_kernel<kK1Rows, kK1Warps, T, MINB, UQ>;
-  cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem<T>());
+  auto fn = k1_kernel<kK1Rows, W, T, MINB, UQ>;
+  cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem<W, T>());
   int n = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, kK1Warps * 32, k1_smem<T>()) != cudaSuccess) n = 8;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, W * 32, k1_smem<W, T>()) != cudaSuccess) n = 8;
   return n > 0 ? n : 1;
 }
 int k1_blocks_per_sm() {
   static int v = -1;
   if (v < 0) {
-    const int k = k1_variant();
-    v = k == 1 ? k1_occ<4, 3, 4>() : k == 2 ? k1_occ<8, 3, 4>() : k == 3 ? k1_occ<8, 2, 8>() : k1_occ<8, 2, 4>();
+    switch (k1_variant()) {
+      case 0: v = k1_occ<8, 8, 2, 4>(); break;
+      case 1: v = k1_occ<8, 4, 3, 4>(); break;
+      case 2: v = k1_occ<8, 8, 3, 4>(); break;
+      case 4: v = k1_occ<4, 8, 4, 8>(); break;
+      default: v = k1_occ<8, 8, 2, 8>(); break;
+    }
   }
   return v;
 }
+int k1_band_rows() { return k1_variant() == 4 ? kK1Rows * 4 : kK1Rows * 8; }
 
 void launch_k1(const K1Args &a, int n_groups, int, int, cudaStream_t st, int) {
   if (n_groups <= 0) return;
   k1_blocks_per_sm();  // sets the smem attribute once
-  const int k = k1_variant();
-  const dim3 g(n_groups), b(kK1Warps * 32);
-  if (k == 1) k1_kernel<kK1Rows, kK1Warps, 4, 3, 4><<<g, b, k1_smem<4>(), st>>>(a);
-  else if (k == 2) k1_kernel<kK1Rows, kK1Warps, 8, 3, 4><<<g, b, k1_smem<8>(), st>>>(a);
-  else if (k == 3) k1_kernel<kK1Rows, kK1Warps, 8, 2, 8><<<g, b, k1_smem<8>(), st>>>(a);
-  else k1_kernel<kK1Rows, kK1Warps, 8, 2, 4><<<g, b, k1_smem<8>(), st>>>(a);
+  const dim3 g(n_groups);
+  switch (k1_variant()) {
+    case 0: k1_kernel<kK1Rows, 8, 8, 2, 4><<<g, 256, k1_smem<8, 8>(), st>>>(a); break;
+    case 1: k1_kernel<kK1Rows, 8, 4, 3, 4><<<g, 256, k1_smem<8, 4>(), st>>>(a); break;
+    case 2: k1_kernel<kK1Rows, 8, 8, 3, 4><<<g, 256, k1_smem<8, 8>(), st>>>(a); break;
+    case 4: k1_kernel<kK1Rows, 4, 8, 4, 8><<<g, 128, k1_smem<4, 8>(), st>>>(a); break;
+    default: k1_kernel<kK1Rows, 8, 8, 2, 8><<<g, 256, k1_smem<8, 8>(), st>>>(a); break;
+  }
 }
 
 // ------------------------------------------------------------------------------------

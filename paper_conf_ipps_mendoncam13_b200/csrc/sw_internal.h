@@ -110,6 +110,7 @@ void launch_max_merge(int32_t *dst, const int32_t *src, int64_t n, cudaStream_t 
 void launch_topk(const int32_t *scores, int32_t nq, int64_t ndb, int32_t k, int2 *hits,
                  cudaStream_t st);
 int k1_blocks_per_sm();
+int k1_band_rows();   // rows per K1 band (W*K of the selected variant)
 
 // ---- host packing (pack.cpp) ----------------------------------------------------------------
 int encode_residue(int ascii);   // -1 if invalid
