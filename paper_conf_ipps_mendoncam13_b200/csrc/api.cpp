@@ -685,7 +685,10 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
             }
           }
           if (done && pending.empty() && n_inflight == 0) break;
-          if (!progressed) std::this_thread::sleep_for(std::chrono::microseconds(20));
+          // poll completions every 20 us; an idle worker (nothing in flight, nothing granted)
+          // asks the master again every 100 us
+          if (!progressed)
+            std::this_thread::sleep_for(std::chrono::microseconds(n_inflight > 0 ? 20 : 100));
         }
         // int32 re-run of saturated pairs (K2), on this device's own list
         for (int k = 0; k < depth; k++) CK(cudaStreamSynchronize(D.streams[k]));
