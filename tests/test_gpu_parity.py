@@ -232,3 +232,41 @@ def test_c4_full_size_sampled():
     r = _search(w.db, w.queries, top_k=10)
     _sampled_parity(w, r, 1000, 4)
     assert (np.asarray(r.scores) >= 0).all()
+
+
+def test_paper_figures_on_gpu():
+    """The paper's printed values through the CUDA path: Fig. 2 (GAAGCTA x GCTGACCT,
+    linear gap -2, score 3, P12/P14) and Fig. 1's pair (SW >= the printed global 4)."""
+    M = np.full((24, 24), -1, np.int8)
+    np.fill_diagonal(M, 1)
+    qs = seqgen.SeqSet.from_list(["GAAGCTA", "ACTTGTCCG"])
+    db = seqgen.SeqSet.from_list(["GCTGACCT", "ATTGTCAG"])
+    r = _search(db, qs, matrix=M, gap_open=0, gap_extend=2, top_k=2)
+    assert r.scores[0, 0] == 3
+    assert r.scores[1, 1] >= 4
+    assert (r.scores == oracle.search(qs, db, matrix=M, gap_open=0, gap_extend=2)).all()
+
+
+@pytest.mark.parametrize("cfg", ["C3", "RAT", "MOUSE"])
+def test_other_databases_full_size_sampled(cfg):
+    """Table II's other database shapes (RefSeq Human, Ensembl Rat, RefSeq Mouse)."""
+    w = seqgen.make_workload(cfg)
+    r = _search(w.db, w.queries, top_k=10)
+    _sampled_parity(w, r, 600, 7)
+
+
+def test_c5_full_size_sampled():
+    """C5 at full size: 8 x 5,000-aa queries vs 2,048 sequences of 10k-35k aa (K3 + the
+    planted overflow pair re-scored in int32)."""
+    w = seqgen.make_workload("C5")
+    r = _search(w.db, w.queries, top_k=5)
+    assert r.stats["n_overflow_pairs"] >= 1 and r.stats["cells_k3"] == r.stats["cells"]
+    rng = np.random.default_rng(5)
+    qi = rng.integers(0, w.queries.n, 24).astype(np.int32)
+    di = rng.integers(0, w.db.n, 24).astype(np.int32)
+    pq = np.array([p["query"] for p in w.meta["planted"]], np.int32)
+    pd = np.array([p["slot"] for p in w.meta["planted"]], np.int32)
+    qi, di = np.concatenate([qi, pq]), np.concatenate([di, pd])
+    ref = oracle.pairs(w.queries, w.db, qi, di)
+    assert (np.asarray(r.scores)[qi, di] == ref).all()
+    assert ref.max() > 32767
