@@ -280,7 +280,9 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
     for (int32_t g = gl; g < ng;) {
       int32_t e = g;
       int64_t cells = 0, work = 0;
-      while (e < ng && (cells < target || e == g)) {
+      // (units do not straddle the kWideCols boundary: each launch uses one K1 instance)
+      const bool wide = db.groups[g].ncols >= kWideCols;
+      while (e < ng && (cells < target || e == g) && (db.groups[e].ncols >= kWideCols) == wide) {
         cells += rows_eff * grp_res[e];
         work += rows_k1 * db.groups[e].ncols * kGroup;
         e++;
@@ -329,7 +331,7 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     a.slot_busy = D.slot_busy.p;
     a.abort_flag = S.abort_d + uidx;
     a.na = na; a.nb = nbm;
-    launch_k1(a, U.b1 - U.b0, 0, P.pairs[U.pair].rows_padded, st, 0);
+    launch_k1(a, U.b1 - U.b0, db.groups[U.b1 - 1].ncols, P.pairs[U.pair].rows_padded, st, 0);
   } else {
     K3Args a;
     a.packed = D.packed.p; a.groups = D.groups.p; a.perm = D.perm.p; a.sorted_len = D.sorted_len.p;

@@ -128,7 +128,7 @@ __device__ __forceinline__ void dp_tile(const uint32_t *const (&prc)[G], uint32_
 // UQ: 8 = one skewed tile over all 8 columns of a step, otherwise tiles of 4 columns
 template <int K, int W, int T, int MINB, int UQ>
 __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
-  static_assert(T == 4 || T == 8, "tile = one or two 32-bit words of residues");
+  static_assert(T == 4 || T == 8 || T == 16, "tile = 1, 2 or 4 32-bit words of residues");
   constexpr int BAND = W * K;
   constexpr int S = BAND + 1;  // odd stride: lanes reading one row with different codes hit
                                // different banks
@@ -146,7 +146,7 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   const QueryPair P = a.pairs[a.pair];
   const int rows = P.la > P.lb ? P.la : P.lb;
   const int nb = (rows + BAND - 1) / BAND;
-  const int nt = G.ncols / T;
+  const int nt = G.ncols / T;   // groups are padded to a multiple of T (pack.cpp)
   const int total = nb * nt;
   const uint32_t koff = pk2(kOff), na = a.na, nbeta = a.nb;
   const int32_t *gprof = a.prof + P.prof_off;
@@ -239,14 +239,14 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
       // rows of the last band past the longer query are padding: skip them (nobody reads
       // their output; the last band writes no border)
       const bool live = band < nb - 1 || warp * K < rows - (nb - 1) * BAND;
-      constexpr int G = (UQ == 8) ? 8 : 4;   // columns interleaved in one skewed tile
+      constexpr int GS = (UQ == 8) ? 8 : 4;   // columns interleaved in one skewed tile
 #pragma unroll
-      for (int q = 0; q < T / G && live; q++) {
-        const uint32_t *prc[G];
-        uint32_t hdc[G], fc[G], oh[G];
+      for (int q = 0; q < T / GS && live; q++) {
+        const uint32_t *prc[GS];
+        uint32_t hdc[GS], fc[GS], oh[GS];
 #pragma unroll
-        for (int j = 0; j < G; j++) {
-          const int jj = q * G + j;
+        for (int j = 0; j < GS; j++) {
+          const int jj = q * GS + j;
           const uint32_t word = wds[jj / 4];
           const int c = (word >> (8 * (jj % 4))) & 0xff;
           const uint2 v = inp[jj * 32 + lane];
@@ -255,9 +255,9 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
           fc[j] = v.y;
           hprev_top = v.x;
         }
-        dp_tile<K, G, 1>(prc, H, E, hdc, fc, oh, best, na, nbeta, koff);
+        dp_tile<K, GS, 1>(prc, H, E, hdc, fc, oh, best, na, nbeta, koff);
 #pragma unroll
-        for (int j = 0; j < G; j++) outp[(q * G + j) * 32 + lane] = make_uint2(oh[j], fc[j]);
+        for (int j = 0; j < GS; j++) outp[(q * GS + j) * 32 + lane] = make_uint2(oh[j], fc[j]);
       }
       if (warp == W - 1 && band < nb - 1) {
 #pragma unroll
@@ -306,7 +306,8 @@ static size_t k1_smem() {
 
 // K1 variants (tuning; SW_K1_VARIANT), (warps per block W, tile T, min blocks/SM, skew G):
 // 0 = (8, 8, 2, 4), 1 = (8, 4, 3, 4), 2 = (8, 8, 3, 4), 3 = (8, 8, 2, 8) (default),
-// 4 = (4, 8, 4, 8)
+// 4 = (4, 8, 4, 8).  Groups of >= kWideCols columns use (8, 16, 2, 8) unless SW_K1_WIDE=0
+// (half the pipeline steps and barriers; needs nt >= W+1 tiles of 16 columns).
 static int k1_variant() {
   static int v = -1;
   if (v < 0) {
@@ -338,11 +339,24 @@ int k1_blocks_per_sm() {
   return v;
 }
 int k1_band_rows() { return k1_variant() == 4 ? kK1Rows * 4 : kK1Rows * 8; }
+static bool k1_wide_enabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = getenv("SW_K1_WIDE");
+    v = (e && atoi(e) == 0) ? 0 : 1;
+    if (v) k1_occ<8, 16, 2, 8>();
+  }
+  return v == 1;
+}
 
-void launch_k1(const K1Args &a, int n_groups, int, int, cudaStream_t st, int) {
+void launch_k1(const K1Args &a, int n_groups, int min_cols, int, cudaStream_t st, int) {
   if (n_groups <= 0) return;
   k1_blocks_per_sm();  // sets the smem attribute once
   const dim3 g(n_groups);
+  if (min_cols >= kWideCols && k1_variant() == 3 && k1_wide_enabled()) {
+    k1_kernel<kK1Rows, 8, 16, 2, 8><<<g, 256, k1_smem<8, 16>(), st>>>(a);
+    return;
+  }
   switch (k1_variant()) {
     case 0: k1_kernel<kK1Rows, 8, 8, 2, 4><<<g, 256, k1_smem<8, 8>(), st>>>(a); break;
     case 1: k1_kernel<kK1Rows, 8, 4, 3, 4><<<g, 256, k1_smem<8, 4>(), st>>>(a); break;

@@ -45,6 +45,7 @@ struct GroupInfo {       // one packing group of up to 32 length-sorted sequence
   int32_t pad_;
 };
 constexpr int kColAlign = 8;       // group columns rounded to one K1 tile
+constexpr int kWideCols = 144;     // groups this wide run the 16-column-step K1 instance
 constexpr int kMinCols = 80;       // groups padded to >= (W+1)*T columns (rounded to 16): the K1 pipeline
                                    // prefetches warp 0's border one step ahead
 
@@ -101,7 +102,7 @@ struct K2Args {   // int32 re-run of saturated pairs (warp per pair)
 
 void launch_profile(const uint8_t *qcodes, const int64_t *qoff, const QueryPair *pairs, int npairs,
                     const int8_t *matrix, int32_t *prof, int64_t prof_total, cudaStream_t st);
-void launch_k1(const K1Args &a, int n_groups, int max_cols, int rows_padded, cudaStream_t st,
+void launch_k1(const K1Args &a, int n_groups, int min_cols, int rows_padded, cudaStream_t st,
                int sm_cap);
 void launch_k3(const K3Args &a, int rows_padded, cudaStream_t st);
 void launch_k2(const K2Args &a, int blocks, cudaStream_t st);

@@ -15,7 +15,7 @@ __device__ __forceinline__ uint32_t pk(int v) { return ((uint32_t)(v & 0xffff)) 
 
 // profile entries: P[c][i] s16x2 (natural), Pa = S + alpha (s16x2), V = signed-packed int32 S
 template <int K, int VAR>
-__global__ void __launch_bounds__(256) dp(const uint4 *__restrict__ db, const uint32_t *__restrict__ gprof,
+__global__ void __launch_bounds__(256, (VAR == 11 ? 2 : 1)) dp(const uint4 *__restrict__ db, const uint32_t *__restrict__ gprof,
                                           int alpha, int beta, uint32_t *out, int reps) {
   __shared__ uint32_t P[NC * (K + 1)];
   for (int k = threadIdx.x; k < NC * (K + 1); k += blockDim.x) P[k] = gprof[k];
@@ -33,6 +33,42 @@ __global__ void __launch_bounds__(256) dp(const uint4 *__restrict__ db, const ui
       else { H[i] = Kp; E[i] = Kp; }                    // offset repr, floored E
     }
     const uint4 *p = db + tid;
+    if (VAR == 11) {   // VAR2 cell, 8 columns per tile with explicit row skew (ILP 8)
+      uint32_t hprev = Kp;
+      for (int w = 0; w < NCOL / 16; w++) {
+        uint4 r4 = p[(size_t)w * gridDim.x * blockDim.x];
+        uint32_t rw[4] = {r4.x, r4.y, r4.z, r4.w};
+#pragma unroll
+        for (int half = 0; half < 2; half++) {
+          const uint32_t *prc[8];
+          uint32_t hdc[8], fc[8];
+#pragma unroll
+          for (int g = 0; g < 8; g++) {
+            const int b = half * 8 + g;
+            const int c = (rw[b >> 2] >> ((b & 3) * 8)) & 31;
+            prc[g] = P + c * (K + 1);
+            hdc[g] = hprev; fc[g] = Kp; hprev = Kp;
+          }
+#pragma unroll
+          for (int k = 0; k < K + 7; k++) {
+#pragma unroll
+            for (int g = 0; g < 8; g++) {
+              const int i = k - g;
+              if (i >= 0 && i < K) {
+                uint32_t x = hdc[g] + prc[g][i];
+                uint32_t h = __vimax3_s16x2(x, E[i], fc[g]);
+                uint32_t t = __viaddmax_s16x2(h, na, Kp);
+                E[i] = __viaddmax_s16x2(E[i], nb, t);
+                fc[g] = __viaddmax_s16x2(fc[g], nb, t);
+                hdc[g] = H[i]; H[i] = h;
+                best = __vmaxs2(best, h);
+              }
+            }
+          }
+        }
+      }
+      continue;
+    }
     for (int w = 0; w < NCOL / 16; w++) {
       uint4 r4 = p[(size_t)w * gridDim.x * blockDim.x];
       uint32_t rw[4] = {r4.x, r4.y, r4.z, r4.w};
@@ -263,12 +299,11 @@ int main() {
   double ghz = 1.965;  // nominal max; actual printed by nvidia-smi sampling
   std::vector<uint32_t> r0, r1, r2, r3;
   int reps = 2;
-  std::vector<uint32_t> r4, r10;
+  std::vector<uint32_t> r11;
   for (int pass = 0; pass < 2; pass++) {
     run<16, 2>(nthreads, ddb, 12, 2, dout, r2, reps, ghz, nsm);
-    run<16, 10>(nthreads, ddb, 12, 2, dout, r10, reps, ghz, nsm);
-    run<16, 5>(nthreads, ddb, 12, 2, dout, r4, reps, ghz, nsm);
-    printf("agree16: %d %d\n", r2 == r10, r2 == r4);
+    run<16, 11>(nthreads, ddb, 12, 2, dout, r11, reps, ghz, nsm);
+    printf("agree16: %d\n", r2 == r11);
   }
   return 0;
 }
