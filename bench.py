@@ -145,11 +145,14 @@ def reference_arm(args):
 
 
 def load_traffic():
+    """DRAM bytes per cell of the K1 launch captured with ncu --set full (profiles/)."""
     p = os.path.join(ROOT, "profiles", "ncu_k1_summary.json")
     try:
         with open(p) as f:
             d = json.load(f)
-        return d.get("dram_bytes_per_launch"), d
+        if d.get("cells"):
+            return d["dram_bytes_per_launch"] / d["cells"], d
+        return None, d
     except Exception:
         return None, None
 
@@ -181,10 +184,18 @@ def main():
     from paper_conf_ipps_mendoncam13_b200 import dist as swdist
 
     rank, world, local = env_rank()
+    # SW_BENCH_ONE_GPU=1: every rank on cuda:0 with a gloo merge (validates the multi-process
+    # path on a one-GPU box; NCCL refuses two ranks on one device)
+    one_gpu = os.environ.get("SW_BENCH_ONE_GPU") == "1"
+    if one_gpu:
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
         import torch.distributed as tdist
-        tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if one_gpu:
+            tdist.init_process_group("gloo")
+        else:
+            tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
 
     t = time.perf_counter()
     w = seqgen.make_workload(args.config, n_db=args.n_db)
@@ -201,10 +212,21 @@ def main():
             tdist.barrier()
             torch.cuda.synchronize()
             _, _, _, st = swdist.search(D, w.queries, rank, world, top_k=args.top_k, **kw)
-            torch.cuda.synchronize()   # NCCL merge + top-k ran on torch's stream after libsw
-            return st["seconds_device"], st
+            # libsw device time (common start after every slave registered) + the merge and
+            # top-k on torch's stream (CUDA events)
+            return st["seconds_device"] + st["merge_seconds"], st
         r = D.search(w.queries, top_k=args.top_k, outputs_on_device=True, **kw)
         return r.stats["seconds_device"], r.stats
+
+    # L2 (126 MB): the C4 packed DB (196 MB) exceeds it; smaller databases are flushed
+    # before every timed step by writing a 512 MB buffer (outside libsw's timed span)
+    db_bytes = int(w.db.total)
+    flush = None if db_bytes > 126_000_000 else torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
+
+    def flush_l2():
+        if flush is not None:
+            flush.fill_(1)
+            torch.cuda.synchronize()
 
     for _ in range(args.warmup):
         step()
@@ -217,13 +239,8 @@ def main():
     dev_s, launches, wall0 = 0.0, 0, time.perf_counter()
     stats = []
     for _ in range(args.steps):
-        t0 = time.perf_counter()
+        flush_l2()
         sec, st = step()
-        t1 = time.perf_counter()
-        if world > 1:
-            # merge time is part of the step: use the host span of the step as the upper
-            # bound on top of the device time of libsw (both measured on this rank)
-            sec = max(sec, t1 - t0)
         dev_s += sec
         launches += st["kernel_launches"]
         stats.append(st)
@@ -278,13 +295,32 @@ def main():
     peak = nsm * sm_mhz * 1e6 * DPX_RATE / DPX_PER_CELL / 1e9
     peak_max = nsm * 1965e6 * DPX_RATE / DPX_PER_CELL / 1e9
     per_gpu = value / world
-    traffic, _ = load_traffic()
-    roofline = {"bound": "alu", "achieved": per_gpu, "peak": peak, "unit": "GCUPS",
-                "frac": per_gpu / peak, "traffic": traffic,
-                "peak_at_max_clock": peak_max, "frac_at_max_clock": per_gpu / peak_max,
-                "kernel": "k1_kernel (inter-task) + k3_kernel (intra-task): whole step per GPU",
+    # the dominant kernel alone: one search with a single stream, so every inter-task (K1)
+    # launch runs by itself; achieved = K1 cells per launch / average K1 launch duration
+    # (CUDA events around each launch on its stream, inside libsw)
+    flush_l2()
+    alone = D.search(w.queries, top_k=args.top_k, outputs_on_device=True, streams=1,
+                     **{k: v for k, v in kw.items() if k != "streams"}).stats if world == 1 else None
+    k1_launches = sum(1 for e in (alone or {}).get("unit_log", []) if e["kind"] == 0)
+    k1_alone = (alone["cells_k1"] / alone["kernel_seconds_k1"] / 1e9) if alone and alone["kernel_seconds_k1"] > 0 else None
+    k3_alone = (alone["cells_k3"] / alone["kernel_seconds_k3"] / 1e9) if alone and alone["kernel_seconds_k3"] > 0 else None
+    bytes_per_cell, ncu = load_traffic()
+    cells_per_launch = alone["cells_k1"] / k1_launches if k1_launches else None
+    traffic = (bytes_per_cell * cells_per_launch) if (bytes_per_cell and cells_per_launch) else None
+    achieved = k1_alone if k1_alone else per_gpu
+    roofline = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "GCUPS",
+                "frac": achieved / peak, "traffic": traffic,
+                "kernel": "k1_kernel (inter-task DP), each launch alone (1 stream)",
+                "k1_launches": k1_launches, "k1_cells_per_launch": cells_per_launch,
+                "k1_avg_launch_ms": (1e3 * alone["kernel_seconds_k1"] / k1_launches) if k1_launches else None,
+                "k3_alone_gcups": k3_alone,
+                "step_gcups_per_gpu": per_gpu, "step_frac": per_gpu / peak,
+                "peak_at_max_clock": peak_max,
                 "derivation": f"{nsm} SMs x {sm_mhz:.0f} MHz (median under load) x {DPX_RATE:.0f} "
-                              f"DPX lane-ops/clk/SM (measured) / {DPX_PER_CELL:.0f} DPX per cell",
+                              f"DPX lane-ops/clk/SM (measured, tools/dpx_peak.cu) / "
+                              f"{DPX_PER_CELL:.0f} three-input DPX per cell (4 per s16x2 lane word)",
+                "traffic_note": "dram__bytes_read+write per K1 launch, scaled from the ncu --set full "
+                                "capture in profiles/ncu_k1_summary.json (bytes per cell x cells per launch)",
                 "k1_cells_share": last["cells_k1"] / max(1, last["cells_k1"] + last["cells_k3"])}
 
     cpu = None
@@ -301,8 +337,10 @@ def main():
                            "n_queries": nq, "db_residues": int(w.db.total),
                            "cells_per_step": cells, "policy": args.policy,
                            "workload_adjust": not args.no_wa, "streams_per_gpu": args.streams,
-                           "top_k": args.top_k, "l2": "inputs larger than L2 (packed DB "
-                           f"{w.db.total / 1e6:.0f} MB > 126 MB); no flush",
+                           "top_k": args.top_k,
+                           "l2": (f"inputs larger than L2 (packed DB {db_bytes / 1e6:.0f} MB > 126 MB); no flush"
+                                  if flush is None else
+                                  f"packed DB {db_bytes / 1e6:.0f} MB < L2: 512 MB buffer written before each step"),
                            "units_per_step": last["n_units"],
                            "overflow_pairs": last["n_overflow_pairs"],
                            "wa_grants": last["n_wa_grants"],

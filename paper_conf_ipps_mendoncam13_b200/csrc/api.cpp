@@ -331,7 +331,7 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     a.slot_busy = D.slot_busy.p;
     a.abort_flag = S.abort_d + uidx;
     a.na = na; a.nb = nbm;
-    launch_k1(a, U.b1 - U.b0, db.groups[U.b1 - 1].ncols, P.pairs[U.pair].rows_padded, st, 0);
+    launch_k1(a, U.b1 - U.b0, db.groups[U.b1 - 1].ncols, P.pairs[U.pair].rows_padded, st, D.n_sm);
   } else {
     K3Args a;
     a.packed = D.packed.p; a.groups = D.groups.p; a.perm = D.perm.p; a.sorted_len = D.sorted_len.p;

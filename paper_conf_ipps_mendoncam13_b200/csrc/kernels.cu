@@ -22,6 +22,7 @@
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
+#include <algorithm>
 #include "sw_internal.h"
 
 namespace sw {
@@ -132,35 +133,36 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   constexpr int BAND = W * K;
   constexpr int S = BAND + 1;  // odd stride: lanes reading one row with different codes hit
                                // different banks
+  constexpr int TPW = kWordCols / T;   // tiles per 16-column residue word
   extern __shared__ __align__(16) uint32_t smem[];
-  uint32_t *prof_s = smem;                                       // [2][kNCodes][S]
-  uint2 *hand = reinterpret_cast<uint2 *>(smem + 2 * kNCodes * S);  // [W][2][T][32]
-  uint32_t *red = reinterpret_cast<uint32_t *>(hand + W * 2 * T * 32);  // [W][32]
-  uint2 *bsm = reinterpret_cast<uint2 *>(red + W * 32);                  // [2][T][32]
-  uint2 *kin = bsm + 2 * T * 32;                                         // [T][32] = (kOff, kOff)
+  uint32_t *prof_s = smem;                                            // [2][kNCodes][S]
+  uint2 *hand = reinterpret_cast<uint2 *>(smem + 2 * kNCodes * S);    // [W][2][T][32]
+  uint32_t *red = reinterpret_cast<uint32_t *>(hand + W * 2 * T * 32);  // [2][W][32]
+  uint2 *bsm = reinterpret_cast<uint2 *>(red + 2 * W * 32);           // [2][T][32]
+  uint2 *kin = bsm + 2 * T * 32;                                      // [T][32] = (kOff, kOff)
   __shared__ int slot_s;
 
   if (block_aborted(a.abort_flag)) return;  // WA: this replica lost the race
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const GroupInfo G = a.groups[a.g0 + blockIdx.x];
   const QueryPair P = a.pairs[a.pair];
   const int rows = P.la > P.lb ? P.la : P.lb;
-  const int nb = (rows + BAND - 1) / BAND;
-  const int nt = G.ncols / T;   // groups are padded to a multiple of T (pack.cpp)
-  const int total = nb * nt;
+  // >= 1 band even for two empty queries (all rows skipped, scores 0)
+  const int nb = rows > 0 ? (rows + BAND - 1) / BAND : 1;
   const uint32_t koff = pk2(kOff), na = a.na, nbeta = a.nb;
   const int32_t *gprof = a.prof + P.prof_off;
+  // this block streams through groups gfirst, gfirst + gridDim.x, ... of the unit without
+  // draining the warp pipeline between them
+  const int gfirst = a.g0 + blockIdx.x, gend = a.g0 + a.n_groups, gstride = gridDim.x;
+  int total = 0;
+  for (int g = gfirst; g < gend; g += gstride) total += nb * (a.groups[g].ncols / T);
 
-  // border slot (only when there is more than one band)
   uint2 *border = nullptr;
-  if (nb > 1) {
-    if (threadIdx.x == 0) {
-      const int base = (int)smid() * a.slots_per_sm;
-      int k = 0;
-      for (;; k = (k + 1) % a.slots_per_sm)
-        if (atomicCAS(&a.slot_busy[base + k], 0, 1) == 0) break;
-      slot_s = base + k;
-    }
+  if (nb > 1 && threadIdx.x == 0) {   // a border-row slot of this SM (released at exit)
+    const int base = (int)smid() * a.slots_per_sm;
+    int k = 0;
+    for (;; k = (k + 1) % a.slots_per_sm)
+      if (atomicCAS(&a.slot_busy[base + k], 0, 1) == 0) break;
+    slot_s = base + k;
   }
   auto load_band = [&](int b, int slot) {
     uint32_t *dst = prof_s + slot * kNCodes * S;
@@ -175,23 +177,44 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   __syncthreads();
   if (nb > 1) border = a.border + (size_t)slot_s * a.border_slot_cols * 32;
 
+  // block-uniform tracker of warp 0's band starts: the profile of global band B+1 is
+  // loaded into slot (B+1)&1 when warp W-1 leaves band B-1, i.e. W-1 steps after warp 0
+  // starts band B (every band has nt >= W+1 steps, so warp 0 needs it later)
+  int t_g = gfirst, t_band = 0, t_nt = a.groups[gfirst].ncols / T, t_start = 0, t_B = 0;
+  int rl_step = -1, rl_band = 0, rl_slot = 0;
+
+  // per-warp iterator over (group, band, tile)
+  int g = gfirst, gk = 0, band = 0, tile = 0, gband = 0;
+  GroupInfo G = a.groups[g];
+  int nt = G.ncols / T, nwords = (G.ncols + kWordCols - 1) / kWordCols, wnext = nwords > 1 ? 1 : 0;
+  const uint4 *wp = a.packed + G.word_off + lane;
+  uint4 r4 = wp[0], r4n = wp[(size_t)wnext * 32];
   uint32_t H[K], E[K];
   uint32_t best = koff, hprev_top = koff;
-  int band = 0, tile = 0;
-  const uint4 *wp = a.packed + G.word_off + lane;
-  const int nwords = (G.ncols + kWordCols - 1) / kWordCols;
-  constexpr int TPW = kWordCols / T;   // tiles per 16-column residue word
-  // residue words: current and the next one (prefetched a word ahead)
-  uint4 r4 = wp[0];
-  uint4 r4n = wp[(size_t)(nwords > 1 ? 1 : 0) * 32];
-  int wnext = nwords > 1 ? 1 : 0;
+
   const int steps = total + W - 1;
   for (int s = 0; s < steps; s++) {
-    // band b+2 reuses the profile slot of band b once every warp has left band b
-    if (s >= W - 1 && (s - (W - 1)) % nt == 0) {
-      const int bl = (s - (W - 1)) / nt - 1;
-      if (bl >= 0 && bl + 2 < nb) {
-        load_band(bl + 2, bl & 1);
+    if (nb > 2) {
+      if (s == t_start + t_nt) {   // warp 0 enters its next band at this step
+        t_start += t_nt;
+        t_B++;
+        if (++t_band == nb) {
+          t_band = 0;
+          t_g += gstride;
+          if (t_g < gend) t_nt = a.groups[t_g].ncols / T;
+        }
+        // the band after this one: rows (t_band+1) mod nb, slot (t_B+1)&1
+        if (t_B + 1 >= 2) {
+          const bool last_overall = t_g >= gend || (t_band == nb - 1 && t_g + gstride >= gend);
+          if (!last_overall) {
+            rl_step = t_start + W - 1;
+            rl_band = t_band + 1 == nb ? 0 : t_band + 1;
+            rl_slot = (t_B + 1) & 1;
+          }
+        }
+      }
+      if (s == rl_step) {
+        load_band(rl_band, rl_slot);
         __syncthreads();
       }
     }
@@ -201,34 +224,34 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
 #pragma unroll
         for (int i = 0; i < K; i++) { H[i] = koff; E[i] = koff; }
         hprev_top = koff;
-      }
-      if (tile != 0 && (tile % TPW) == 0) {
+        if (band > 0) {   // new band of the same group: restart at word 0 (prefetched)
+          r4 = r4n;
+          wnext = nwords > 1 ? 1 : 0;
+          r4n = wp[(size_t)wnext * 32];
+        }
+      } else if ((tile % TPW) == 0) {
         r4 = r4n;
         wnext = (wnext + 1 == nwords) ? 0 : wnext + 1;
         r4n = wp[(size_t)wnext * 32];
-      } else if (tile == 0 && band > 0) {
-        // new band: restart at word 0 (prefetched at the end of the previous band)
-        r4 = r4n;
-        wnext = nwords > 1 ? 1 : 0;
-        r4n = wp[(size_t)wnext * 32];
       }
-      // warp 0: copy the border row of its next element (band2, tile2) into shared memory
-      // with cp.async, one step ahead (warp W-1 wrote it >= 1 step earlier: nt >= W+1)
+      // warp 0: copy the border row of its next element into shared memory with cp.async,
+      // one step ahead (warp W-1 wrote it >= 1 step earlier: nt >= W+1)
       if (warp == 0) {
-        const int tile2 = tile + 1 == nt ? 0 : tile + 1;
-        const int band2 = tile + 1 == nt ? band + 1 : band;
+        const bool wrap = tile + 1 == nt;
+        const int band2 = wrap ? band + 1 : band, tile2 = wrap ? 0 : tile + 1;
         if (band2 >= 1 && band2 < nb) {
 #pragma unroll
           for (int jj = 0; jj < T; jj++)
             cp_async8(&bsm[(((s + 1) & 1) * T + jj) * 32 + lane], &border[(size_t)(tile2 * T + jj) * 32 + lane]);
         }
       }
-      // top input of this tile (all in shared memory, so the column loop is branch-free):
+      // top input of this tile (shared memory, so the column loop is branch-free):
       // warp 0 <- constant row (band 0) or the cp.async'd border; warp w <- warp w-1
       const uint2 *inp = warp == 0 ? (band == 0 ? kin : bsm + (s & 1) * T * 32)
                                    : hand + ((warp - 1) * 2 + ((s - 1) & 1)) * T * 32;
       uint2 *outp = hand + (warp * 2 + (s & 1)) * T * 32;
-      const uint32_t *pr_base = prof_s + (band & 1) * kNCodes * S + warp * K;
+      const int slot = nb <= 2 ? band : (gband & 1);
+      const uint32_t *pr_base = prof_s + slot * kNCodes * S + warp * K;
       const int wq = (tile % TPW) * (T / 4);   // first 32-bit word of r4 used by this tile
       uint32_t wds[T / 4];
 #pragma unroll
@@ -263,45 +286,64 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
 #pragma unroll
         for (int jj = 0; jj < T; jj++) border[(size_t)(tile * T + jj) * 32 + lane] = outp[jj * 32 + lane];
       }
-      if (++tile == nt) { tile = 0; band++; }
+      // advance; at the end of a group publish this warp's best and move on
+      if (++tile == nt) {
+        tile = 0;
+        gband++;
+        if (++band == nb) {
+          band = 0;
+          uint32_t *rd = red + (gk & 1) * W * 32;
+          rd[warp * 32 + lane] = best;
+          best = koff;
+          if (warp == W - 1) {   // the last warp to finish the group reduces and writes
+            uint32_t m = rd[(W - 1) * 32 + lane];   // this warp's own, just written
+#pragma unroll
+            for (int w = 0; w < W - 1; w++) m = __vmaxs2(m, rd[w * 32 + lane]);
+            if (lane < G.count) {
+              const int ss = G.first + lane;
+              const int orig = a.perm[ss];
+              const int lo = (int)(int16_t)(m & 0xffff), hi = (int)(int16_t)(m >> 16);
+              if (lo >= a.thresh) {
+                const int k = atomicAdd(a.ovf_count, 1);
+                if (k < a.ovf_cap) a.ovf[k] = make_int2(P.qa, ss);
+              } else {
+                a.scores[(int64_t)P.qa * a.ndb + orig] = lo - kOff;
+              }
+              if (P.qb >= 0) {
+                if (hi >= a.thresh) {
+                  const int k = atomicAdd(a.ovf_count, 1);
+                  if (k < a.ovf_cap) a.ovf[k] = make_int2(P.qb, ss);
+                } else {
+                  a.scores[(int64_t)P.qb * a.ndb + orig] = hi - kOff;
+                }
+              }
+            }
+          }
+          gk++;
+          g += gstride;
+          if (g < gend) {
+            G = a.groups[g];
+            nt = G.ncols / T;
+            nwords = (G.ncols + kWordCols - 1) / kWordCols;
+            wnext = nwords > 1 ? 1 : 0;
+            wp = a.packed + G.word_off + lane;
+            r4 = wp[0];
+            r4n = wp[(size_t)wnext * 32];
+          }
+        }
+      }
       if (warp == 0) cp_async_commit_wait();
     }
     __syncthreads();
   }
-  red[warp * 32 + lane] = best;
-  __syncthreads();
   if (nb > 1 && threadIdx.x == 0) atomicExch(&a.slot_busy[slot_s], 0);
-  if (warp == 0) {
-    uint32_t m = red[lane];
-#pragma unroll
-    for (int w = 1; w < W; w++) m = __vmaxs2(m, red[w * 32 + lane]);
-    if (lane < G.count) {
-      const int ss = G.first + lane;
-      const int orig = a.perm[ss];
-      const int lo = (int)(int16_t)(m & 0xffff), hi = (int)(int16_t)(m >> 16);
-      if (lo >= a.thresh) {
-        const int k = atomicAdd(a.ovf_count, 1);
-        if (k < a.ovf_cap) a.ovf[k] = make_int2(P.qa, ss);
-      } else {
-        a.scores[(int64_t)P.qa * a.ndb + orig] = lo - kOff;
-      }
-      if (P.qb >= 0) {
-        if (hi >= a.thresh) {
-          const int k = atomicAdd(a.ovf_count, 1);
-          if (k < a.ovf_cap) a.ovf[k] = make_int2(P.qb, ss);
-        } else {
-          a.scores[(int64_t)P.qb * a.ndb + orig] = hi - kOff;
-        }
-      }
-    }
-  }
 }
 
 template <int W, int T>
 static size_t k1_smem() {
   constexpr int S = kK1Rows * W + 1;
   return sizeof(uint32_t) * 2 * kNCodes * S + sizeof(uint2) * W * 2 * T * 32 +
-         sizeof(uint32_t) * W * 32 + sizeof(uint2) * 3 * T * 32;
+         sizeof(uint32_t) * 2 * W * 32 + sizeof(uint2) * 3 * T * 32;
 }
 
 // K1 variants (tuning; SW_K1_VARIANT), (warps per block W, tile T, min blocks/SM, skew G):
@@ -349,10 +391,13 @@ static bool k1_wide_enabled() {
   return v == 1;
 }
 
-void launch_k1(const K1Args &a, int n_groups, int min_cols, int, cudaStream_t st, int) {
+void launch_k1(const K1Args &a_in, int n_groups, int min_cols, int, cudaStream_t st, int n_sm) {
   if (n_groups <= 0) return;
-  k1_blocks_per_sm();  // sets the smem attribute once
-  const dim3 g(n_groups);
+  K1Args a = a_in;
+  a.n_groups = n_groups;
+  // one wave of blocks (each streams through n_groups / grid groups)
+  const int cap = std::max(1, n_sm) * k1_blocks_per_sm();
+  const dim3 g(std::min(n_groups, cap));
   if (min_cols >= kWideCols && k1_variant() == 3 && k1_wide_enabled()) {
     k1_kernel<kK1Rows, 8, 16, 2, 8><<<g, 256, k1_smem<8, 16>(), st>>>(a);
     return;

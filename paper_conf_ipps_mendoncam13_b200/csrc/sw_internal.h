@@ -71,7 +71,8 @@ struct QueryPair {
 struct K1Args {
   const uint4 *packed; const GroupInfo *groups; const int32_t *perm;
   const int32_t *prof; const QueryPair *pairs;
-  int32_t pair; int32_t g0;          // unit: pair, first group (grid.x groups)
+  int32_t pair; int32_t g0;          // unit: pair, first group
+  int32_t n_groups;                  // groups [g0, g0 + n_groups) (set by launch_k1)
   int32_t *scores; int64_t ndb;      // [nq][ndb]
   int32_t thresh;                    // overflow threshold on best~ (offset repr)
   int2 *ovf; int32_t *ovf_count; int32_t ovf_cap;
@@ -103,7 +104,7 @@ struct K2Args {   // int32 re-run of saturated pairs (warp per pair)
 void launch_profile(const uint8_t *qcodes, const int64_t *qoff, const QueryPair *pairs, int npairs,
                     const int8_t *matrix, int32_t *prof, int64_t prof_total, cudaStream_t st);
 void launch_k1(const K1Args &a, int n_groups, int min_cols, int rows_padded, cudaStream_t st,
-               int sm_cap);
+               int n_sm);
 void launch_k3(const K3Args &a, int rows_padded, cudaStream_t st);
 void launch_k2(const K2Args &a, int blocks, cudaStream_t st);
 void launch_fill(int32_t *p, int64_t n, int32_t v, cudaStream_t st);

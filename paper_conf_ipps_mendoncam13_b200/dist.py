@@ -60,12 +60,26 @@ def merge_hits(scores: torch.Tensor, index: torch.Tensor, k: int, group=None):
 def search(database, queries, rank: int, world: int, top_k: int = 10, host: str = "127.0.0.1",
            port: int | None = None, **kw):
     """One distributed search step.  Returns (scores on rank 0 else None, hit scores,
-    hit index (rank 0), per-rank libsw stats)."""
+    hit index (rank 0), per-rank libsw stats with "merge_seconds" added: the device time of
+    the cross-rank merge and the top-k on this rank, CUDA events on torch's stream)."""
+    import torch
     port = port or master_port()
     r = database.search(queries, top_k=top_k, outputs_on_device=True,
                         dist=dict(rank=rank, world=world, port=port, host=host), **kw)
-    merged = merge_scores(r.scores)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record()
+    if dist.get_backend() == "gloo":   # tests / single-GPU runs: the merge goes through the host
+        part = r.scores.cpu()
+        merge_scores(part)
+        merged = part.to(r.scores.device) if rank == 0 else r.scores
+    else:
+        merged = merge_scores(r.scores)
+    hs = hi = None
+    if rank == 0 and top_k > 0:
+        hs, hi = database.topk_device(merged, top_k)
+    ev1.record()
+    torch.cuda.synchronize()
+    r.stats["merge_seconds"] = ev0.elapsed_time(ev1) * 1e-3
     if rank == 0:
-        hs, hi = database.topk_device(merged, top_k) if top_k > 0 else (None, None)
         return merged, hs, hi, r.stats
     return None, None, None, r.stats

@@ -18,6 +18,7 @@ ap.add_argument("--n-queries", type=int, default=None)
 ap.add_argument("--streams", type=int, default=3)
 ap.add_argument("--long-threshold", type=int, default=0)
 ap.add_argument("--dump-log", default=None)
+ap.add_argument("--print-k1", type=int, default=0, help="print the first N K1 units (launch order)")
 args = ap.parse_args()
 w = seqgen.make_workload(args.config, n_db=args.n_db, n_queries=args.n_queries)
 D = Database(w.db)
@@ -29,6 +30,10 @@ for s in range(args.steps):
     print(f"step {s}: {st['gcups']:.1f} GCUPS dev {st['seconds_device']:.3f}s wall {time.perf_counter()-t:.3f}s "
           f"k1 {st['kernel_seconds_k1']:.3f}s/{st['cells_k1']:.3e} k3 {st['kernel_seconds_k3']:.3f}s/{st['cells_k3']:.3e} "
           f"units {st['n_units']} launches {st['kernel_launches']}", flush=True)
+    if args.print_k1:
+        k1 = sorted((e for e in st["unit_log"] if e["kind"] == 0), key=lambda e: e["t_start"])
+        for e in k1[:args.print_k1]:
+            print(f"k1 unit {e['unit']} cells {e['cells']} pair {e['pair']}")
     if args.dump_log:
         import json
         json.dump(st["unit_log"], open(args.dump_log, "w"))
