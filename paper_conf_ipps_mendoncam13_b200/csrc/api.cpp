@@ -340,7 +340,7 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     a.scores = S.scores; a.ndb = db.n;
     a.thresh = thresh;
     a.ovf = S.ovf.p; a.ovf_count = S.ovf_count.p; a.ovf_cap = kOvfCap;
-    const int64_t stride = std::max<int64_t>(P.max_len, 1);
+    const int64_t stride = (std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16;  // >= tiles * T
     a.border = S.k3_border.p + (size_t)stream_idx * P.max_k3_seqs * stride;
     a.border_stride = stride;
     a.abort_flag = S.abort_d + uidx;
@@ -510,7 +510,8 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       else { X.scores_own.ensure(D.id, nsc); X.scores = X.scores_own.p; }
       X.ovf.ensure(D.id, kOvfCap);
       X.ovf_count.ensure(D.id, 1);
-      const size_t k3b = (size_t)depth * std::max(P.max_k3_seqs, 1) * std::max<int64_t>(P.max_len, 1);
+      const size_t k3b = (size_t)depth * std::max(P.max_k3_seqs, 1) *
+                         ((std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16);
       if (P.n_long_seqs > 0) X.k3_border.ensure(D.id, k3b);
       const size_t nu = std::max<size_t>(P.units.size(), 1);
       X.abort_dev.ensure(D.id, nu);

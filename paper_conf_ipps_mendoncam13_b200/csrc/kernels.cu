@@ -425,7 +425,9 @@ void launch_k1(const K1Args &a_in, int n_groups, int min_cols, int, cudaStream_t
 // ------------------------------------------------------------------------------------
 template <int K, int T>
 __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
-  static_assert(T == 4, "one 32-bit word of packed residues per tile");
+  static_assert(T == 4 || T == 8, "tile = one or two 32-bit words of packed residues");
+  constexpr int NW = T / 4;          // 32-bit residue words per tile
+  constexpr int TPU = 4 / NW;        // tiles per 128-bit word
   constexpr int CH = 32 * K;
   extern __shared__ __align__(16) uint32_t smem[];  // [kNCodes][K][32]
   if (block_aborted(a.abort_flag)) return;
@@ -458,32 +460,39 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
     uint32_t H[K], E[K];
 #pragma unroll
     for (int i = 0; i < K; i++) { H[i] = koff; E[i] = koff; }
-    uint32_t hprev_top = koff, out_c = padw;
-    uint32_t out_h[T], out_f[T];
+    uint32_t hprev_top = koff;
+    uint32_t out_h[T], out_f[T], out_c[NW];
     uint2 bn[T];
 #pragma unroll
     for (int jj = 0; jj < T; jj++) { out_h[jj] = koff; out_f[jj] = koff; bn[jj] = make_uint2(koff, koff); }
-    // lane 0's residue words (current, next) and border prefetch for tile 0
+#pragma unroll
+    for (int q = 0; q < NW; q++) out_c[q] = padw;
+    // lane 0's residue words (current, next 128-bit word) and border prefetch for tile 0
     uint4 wcur = make_uint4(padw, padw, padw, padw), wnx = wcur;
     if (lane == 0) {
       wcur = wp[0];
-      if (ntile > 4) wnx = wp[kGroup];
+      if (ntile > TPU) wnx = wp[kGroup];
       if (ch > 0)
 #pragma unroll
         for (int jj = 0; jj < T; jj++) bn[jj] = border[jj];
     }
     const int steps = ntile + 31;
     for (int t = 0; t < steps; t++) {
-      uint32_t in_h[T], in_f[T];
+      uint32_t in_h[T], in_f[T], in_c[NW];
 #pragma unroll
       for (int jj = 0; jj < T; jj++) {
         in_h[jj] = __shfl_up_sync(0xffffffffu, out_h[jj], 1);
         in_f[jj] = __shfl_up_sync(0xffffffffu, out_f[jj], 1);
       }
-      uint32_t in_c = __shfl_up_sync(0xffffffffu, out_c, 1);
+#pragma unroll
+      for (int q = 0; q < NW; q++) in_c[q] = __shfl_up_sync(0xffffffffu, out_c[q], 1);
       if (lane == 0 && t < ntile) {
-        const int q = t & 3;
-        in_c = q == 0 ? wcur.x : q == 1 ? wcur.y : q == 2 ? wcur.z : wcur.w;
+        const int q0 = (t % TPU) * NW;
+#pragma unroll
+        for (int q = 0; q < NW; q++) {
+          const int k = q0 + q;
+          in_c[q] = k == 0 ? wcur.x : k == 1 ? wcur.y : k == 2 ? wcur.z : wcur.w;
+        }
         if (ch == 0) {
 #pragma unroll
           for (int jj = 0; jj < T; jj++) { in_h[jj] = koff; in_f[jj] = koff; }
@@ -494,10 +503,10 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
 #pragma unroll
             for (int jj = 0; jj < T; jj++) bn[jj] = border[(t + 1) * T + jj];
         }
-        if (q == 3) {   // move to the next 16-column word, prefetch the one after
+        if (t % TPU == TPU - 1) {   // next 128-bit word; prefetch the one after
           wcur = wnx;
-          const int nw = (t >> 2) + 2;
-          if (nw * 4 < ntile) wnx = wp[(size_t)nw * kGroup];
+          const int nw = t / TPU + 2;
+          if (nw * TPU < ntile) wnx = wp[(size_t)nw * kGroup];
         }
       }
       const int tile = t - lane;
@@ -506,14 +515,15 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
         uint32_t hdc[T];
 #pragma unroll
         for (int jj = 0; jj < T; jj++) {
-          const uint32_t c = (in_c >> (8 * jj)) & 0xffu;
+          const uint32_t c = (in_c[jj / 4] >> (8 * (jj % 4))) & 0xffu;
           prc[jj] = smem + c * K * 32 + lane;
           hdc[jj] = hprev_top;
           out_f[jj] = in_f[jj];
           hprev_top = in_h[jj];
         }
         dp_tile<K, T, 32>(prc, H, E, hdc, out_f, out_h, best, na, nbeta, koff);
-        out_c = in_c;
+#pragma unroll
+        for (int q = 0; q < NW; q++) out_c[q] = in_c[q];
         if (lane == 31 && ch < nch - 1)
 #pragma unroll
           for (int jj = 0; jj < T; jj++) border[tile * T + jj] = make_uint2(out_h[jj], out_f[jj]);
@@ -543,14 +553,28 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
   }
 }
 
+// K3 tile width (tuning; SW_K3_T): 8 columns per lane step (default) or 4
+static int k3_tile() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = getenv("SW_K3_T");
+    v = (e && atoi(e) == 4) ? 4 : 8;
+  }
+  return v;
+}
 void launch_k3(const K3Args &a, int, cudaStream_t st) {
   const int n = a.l1 - a.l0;
   if (n <= 0) return;
   const size_t smem = sizeof(uint32_t) * kNCodes * kK3Rows * 32;
-  auto fn = k3_kernel<kK3Rows, 4>;
   static bool attr = false;
-  if (!attr) { cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); attr = true; }
-  fn<<<(n + kK3Warps - 1) / kK3Warps, kK3Warps * 32, smem, st>>>(a);
+  if (!attr) {
+    cudaFuncSetAttribute(k3_kernel<kK3Rows, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(k3_kernel<kK3Rows, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    attr = true;
+  }
+  const int blocks = (n + kK3Warps - 1) / kK3Warps;
+  if (k3_tile() == 4) k3_kernel<kK3Rows, 4><<<blocks, kK3Warps * 32, smem, st>>>(a);
+  else k3_kernel<kK3Rows, 8><<<blocks, kK3Warps * 32, smem, st>>>(a);
 }
 
 // ------------------------------------------------------------------------------------
