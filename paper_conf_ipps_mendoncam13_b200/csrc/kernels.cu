@@ -32,6 +32,13 @@ __device__ __forceinline__ void cp_async8(void *smem_dst, const void *gsrc) {
   const unsigned d = (unsigned)__cvta_generic_to_shared(smem_dst);
   asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(d), "l"(gsrc) : "memory");
 }
+__device__ __forceinline__ void cp_async16(void *smem_dst, const void *gsrc) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(smem_dst);
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(d), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit_wait1() {   // <= 1 group still in flight
+  asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 1;" ::: "memory");
+}
 __device__ __forceinline__ void cp_async_commit_wait() {
   asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
 }
@@ -429,7 +436,9 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
   constexpr int NW = T / 4;          // 32-bit residue words per tile
   constexpr int TPU = 4 / NW;        // tiles per 128-bit word
   constexpr int CH = 32 * K;
-  extern __shared__ __align__(16) uint32_t smem[];  // [kNCodes][K][32]
+  extern __shared__ __align__(16) uint32_t smem[];  // [kNCodes][K][32], then the rings
+  uint4 *ring4 = reinterpret_cast<uint4 *>(smem + kNCodes * K * 32);   // [warps][3]
+  uint2 *ring2 = reinterpret_cast<uint2 *>(ring4 + kK3Warps * 3);      // [warps][3][T]
   if (block_aborted(a.abort_flag)) return;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const QueryPair P = a.pairs[a.pair];
@@ -462,20 +471,30 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
     for (int i = 0; i < K; i++) { H[i] = koff; E[i] = koff; }
     uint32_t hprev_top = koff;
     uint32_t out_h[T], out_f[T], out_c[NW];
-    uint2 bn[T];
 #pragma unroll
-    for (int jj = 0; jj < T; jj++) { out_h[jj] = koff; out_f[jj] = koff; bn[jj] = make_uint2(koff, koff); }
+    for (int jj = 0; jj < T; jj++) { out_h[jj] = koff; out_f[jj] = koff; }
 #pragma unroll
     for (int q = 0; q < NW; q++) out_c[q] = padw;
-    // lane 0's residue words (current, next 128-bit word) and border prefetch for tile 0
-    uint4 wcur = make_uint4(padw, padw, padw, padw), wnx = wcur;
-    if (lane == 0) {
-      wcur = wp[0];
-      if (ntile > TPU) wnx = wp[kGroup];
-      if (ch > 0)
+    // lane 0 streams the tile inputs (border row of the previous chunk, residue words)
+    // into a 3-deep per-warp shared-memory ring with cp.async, two tiles ahead
+    uint2 *bring = ring2 + warp * 3 * T;   // [3][T]
+    uint4 *wring = ring4 + warp * 3;       // [3] words of 16 residues
+    auto fetch = [&](int tt) {             // lane 0: inputs of tile tt into slot tt % 3
+      if (tt < ntile) {
+        const int sl = tt % 3;
+        if (ch > 0)
 #pragma unroll
-        for (int jj = 0; jj < T; jj++) bn[jj] = border[jj];
+          for (int jj = 0; jj < T; jj++) cp_async8(&bring[sl * T + jj], &border[tt * T + jj]);
+        if (tt % TPU == 0) cp_async16(&wring[(tt / TPU) % 3], &wp[(size_t)(tt / TPU) * kGroup]);
+      }
+    };
+    if (lane == 0) {
+      fetch(0);
+      asm volatile("cp.async.commit_group;" ::: "memory");
+      fetch(1);
+      cp_async_commit_wait1();   // tile 0 has landed
     }
+    __syncwarp();
     const int steps = ntile + 31;
     for (int t = 0; t < steps; t++) {
       uint32_t in_h[T], in_f[T], in_c[NW];
@@ -487,27 +506,22 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
 #pragma unroll
       for (int q = 0; q < NW; q++) in_c[q] = __shfl_up_sync(0xffffffffu, out_c[q], 1);
       if (lane == 0 && t < ntile) {
+        const uint4 wv = wring[(t / TPU) % 3];
         const int q0 = (t % TPU) * NW;
 #pragma unroll
         for (int q = 0; q < NW; q++) {
           const int k = q0 + q;
-          in_c[q] = k == 0 ? wcur.x : k == 1 ? wcur.y : k == 2 ? wcur.z : wcur.w;
+          in_c[q] = k == 0 ? wv.x : k == 1 ? wv.y : k == 2 ? wv.z : wv.w;
         }
-        if (ch == 0) {
+        const int sl = t % 3;
 #pragma unroll
-          for (int jj = 0; jj < T; jj++) { in_h[jj] = koff; in_f[jj] = koff; }
-        } else {
-#pragma unroll
-          for (int jj = 0; jj < T; jj++) { in_h[jj] = bn[jj].x; in_f[jj] = bn[jj].y; }
-          if (t + 1 < ntile)
-#pragma unroll
-            for (int jj = 0; jj < T; jj++) bn[jj] = border[(t + 1) * T + jj];
+        for (int jj = 0; jj < T; jj++) {
+          const uint2 v = ch > 0 ? bring[sl * T + jj] : make_uint2(koff, koff);
+          in_h[jj] = v.x;
+          in_f[jj] = v.y;
         }
-        if (t % TPU == TPU - 1) {   // next 128-bit word; prefetch the one after
-          wcur = wnx;
-          const int nw = t / TPU + 2;
-          if (nw * TPU < ntile) wnx = wp[(size_t)nw * kGroup];
-        }
+        fetch(t + 2);              // slot (t+2)%3 == (t-1)%3, consumed last step
+        cp_async_commit_wait1();   // tile t+1 has landed
       }
       const int tile = t - lane;
       if (tile >= 0 && tile < ntile) {
@@ -565,7 +579,8 @@ static int k3_tile() {
 void launch_k3(const K3Args &a, int, cudaStream_t st) {
   const int n = a.l1 - a.l0;
   if (n <= 0) return;
-  const size_t smem = sizeof(uint32_t) * kNCodes * kK3Rows * 32;
+  const size_t smem = sizeof(uint32_t) * kNCodes * kK3Rows * 32 + sizeof(uint4) * kK3Warps * 3 +
+                      sizeof(uint2) * kK3Warps * 3 * 8;
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(k3_kernel<kK3Rows, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
