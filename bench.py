@@ -307,20 +307,24 @@ def main():
     bytes_per_cell, ncu = load_traffic()
     cells_per_launch = alone["cells_k1"] / k1_launches if k1_launches else None
     traffic = (bytes_per_cell * cells_per_launch) if (bytes_per_cell and cells_per_launch) else None
-    achieved = k1_alone if k1_alone else per_gpu
+    # achieved: the DP kernels (K1 inter-task + K3 intra-task are the whole step; they run
+    # concurrently on 4 streams, so per-launch durations overlap) -> cells of the timed
+    # steps / device time of the timed steps, per GPU.  The isolated per-launch rate of K1
+    # (1 stream, each launch alone incl. its own wave tail) is reported beside it.
+    achieved = per_gpu
     roofline = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "GCUPS",
                 "frac": achieved / peak, "traffic": traffic,
-                "kernel": "k1_kernel (inter-task DP), each launch alone (1 stream)",
+                "kernel": "k1_kernel + k3_kernel (all DP launches of the timed steps, per GPU)",
+                "k1_alone_gcups": k1_alone, "k1_alone_frac": (k1_alone / peak) if k1_alone else None,
                 "k1_launches": k1_launches, "k1_cells_per_launch": cells_per_launch,
                 "k1_avg_launch_ms": (1e3 * alone["kernel_seconds_k1"] / k1_launches) if k1_launches else None,
                 "k3_alone_gcups": k3_alone,
-                "step_gcups_per_gpu": per_gpu, "step_frac": per_gpu / peak,
                 "peak_at_max_clock": peak_max,
                 "derivation": f"{nsm} SMs x {sm_mhz:.0f} MHz (median under load) x {DPX_RATE:.0f} "
                               f"DPX lane-ops/clk/SM (measured, tools/dpx_peak.cu) / "
                               f"{DPX_PER_CELL:.0f} three-input DPX per cell (4 per s16x2 lane word)",
-                "traffic_note": "dram__bytes_read+write per K1 launch, scaled from the ncu --set full "
-                                "capture in profiles/ncu_k1_summary.json (bytes per cell x cells per launch)",
+                "traffic_note": "dram__bytes_read+write per K1 launch: bytes per cell of the ncu --set full "
+                                "capture (profiles/ncu_k1_summary.json) x the average cells per K1 launch",
                 "k1_cells_share": last["cells_k1"] / max(1, last["cells_k1"] + last["cells_k3"])}
 
     cpu = None
