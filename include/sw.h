@@ -164,6 +164,32 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
 int sw_topk_device(sw_db *db, const int32_t *scores_dev, int32_t nq, int32_t ndb, int32_t top_k,
                    sw_hit *hits_dev);
 
+/* ---- Phase 2: the alignments of selected pairs (NEXT-3) ---------------------------------
+ * P12 §II.A.2: "In order to obtain the optimal local alignment, the algorithm starts from
+ * the cell that has the highest value in H i, j, following the arrows until the value zero
+ * is reached."  For each requested (query, database sequence) pair the GPU recomputes the
+ * Gotoh matrices in int32 (one warp per pair, the same recurrence as sw_search) storing one
+ * direction byte per cell, picks the highest cell (ties: smallest query row, then smallest
+ * database column) and follows the arrows back to a zero.
+ * Ops: 'M' = q_i aligned with d_j (match or mismatch), 'I' = q_i against a gap, 'D' = d_j
+ * against a gap; listed from the alignment start.  Coordinates are 0-based, end-exclusive:
+ * the alignment covers q[q_begin, q_end) and d[d_begin, d_end) of the ORIGINAL sequences.
+ * An empty alignment (score 0) has n_ops = 0 and all coordinates 0. */
+typedef struct {
+  int32_t score;
+  int32_t q_begin, q_end, d_begin, d_end;
+  int32_t n_ops;
+  int64_t ops_offset;       /* into the caller's ops buffer */
+} sw_alignment;
+
+/* query_index[k], db_index[k] (original indices), k < n_pairs.  `ops` is caller-owned with
+ * ops_capacity bytes; sum over pairs of (|q| + |d|) always suffices (SW_EINVAL names the
+ * size needed otherwise).  Host pointers.  Device memory for the direction bytes is
+ * bounded (pairs are processed in batches). */
+int sw_align(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t gap_open,
+             int32_t gap_extend, const int32_t *query_index, const int32_t *db_index,
+             int32_t n_pairs, sw_alignment *out, char *ops, int64_t ops_capacity);
+
 /* Thread-local message of the last error on this thread ("" if none). */
 const char *sw_last_error(void);
 

@@ -44,6 +44,12 @@ class sw_opts(ctypes.Structure):
                 ("reserved", ctypes.c_int32 * 7)]
 
 
+class sw_alignment(ctypes.Structure):
+    _fields_ = [("score", ctypes.c_int32), ("q_begin", ctypes.c_int32), ("q_end", ctypes.c_int32),
+                ("d_begin", ctypes.c_int32), ("d_end", ctypes.c_int32), ("n_ops", ctypes.c_int32),
+                ("ops_offset", ctypes.c_int64)]
+
+
 class sw_stats(ctypes.Structure):
     _fields_ = [("cells", ctypes.c_int64), ("seconds_device", ctypes.c_double),
                 ("seconds_wall", ctypes.c_double), ("gcups", ctypes.c_double),
@@ -64,7 +70,7 @@ EXPORTS = ["sw_opts_default", "sw_db_create", "sw_db_destroy", "sw_db_residues",
            "sw_sched_committed_by", "sw_sched_replicas", "sw_sched_phi", "sw_sched_rate",
            "sw_sched_counter", "sw_sched_log_json", "sw_master_start", "sw_master_stop",
            "sw_slave_connect", "sw_slave_request", "sw_slave_report", "sw_slave_complete",
-           "sw_slave_abandon", "sw_slave_is_finished", "sw_slave_done"]
+           "sw_slave_abandon", "sw_slave_is_finished", "sw_slave_done", "sw_align"]
 
 
 def lib():
@@ -141,6 +147,10 @@ def lib():
     L.sw_slave_is_finished.argtypes = [ctypes.c_void_p, ctypes.c_int32]
     L.sw_slave_is_finished.restype = ctypes.c_int32
     L.sw_slave_done.argtypes = [ctypes.c_void_p]
+    L.sw_align.argtypes = [P(sw_seqset), ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32,
+                           ctypes.c_int32, P(ctypes.c_int32), P(ctypes.c_int32), ctypes.c_int32,
+                           P(sw_alignment), ctypes.c_char_p, ctypes.c_int64]
+    L.sw_align.restype = ctypes.c_int
     _lib = L
     return L
 
@@ -186,6 +196,7 @@ class Database:
             _check(lib().sw_db_create(ctypes.byref(ss), None, 0, ctypes.byref(h)))
         self._h = h
         self.n = db.n
+        self.lengths = np.diff(np.asarray(db.offsets)).astype(np.int64)
         self.devices = list(devices) if devices else [0]
 
     def close(self):
@@ -256,6 +267,33 @@ class Database:
         hs = hits[..., 0] if hits is not None else None
         hi = hits[..., 1] if hits is not None else None
         return SearchResult(scores, hs, hi, _stats_dict(st))
+
+    def align(self, queries, query_index, db_index, matrix=None, gap_open=10, gap_extend=2):
+        """Phase 2 (sw_align): the optimal local alignment of each (query, db) pair.
+        Returns a list of dicts: score, q_begin, q_end, d_begin, d_end (0-based, end
+        exclusive) and ops ('M' aligned pair, 'I' query residue vs gap, 'D' db residue vs gap)."""
+        keep = []
+        qs = _seqset(queries, keep)
+        qi = np.ascontiguousarray(query_index, dtype=np.int32)
+        di = np.ascontiguousarray(db_index, dtype=np.int32)
+        n = len(qi)
+        out = (sw_alignment * max(n, 1))()
+        qlen = np.diff(np.asarray(queries.offsets))
+        cap = int(qlen[qi].sum() + self.lengths[di].sum()) if n else 1
+        buf = ctypes.create_string_buffer(max(cap, 1))
+        mat = None
+        if matrix is not None:
+            mat = np.ascontiguousarray(np.asarray(matrix, dtype=np.int8).reshape(24, 24))
+        _check(lib().sw_align(ctypes.byref(qs), self._h, mat.ctypes.data if mat is not None else None,
+                              gap_open, gap_extend, qi.ctypes.data_as(ctypes.POINTER(ctypes.c_int32)),
+                              di.ctypes.data_as(ctypes.POINTER(ctypes.c_int32)), n, out, buf, cap))
+        res = []
+        raw = buf.raw
+        for k in range(n):
+            a = out[k]
+            res.append(dict(score=a.score, q_begin=a.q_begin, q_end=a.q_end, d_begin=a.d_begin,
+                            d_end=a.d_end, ops=raw[a.ops_offset:a.ops_offset + a.n_ops].decode()))
+        return res
 
     def topk_device(self, scores_dev, top_k):
         """Top-k of a torch CUDA score matrix (entries < 0 ignored) -> (scores, index)."""

@@ -837,4 +837,110 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
   return rc;
 }
 
+int sw_align(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t gap_open,
+             int32_t gap_extend, const int32_t *query_index, const int32_t *db_index, int32_t n_pairs,
+             sw_alignment *out, char *ops, int64_t ops_capacity) {
+  if (db && db->busy.exchange(1)) {
+    g_err = "a search is already running on this sw_db";
+    return SW_EBUSY;
+  }
+  int rc = guarded([&] {
+    if (!db || db->devs.empty()) throw Error(SW_EINVAL, "db is NULL");
+    validate_seqset(queries, "queries");
+    if (gap_open < 0 || gap_extend < 0) throw Error(SW_EINVAL, "gap penalties must be >= 0");
+    if ((int64_t)gap_open + 2 * (int64_t)gap_extend > (1 << 20))
+      throw Error(SW_EINVAL, "gap_open + 2*gap_extend must be <= 2^20");
+    if (n_pairs < 0) throw Error(SW_EINVAL, "n_pairs < 0");
+    if (n_pairs == 0) return;
+    if (!query_index || !db_index || !out) throw Error(SW_EINVAL, "NULL pair or output array");
+    const PackedDB &Hd = db->host;
+    const int8_t *M = matrix ? matrix : blosum62();
+    // inverse of the length sort: original -> sorted index
+    std::vector<int32_t> inv(Hd.n);
+    for (int32_t k = 0; k < Hd.n; k++) inv[Hd.perm[k]] = k;
+    // encode the queries
+    const int32_t nq = queries->n;
+    std::vector<int64_t> qoff(nq + 1, 0);
+    for (int32_t k = 0; k < nq; k++) qoff[k + 1] = qoff[k] + (queries->offsets[k + 1] - queries->offsets[k]);
+    std::vector<uint8_t> qc(std::max<int64_t>(qoff[nq], 1));
+    for (int32_t k = 0; k < nq; k++)
+      for (int64_t p = 0; p < qoff[k + 1] - qoff[k]; p++) {
+        const int c = encode_residue((unsigned char)queries->residues[queries->offsets[k] + p]);
+        if (c < 0) throw Error(SW_ERESIDUE, "query " + std::to_string(k) + ": invalid residue at position " + std::to_string(p));
+        qc[qoff[k] + p] = (uint8_t)c;
+      }
+    int64_t need = 0;
+    for (int32_t k = 0; k < n_pairs; k++) {
+      if (query_index[k] < 0 || query_index[k] >= nq || db_index[k] < 0 || db_index[k] >= Hd.n)
+        throw Error(SW_EINVAL, "pair " + std::to_string(k) + ": index out of range");
+      need += (qoff[query_index[k] + 1] - qoff[query_index[k]]) + Hd.sorted_len[inv[db_index[k]]];
+    }
+    if (!ops || ops_capacity < need)
+      throw Error(SW_EINVAL, "ops buffer too small: need " + std::to_string(need) + " bytes");
+    Device &D = *db->devs[0];
+    CK(cudaSetDevice(D.id));
+    DBuf<uint8_t> dq; dq.alloc(D.id, qc.size());
+    CK(cudaMemcpy(dq.p, qc.data(), qc.size(), cudaMemcpyHostToDevice));
+    DBuf<int8_t> dm; dm.alloc(D.id, 24 * 24);
+    CK(cudaMemcpy(dm.p, M, 24 * 24, cudaMemcpyHostToDevice));
+    const int64_t kBudget = int64_t(2) << 30;   // direction bytes per batch
+    int64_t ops_pos = 0;
+    for (int32_t p0 = 0; p0 < n_pairs;) {
+      std::vector<TbPair> batch;
+      int64_t dir_total = 0, ops_total = 0;
+      int32_t max_n = 1;
+      int32_t p1 = p0;
+      while (p1 < n_pairs) {
+        TbPair T;
+        T.m = (int32_t)(qoff[query_index[p1] + 1] - qoff[query_index[p1]]);
+        T.sorted = inv[db_index[p1]];
+        T.n = Hd.sorted_len[T.sorted];
+        const int64_t cells = (int64_t)T.m * T.n;
+        if (!batch.empty() && dir_total + cells > kBudget) break;
+        T.q_off = qoff[query_index[p1]];
+        T.pad_ = 0;
+        T.dir_off = dir_total;
+        T.ops_off = ops_total;
+        dir_total += cells;
+        ops_total += T.m + T.n;
+        max_n = std::max(max_n, T.n);
+        batch.push_back(T);
+        p1++;
+      }
+      const int nb = (int)batch.size();
+      DBuf<TbPair> dp; dp.alloc(D.id, nb);
+      CK(cudaMemcpy(dp.p, batch.data(), sizeof(TbPair) * nb, cudaMemcpyHostToDevice));
+      DBuf<uint8_t> ddir; ddir.alloc(D.id, std::max<int64_t>(dir_total, 1));
+      DBuf<char> dops; dops.alloc(D.id, std::max<int64_t>(ops_total, 1));
+      DBuf<TbResult> dres; dres.alloc(D.id, nb);
+      DBuf<int32_t> dborder; dborder.alloc(D.id, (size_t)nb * max_n * 2);
+      TbArgs a;
+      a.qcodes = dq.p; a.packed = D.packed.p; a.groups = D.groups.p; a.matrix = dm.p;
+      a.pairs = dp.p; a.dir = ddir.p; a.ops = dops.p; a.results = dres.p;
+      a.border = dborder.p; a.border_stride = max_n;
+      a.alpha = gap_open + gap_extend; a.beta = gap_extend;
+      launch_traceback(a, nb, 0);
+      CK(cudaGetLastError());
+      CK(cudaDeviceSynchronize());
+      std::vector<TbResult> res(nb);
+      std::vector<char> hops(std::max<int64_t>(ops_total, 1));
+      CK(cudaMemcpy(res.data(), dres.p, sizeof(TbResult) * nb, cudaMemcpyDeviceToHost));
+      CK(cudaMemcpy(hops.data(), dops.p, ops_total, cudaMemcpyDeviceToHost));
+      for (int k = 0; k < nb; k++) {
+        const TbPair &T = batch[k];
+        const TbResult &R = res[k];
+        sw_alignment &A = out[p0 + k];
+        A.score = R.score; A.q_begin = R.q_begin; A.q_end = R.q_end;
+        A.d_begin = R.d_begin; A.d_end = R.d_end; A.n_ops = R.n_ops;
+        A.ops_offset = ops_pos;
+        std::memcpy(ops + ops_pos, hops.data() + T.ops_off + (T.m + T.n) - R.n_ops, R.n_ops);
+        ops_pos += R.n_ops;
+      }
+      p0 = p1;
+    }
+  });
+  if (db) db->busy.store(0);
+  return rc;
+}
+
 }  // extern "C"

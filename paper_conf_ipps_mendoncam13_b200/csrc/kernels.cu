@@ -670,6 +670,125 @@ void launch_k2(const K2Args &a, int blocks, cudaStream_t st) {
 }
 
 // ------------------------------------------------------------------------------------
+// K6: Phase 2 (P12 §II.A.2, NEXT-3): direction bytes + traceback of selected pairs.
+// One warp per pair, int32, the same wavefront as K2 (lane l owns rows [l*R, (l+1)*R) of
+// each 32*R-row chunk).  Byte per cell: bits 0-1 = H source (0 zero, 1 diagonal, 2 E,
+// 3 F), bit 2 = E extends E(i,j-1), bit 3 = F extends F(i-1,j).  The highest cell (ties:
+// smallest row, then smallest column) is found by a warp reduction; lane 0 then follows
+// the arrows back to a zero, writing ops ('M', 'I', 'D') backwards.
+// ------------------------------------------------------------------------------------
+constexpr int K6R = 8;
+__global__ void __launch_bounds__(32) traceback_kernel(const TbArgs a) {
+  __shared__ int32_t Ms[kNCodes * 32];
+  for (int k = threadIdx.x; k < kNCodes * 32; k += 32) {
+    const int r = k / 32, c = k % 32;
+    Ms[k] = (r < 24 && c < 24) ? (int32_t)a.matrix[r * 24 + c] : kPadScore;
+  }
+  __syncwarp();
+  const int lane = threadIdx.x;
+  const TbPair T = a.pairs[blockIdx.x];
+  const int m = T.m, n = T.n;
+  const uint8_t *qc = a.qcodes + T.q_off;
+  const GroupInfo G = a.groups[T.sorted / kGroup];
+  const int gl = T.sorted % kGroup;
+  const uint8_t *bytes = reinterpret_cast<const uint8_t *>(a.packed);
+  uint8_t *dir = a.dir + T.dir_off;
+  int32_t *border = a.border + (size_t)blockIdx.x * a.border_stride * 2;
+  constexpr int NEG = -(1 << 29);
+  int bv = 0, bi = 0, bj = 0;   // best value and its 1-based cell (0,0 = empty alignment)
+  const int nch = (m + 32 * K6R - 1) / (32 * K6R);
+  for (int ch = 0; ch < nch; ch++) {
+    int qr[K6R];
+#pragma unroll
+    for (int i = 0; i < K6R; i++) {
+      const int row = ch * 32 * K6R + lane * K6R + i;
+      qr[i] = row < m ? qc[row] : kPadCode;
+    }
+    int H[K6R], E[K6R];
+#pragma unroll
+    for (int i = 0; i < K6R; i++) { H[i] = 0; E[i] = NEG; }
+    int hprev_top = 0, out_h = 0, out_f = NEG, out_c = kPadCode;
+    for (int t = 0; t < n + 31; t++) {
+      int in_h = __shfl_up_sync(0xffffffffu, out_h, 1);
+      int in_f = __shfl_up_sync(0xffffffffu, out_f, 1);
+      int in_c = __shfl_up_sync(0xffffffffu, out_c, 1);
+      if (lane == 0 && t < n) {
+        in_c = bytes[(G.word_off + (int64_t)(t >> 4) * kGroup + gl) * 16 + (t & 15)];
+        if (ch == 0) { in_h = 0; in_f = NEG; }
+        else { in_h = border[2 * t]; in_f = border[2 * t + 1]; }
+      }
+      const int col = t - lane;
+      if (col >= 0 && col < n) {
+        int hd = hprev_top, hup = in_h, f = in_f;
+        hprev_top = in_h;
+#pragma unroll
+        for (int i = 0; i < K6R; i++) {
+          const int row = ch * 32 * K6R + lane * K6R + i;   // 0-based query row
+          const int eo = H[i] - a.alpha, ee = E[i] - a.beta;
+          const int e = max(ee, eo);                        // E(i,j)
+          const int fo = hup - a.alpha, fe = f - a.beta;
+          f = max(fe, fo);                                  // F(i,j)
+          const int dg = hd + Ms[qr[i] * 32 + in_c];        // diagonal
+          int h = max(max(dg, e), max(f, 0));               // H(i,j)
+          if (row < m) {
+            const int src = h == 0 ? 0 : h == dg ? 1 : h == e ? 2 : 3;
+            dir[(size_t)row * n + col] = (uint8_t)(src | ((ee > eo) << 2) | ((fe > fo) << 3));
+            if (h > bv || (h == bv && h > 0 && (row + 1 < bi || (row + 1 == bi && col + 1 < bj)))) {
+              bv = h; bi = row + 1; bj = col + 1;
+            }
+          }
+          hd = H[i]; H[i] = h; E[i] = e; hup = h;
+        }
+        out_h = H[K6R - 1]; out_f = f; out_c = in_c;
+        if (lane == 31 && ch < nch - 1) { border[2 * col] = out_h; border[2 * col + 1] = out_f; }
+      }
+    }
+  }
+  // warp reduction of (value desc, row asc, column asc)
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    const int v2 = __shfl_xor_sync(0xffffffffu, bv, o), i2 = __shfl_xor_sync(0xffffffffu, bi, o),
+              j2 = __shfl_xor_sync(0xffffffffu, bj, o);
+    if (v2 > bv || (v2 == bv && (i2 < bi || (i2 == bi && j2 < bj)))) { bv = v2; bi = i2; bj = j2; }
+  }
+  __syncwarp();
+  if (lane != 0) return;
+  TbResult R;
+  R.score = bv;
+  int k = 0;
+  char *ops_end = a.ops + T.ops_off + (m + n);   // ops written backwards from here
+  int i = bi, j = bj, state = 0;                 // 0 = H, 1 = E, 2 = F
+  if (bv > 0) {
+    while (i > 0 && j > 0) {
+      const uint8_t b = dir[(size_t)(i - 1) * n + (j - 1)];
+      if (state == 0) {
+        const int src = b & 3;
+        if (src == 0) break;
+        if (src == 1) { *(--ops_end) = 'M'; k++; i--; j--; }
+        else state = src == 2 ? 1 : 2;
+      } else if (state == 1) {
+        *(--ops_end) = 'D'; k++;
+        state = (b >> 2) & 1 ? 1 : 0;
+        j--;
+      } else {
+        *(--ops_end) = 'I'; k++;
+        state = (b >> 3) & 1 ? 2 : 0;
+        i--;
+      }
+    }
+    R.q_begin = i; R.q_end = bi; R.d_begin = j; R.d_end = bj;
+  } else {
+    R.q_begin = R.q_end = R.d_begin = R.d_end = 0;
+  }
+  R.n_ops = k;
+  a.results[blockIdx.x] = R;
+}
+
+void launch_traceback(const TbArgs &a, int n_pairs, cudaStream_t st) {
+  if (n_pairs > 0) traceback_kernel<<<n_pairs, 32, 0, st>>>(a);
+}
+
+// ------------------------------------------------------------------------------------
 // helpers
 // ------------------------------------------------------------------------------------
 __global__ void fill_kernel(int32_t *p, int64_t n, int32_t v) {

@@ -101,6 +101,23 @@ struct K2Args {   // int32 re-run of saturated pairs (warp per pair)
   int32_t *border; int64_t border_stride; int32_t n_warps_total;
 };
 
+struct TbPair {     // one pair of a traceback batch
+  int32_t m, n;      // query and database lengths
+  int64_t q_off;     // query codes offset
+  int32_t sorted;    // database sequence (sorted order)
+  int32_t pad_;
+  int64_t dir_off;   // direction bytes (m*n) offset in the batch buffer
+  int64_t ops_off;   // ops area (m+n bytes) offset in the batch buffer
+};
+struct TbResult { int32_t score, q_begin, q_end, d_begin, d_end, n_ops; };
+struct TbArgs {
+  const uint8_t *qcodes; const uint4 *packed; const GroupInfo *groups; const int8_t *matrix;
+  const TbPair *pairs; uint8_t *dir; char *ops; TbResult *results;
+  int32_t *border; int64_t border_stride;
+  int32_t alpha, beta;
+};
+void launch_traceback(const TbArgs &a, int n_pairs, cudaStream_t st);
+
 void launch_profile(const uint8_t *qcodes, const int64_t *qoff, const QueryPair *pairs, int npairs,
                     const int8_t *matrix, int32_t *prof, int64_t prof_total, cudaStream_t st);
 void launch_k1(const K1Args &a, int n_groups, int min_cols, int rows_padded, cudaStream_t st,

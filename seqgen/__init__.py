@@ -285,6 +285,8 @@ def make_workload(name: str, n_db: int | None = None, n_queries: int | None = No
     if name == "C5":
         # embed each query inside a long DB sequence (keeps lengths in [10k, 35k])
         for k, q in enumerate(qs):
+            if used >= nd:
+                break
             slot = int(slot_order[used]); used += 1
             L = int(lens[slot])
             flank = residues(stream_seed(seed, f"flank{k}"), 0, max(0, L - len(q)))

@@ -270,3 +270,79 @@ def test_c5_full_size_sampled():
     ref = oracle.pairs(w.queries, w.db, qi, di)
     assert (np.asarray(r.scores)[qi, di] == ref).all()
     assert ref.max() > 32767
+
+
+def _check_alignment(q, d, a, M=None, go=10, ge=2):
+    """An alignment from sw_align is valid and optimal: its ops consume exactly the
+    reported substrings and the oracle's alignment scorer gives the pair's SW score."""
+    ops = a["ops"]
+    assert ops.count("M") + ops.count("I") == a["q_end"] - a["q_begin"]
+    assert ops.count("M") + ops.count("D") == a["d_end"] - a["d_begin"]
+    if a["score"] == 0:
+        assert ops == ""
+        return
+    rq, rd, i, j = [], [], a["q_begin"], a["d_begin"]
+    for op in ops:
+        if op == "M":
+            rq.append(q[i]); rd.append(d[j]); i += 1; j += 1
+        elif op == "I":
+            rq.append(q[i]); rd.append("-"); i += 1
+        else:
+            rq.append("-"); rd.append(d[j]); j += 1
+    assert oracle.alignment_score("".join(rq), "".join(rd), M, go, ge) == a["score"]
+    if go + ge > 0:
+        assert ops[0] == "M" and ops[-1] == "M"
+
+
+def test_traceback_phase2():
+    """NEXT-3 (P12 §II.A.2 Phase 2): alignments of the top hits and of random pairs."""
+    qs, db = _mixed_case(71, nq=8, nd=400, max_len=2500)
+    D = Database(db)
+    r = D.search(qs, top_k=3)
+    qi = np.repeat(np.arange(qs.n), 3)
+    di = np.asarray(r.hit_index).reshape(-1)
+    rng = np.random.default_rng(3)
+    qi = np.concatenate([qi, rng.integers(0, qs.n, 40)]).astype(np.int32)
+    di = np.concatenate([di, rng.integers(0, db.n, 40)]).astype(np.int32)
+    keep = di >= 0
+    qi, di = qi[keep], di[keep]
+    al = D.align(qs, qi, di)
+    ref = oracle.pairs(qs, db, qi, di)
+    for k, a in enumerate(al):
+        assert a["score"] == ref[k]
+        _check_alignment(qs.seq(int(qi[k])).decode(), db.seq(int(di[k])).decode(), a)
+    # Fig. 2 through Phase 2: the printed local alignment score 3 (P12/P14)
+    M = np.full((24, 24), -1, np.int8)
+    np.fill_diagonal(M, 1)
+    D2 = Database(seqgen.SeqSet.from_list(["GCTGACCT"]))
+    a = D2.align(seqgen.SeqSet.from_list(["GAAGCTA"]), [0], [0], matrix=M, gap_open=0, gap_extend=2)[0]
+    assert a["score"] == 3
+    _check_alignment("GAAGCTA", "GCTGACCT", a, M, 0, 2)
+    D.close(); D2.close()
+
+
+def test_traceback_long_and_asymmetric():
+    """Phase 2 on long sequences (several 256-row chunks, 10k+ columns) and with an
+    asymmetric matrix (query residue = row)."""
+    w = seqgen.make_workload("C5", n_db=10)
+    D = Database(w.db)
+    qi = np.array([p["query"] for p in w.meta["planted"]] + [0, 1], np.int32)
+    di = np.array([p["slot"] for p in w.meta["planted"]] + [3, 5], np.int32)
+    al = D.align(w.queries, qi, di)
+    ref = oracle.pairs(w.queries, w.db, qi, di)
+    for k, a in enumerate(al):
+        assert a["score"] == ref[k]
+        _check_alignment(w.queries.seq(int(qi[k])).decode(), w.db.seq(int(di[k])).decode(), a)
+    D.close()
+    M = seqgen.random_matrix(9, lo=-6, hi=9)
+    M[2, 7] = 25
+    qs, db = _mixed_case(81, nq=4, nd=60, max_len=700)
+    D = Database(db)
+    qi = np.repeat(np.arange(qs.n), 15).astype(np.int32)
+    di = np.tile(np.arange(15), qs.n).astype(np.int32)
+    al = D.align(qs, qi, di, matrix=M, gap_open=4, gap_extend=3)
+    ref = oracle.pairs(qs, db, qi, di, matrix=M, gap_open=4, gap_extend=3)
+    for k, a in enumerate(al):
+        assert a["score"] == ref[k]
+        _check_alignment(qs.seq(int(qi[k])).decode(), db.seq(int(di[k])).decode(), a, M, 4, 3)
+    D.close()
