@@ -581,6 +581,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
     std::vector<UnitLog> ulog;
     std::mutex ulog_mu;
     std::atomic<int> ready{0};
+    std::atomic<bool> failed{false};   // a worker failed: the others stop (no hang on its units)
     std::vector<std::string> werr(nW);
     std::vector<int> wcode(nW, 0);
     const double t0 = now_s();
@@ -617,6 +618,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         double last_report = now_s();
         int32_t buf[64];
         while (true) {
+          if (failed.load()) throw Error(SW_ECUDA, "another worker failed");
           bool progressed = false;
           const double tn = now_s();
           // completions
@@ -720,16 +722,21 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       } catch (const Error &e) {
         werr[w] = e.what();
         wcode[w] = e.code;
+        failed.store(true);
         ready.fetch_add(1 << 20);  // release the barrier
       } catch (const std::exception &e) {
         werr[w] = e.what();
         wcode[w] = SW_ECUDA;
+        failed.store(true);
         ready.fetch_add(1 << 20);
       }
     };
     std::vector<std::thread> threads;
     for (int w = 0; w < nW; w++) threads.emplace_back(worker, w);
     for (auto &t : threads) t.join();
+    for (int w = 0; w < nW; w++)
+      if (wcode[w] && werr[w] != "another worker failed")
+        throw Error(wcode[w], "worker " + std::to_string(w) + ": " + werr[w]);
     for (int w = 0; w < nW; w++)
       if (wcode[w]) throw Error(wcode[w], "worker " + std::to_string(w) + ": " + werr[w]);
     if (client) client->done();
