@@ -102,6 +102,7 @@ struct DevSearch {
   DBuf<uint8_t> qcodes;
   DBuf<int64_t> qoff;
   DBuf<QueryPair> pairs;
+  DBuf<SliceInfo> slices;
   DBuf<int8_t> matrix;
   DBuf<int32_t> prof;
   DBuf<int32_t> scores_own;
@@ -170,7 +171,9 @@ namespace sw {
 
 // ---------------------------------------------------------------- search plan
 struct Plan {
-  std::vector<QueryPair> pairs;
+  std::vector<QueryPair> pairs;       // query packs
+  std::vector<SliceInfo> slices;      // all packs' slice tables
+  std::vector<int64_t> real_rows;     // per pack: sum of its query lengths
   std::vector<uint8_t> qcodes;
   std::vector<int64_t> qoff;
   std::vector<Unit> units;
@@ -214,23 +217,66 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
                                      "' at position " + std::to_string(p));
       P.qcodes[P.qoff[k] + p] = (uint8_t)c;
     }
-  // query pairs: sort by length (descending), pair neighbours (two queries per s16x2 lane)
+  // query packs (sw_internal.h): 2*NP half-streams of queries, each query starting on a
+  // 16-row slice; queries (longest first) go to the least loaded half (LPT), halves are
+  // paired by load.  NP ~ total rows / (2 x longest query), so a half is about as long as
+  // the longest query and the halves of a pack differ by little.
   std::vector<int32_t> qo(nq);
   std::iota(qo.begin(), qo.end(), 0);
   std::stable_sort(qo.begin(), qo.end(), [&](int32_t a, int32_t b) {
     return P.qoff[a + 1] - P.qoff[a] > P.qoff[b + 1] - P.qoff[b];
   });
+  auto c16 = [](int64_t x) { return (x + 15) / 16 * 16; };
+  int64_t tot16 = 0, max16 = 16;
+  for (int32_t k = 0; k < nq; k++) {
+    const int64_t l = P.qoff[k + 1] - P.qoff[k];
+    tot16 += c16(std::max<int64_t>(l, 1));
+    max16 = std::max(max16, c16(l));
+  }
+  int32_t np = nq == 0 ? 0 : (int32_t)std::max<int64_t>(1, (tot16 + max16) / (2 * max16));
+  np = std::min(np, std::max(1, (nq + 1) / 2));
+  struct Half { int64_t load = 0; std::vector<int32_t> q; };
+  std::vector<Half> halves(2 * np);
+  for (int32_t k = 0; k < nq; k++) {   // LPT into 2*np halves (first least-loaded wins)
+    const int32_t q = qo[k];
+    int32_t h = 0;
+    for (int32_t j = 1; j < 2 * np; j++)
+      if (halves[j].load < halves[h].load) h = j;
+    halves[h].q.push_back(q);
+    halves[h].load += c16(std::max<int64_t>(P.qoff[q + 1] - P.qoff[q], 1));
+  }
+  std::stable_sort(halves.begin(), halves.end(),
+                   [](const Half &a, const Half &b) { return a.load > b.load; });
   int64_t prof = 0;
-  for (int32_t k = 0; k < nq; k += 2) {
+  P.real_rows.clear();
+  for (int32_t k = 0; k < np; k++) {
+    const Half &lo = halves[2 * k], &hi = halves[2 * k + 1];
     QueryPair qp;
-    qp.qa = qo[k];
-    qp.qb = (k + 1 < nq) ? qo[k + 1] : -1;
-    qp.la = (int32_t)(P.qoff[qp.qa + 1] - P.qoff[qp.qa]);
-    qp.lb = qp.qb >= 0 ? (int32_t)(P.qoff[qp.qb + 1] - P.qoff[qp.qb]) : 0;
-    const int32_t rows = std::max(qp.la, 1);
-    qp.rows_padded = (rows + kProfileRowAlign - 1) / kProfileRowAlign * kProfileRowAlign;
+    qp.rows = (int32_t)std::max<int64_t>(std::max(lo.load, hi.load), 16);
+    qp.rows_padded = (qp.rows + kProfileRowAlign - 1) / kProfileRowAlign * kProfileRowAlign;
     qp.prof_off = prof;
+    qp.slice_off = (int32_t)P.slices.size();
+    qp.pad_ = 0;
     prof += (int64_t)kNCodes * qp.rows_padded;
+    const int32_t ns = qp.rows_padded / 16;
+    std::vector<SliceInfo> sl(ns, SliceInfo{-1, 0, -1, 0});
+    int64_t real = 0;
+    for (int half = 0; half < 2; half++) {
+      int64_t row = 0;
+      for (int32_t q : (half == 0 ? lo : hi).q) {
+        const int64_t l = P.qoff[q + 1] - P.qoff[q];
+        real += l;
+        const int64_t span = c16(std::max<int64_t>(l, 1));
+        for (int64_t r = 0; r < span; r += 16) {
+          SliceInfo &x = sl[(row + r) / 16];
+          if (half == 0) { x.q_lo = q; x.off_lo = (int32_t)r; }
+          else { x.q_hi = q; x.off_hi = (int32_t)r; }
+        }
+        row += span;
+      }
+    }
+    P.slices.insert(P.slices.end(), sl.begin(), sl.end());
+    P.real_rows.push_back(real);
     P.pairs.push_back(qp);
   }
   P.prof_total = prof;
@@ -249,7 +295,7 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
   for (int32_t g = 0; g < ng; g++)
     for (int32_t k = 0; k < db.groups[g].count; k++) grp_res[g] += db.sorted_len[db.groups[g].first + k];
   int64_t total_cells = 0;
-  for (auto &qp : P.pairs) total_cells += (int64_t)(qp.la + qp.lb) * db.residues;
+  for (int64_t r : P.real_rows) total_cells += r * db.residues;
   P.cells = total_cells;
   int64_t target = o.target_unit_cells;
   const int depth = std::max(1, o.streams_per_device);
@@ -260,7 +306,7 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
   }
   for (int32_t p = 0; p < (int32_t)P.pairs.size(); p++) {
     const QueryPair &qp = P.pairs[p];
-    const int64_t rows_eff = (int64_t)qp.la + qp.lb;
+    const int64_t rows_eff = P.real_rows[p];
     // K3 units over the long sequences (multiples of kK3Warps)
     for (int32_t s = 0; s < P.n_long_seqs;) {
       int32_t e = s;
@@ -276,7 +322,7 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
     }
     // K1 units over the short groups
     const int64_t band = k1_band_rows();
-    const int64_t rows_k1 = (int64_t)(std::max(qp.la, 1) + band - 1) / band * band;
+    const int64_t rows_k1 = (int64_t)(qp.rows + band - 1) / band * band;
     for (int32_t g = gl; g < ng;) {
       int32_t e = g;
       int64_t cells = 0, work = 0;
@@ -322,7 +368,7 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
   if (U.kind == kUnitInter) {
     K1Args a;
     a.packed = D.packed.p; a.groups = D.groups.p; a.perm = D.perm.p;
-    a.prof = S.prof.p; a.pairs = S.pairs.p;
+    a.prof = S.prof.p; a.pairs = S.pairs.p; a.slices = S.slices.p;
     a.pair = U.pair; a.g0 = U.b0;
     a.scores = S.scores; a.ndb = db.n;
     a.thresh = thresh;
@@ -335,7 +381,7 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
   } else {
     K3Args a;
     a.packed = D.packed.p; a.groups = D.groups.p; a.perm = D.perm.p; a.sorted_len = D.sorted_len.p;
-    a.prof = S.prof.p; a.pairs = S.pairs.p;
+    a.prof = S.prof.p; a.pairs = S.pairs.p; a.slices = S.slices.p;
     a.pair = U.pair; a.l0 = U.b0; a.l1 = U.b1;
     a.scores = S.scores; a.ndb = db.n;
     a.thresh = thresh;
@@ -504,6 +550,8 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       if (!P.qcodes.empty()) CK(cudaMemcpy(X.qcodes.p, P.qcodes.data(), P.qcodes.size(), cudaMemcpyHostToDevice));
       CK(cudaMemcpy(X.qoff.p, P.qoff.data(), sizeof(int64_t) * P.qoff.size(), cudaMemcpyHostToDevice));
       if (!P.pairs.empty()) CK(cudaMemcpy(X.pairs.p, P.pairs.data(), sizeof(QueryPair) * P.pairs.size(), cudaMemcpyHostToDevice));
+      X.slices.ensure(D.id, P.slices.size());
+      if (!P.slices.empty()) CK(cudaMemcpy(X.slices.p, P.slices.data(), sizeof(SliceInfo) * P.slices.size(), cudaMemcpyHostToDevice));
       CK(cudaMemcpy(X.matrix.p, M, 24 * 24, cudaMemcpyHostToDevice));
       const size_t nsc = (size_t)nq * nd;
       if (w == 0 && o.outputs_on_device && scores && !dist) X.scores = scores;
@@ -599,8 +647,8 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         CK(cudaEventRecord(X.ev_start, s0));
         launch_fill(X.scores, (int64_t)nq * nd, -1, s0);
         CK(cudaMemsetAsync(X.ovf_count.p, 0, sizeof(int32_t), s0));
-        launch_profile(X.qcodes.p, X.qoff.p, X.pairs.p, (int)P.pairs.size(), X.matrix.p, X.prof.p,
-                       P.prof_total, s0);
+        launch_profile(X.qcodes.p, X.qoff.p, X.pairs.p, (int)P.pairs.size(), X.slices.p, X.matrix.p,
+                       X.prof.p, P.prof_total, s0);
         X.launches += 2 + (P.pairs.empty() ? 0 : 1);
         CK(cudaGetLastError());
         cudaEvent_t setup_done;

@@ -61,27 +61,35 @@ __device__ __forceinline__ uint32_t smid() {
 // S_a = S[qa_row][c] (kPadScore past the end of qa or for the pad code), same for qb.
 // ------------------------------------------------------------------------------------
 __global__ void profile_kernel(const uint8_t *__restrict__ qcodes, const int64_t *__restrict__ qoff,
-                               const QueryPair *__restrict__ pairs, const int8_t *__restrict__ M,
-                               int32_t *__restrict__ prof) {
+                               const QueryPair *__restrict__ pairs, const SliceInfo *__restrict__ slices,
+                               const int8_t *__restrict__ M, int32_t *__restrict__ prof) {
   const QueryPair P = pairs[blockIdx.y];
   const int64_t n = (int64_t)kNCodes * P.rows_padded;
   for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < n;
        k += (int64_t)gridDim.x * blockDim.x) {
     const int c = (int)(k / P.rows_padded), row = (int)(k % P.rows_padded);
+    const SliceInfo si = slices[P.slice_off + row / 16];
     int sa = kPadScore, sb = kPadScore;
     if (c < 24) {
-      if (row < P.la) sa = M[qcodes[qoff[P.qa] + row] * 24 + c];
-      if (P.qb >= 0 && row < P.lb) sb = M[qcodes[qoff[P.qb] + row] * 24 + c];
+      if (si.q_lo >= 0) {
+        const int64_t r = si.off_lo + row % 16;
+        if (r < qoff[si.q_lo + 1] - qoff[si.q_lo]) sa = M[qcodes[qoff[si.q_lo] + r] * 24 + c];
+      }
+      if (si.q_hi >= 0) {
+        const int64_t r = si.off_hi + row % 16;
+        if (r < qoff[si.q_hi + 1] - qoff[si.q_hi]) sb = M[qcodes[qoff[si.q_hi] + r] * 24 + c];
+      }
     }
     prof[P.prof_off + k] = sb * 65536 + sa;
   }
 }
 
 void launch_profile(const uint8_t *qcodes, const int64_t *qoff, const QueryPair *pairs, int npairs,
-                    const int8_t *matrix, int32_t *prof, int64_t, cudaStream_t st) {
+                    const SliceInfo *slices, const int8_t *matrix, int32_t *prof, int64_t,
+                    cudaStream_t st) {
   if (npairs == 0) return;
   dim3 grid(64, npairs);
-  profile_kernel<<<grid, 256, 0, st>>>(qcodes, qoff, pairs, matrix, prof);
+  profile_kernel<<<grid, 256, 0, st>>>(qcodes, qoff, pairs, slices, matrix, prof);
 }
 
 // ------------------------------------------------------------------------------------
@@ -101,6 +109,27 @@ struct Cell {
     best = __vmaxs2(best, h);
   }
 };
+
+// One half of a lane's running maximum (offset representation) for query q: saturated
+// halves go to the int32 re-run list, the others raise the score with atomicMax (a query
+// spans several warps / lanes / bands, each contributes the maximum over its rows).
+__device__ __forceinline__ void flush_half(int q, int v, int ss, int orig, int32_t *scores,
+                                           int64_t ndb, int thresh, int2 *ovf, int32_t *ovf_count,
+                                           int ovf_cap) {
+  if (q < 0) return;
+  if (v >= thresh) {
+    const int k = atomicAdd(ovf_count, 1);
+    if (k < ovf_cap) ovf[k] = make_int2(q, ss);
+  } else {
+    atomicMax(scores + (int64_t)q * ndb + orig, v - kOff);
+  }
+}
+__device__ __forceinline__ int lo16(uint32_t v) { return (int)(int16_t)(v & 0xffff); }
+__device__ __forceinline__ int hi16(uint32_t v) { return (int)(int16_t)(v >> 16); }
+// half masks of a slice that starts a query (its input row above is reset to H = F = 0)
+__device__ __forceinline__ uint32_t start_mask(const SliceInfo &n) {
+  return (n.q_lo >= 0 && n.off_lo == 0 ? 0x0000ffffu : 0u) | (n.q_hi >= 0 && n.off_hi == 0 ? 0xffff0000u : 0u);
+}
 
 // G consecutive columns of one lane's K rows, skewed by one row per column so the G
 // dependency chains (row i of column g needs row i of column g-1 and row i-1 of column g)
@@ -152,9 +181,8 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   if (block_aborted(a.abort_flag)) return;  // WA: this replica lost the race
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const QueryPair P = a.pairs[a.pair];
-  const int rows = P.la > P.lb ? P.la : P.lb;
-  // >= 1 band even for two empty queries (all rows skipped, scores 0)
-  const int nb = rows > 0 ? (rows + BAND - 1) / BAND : 1;
+  const int rows = P.rows;   // 16-aligned, >= 16
+  const int nb = (rows + BAND - 1) / BAND;
   const uint32_t koff = pk2(kOff), na = a.na, nbeta = a.nb;
   const int32_t *gprof = a.prof + P.prof_off;
   // this block streams through groups gfirst, gfirst + gridDim.x, ... of the unit without
@@ -190,8 +218,12 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   int t_g = gfirst, t_band = 0, t_nt = a.groups[gfirst].ncols / T, t_start = 0, t_B = 0;
   int rl_step = -1, rl_band = 0, rl_slot = 0;
 
-  // per-warp iterator over (group, band, tile)
+  // per-warp iterator over (group, band, tile); the queries of this warp's current slice
+  // (per half) and the start mask of the slice below it
   int g = gfirst, gk = 0, band = 0, tile = 0, gband = 0;
+  int cq_lo = -1, cq_hi = -1;
+  uint32_t omask = 0;
+  const int nslices = P.rows_padded / 16;
   GroupInfo G = a.groups[g];
   int nt = G.ncols / T, nwords = (G.ncols + kWordCols - 1) / kWordCols, wnext = nwords > 1 ? 1 : 0;
   const uint4 *wp = a.packed + G.word_off + lane;
@@ -231,6 +263,23 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
 #pragma unroll
         for (int i = 0; i < K; i++) { H[i] = koff; E[i] = koff; }
         hprev_top = koff;
+        // this warp's slice in this band: flush a half whose query changed
+        const int sidx = band * W + warp;
+        const SliceInfo si = a.slices[P.slice_off + sidx];
+        if (si.q_lo != cq_lo || si.q_hi != cq_hi) {
+          if (lane < G.count) {
+            const int ss = G.first + lane, orig = a.perm[ss];
+            if (si.q_lo != cq_lo)
+              flush_half(cq_lo, lo16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap);
+            if (si.q_hi != cq_hi)
+              flush_half(cq_hi, hi16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap);
+          }
+          if (si.q_lo != cq_lo) best = (best & 0xffff0000u) | (koff & 0xffffu);
+          if (si.q_hi != cq_hi) best = (best & 0x0000ffffu) | (koff & 0xffff0000u);
+          cq_lo = si.q_lo;
+          cq_hi = si.q_hi;
+        }
+        omask = sidx + 1 < nslices ? start_mask(a.slices[P.slice_off + sidx + 1]) : 0u;
         if (band > 0) {   // new band of the same group: restart at word 0 (prefetched)
           r4 = r4n;
           wnext = nwords > 1 ? 1 : 0;
@@ -286,6 +335,13 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
           hprev_top = v.x;
         }
         dp_tile<K, GS, 1>(prc, H, E, hdc, fc, oh, best, na, nbeta, koff);
+        if (omask) {   // the slice below starts a query: it sees H = F = 0 above
+#pragma unroll
+          for (int j = 0; j < GS; j++) {
+            oh[j] = (oh[j] & ~omask) | (koff & omask);
+            fc[j] = (fc[j] & ~omask) | (koff & omask);
+          }
+        }
 #pragma unroll
         for (int j = 0; j < GS; j++) outp[(q * GS + j) * 32 + lane] = make_uint2(oh[j], fc[j]);
       }
@@ -299,33 +355,13 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
         gband++;
         if (++band == nb) {
           band = 0;
-          uint32_t *rd = red + (gk & 1) * W * 32;
-          rd[warp * 32 + lane] = best;
-          best = koff;
-          if (warp == W - 1) {   // the last warp to finish the group reduces and writes
-            uint32_t m = rd[(W - 1) * 32 + lane];   // this warp's own, just written
-#pragma unroll
-            for (int w = 0; w < W - 1; w++) m = __vmaxs2(m, rd[w * 32 + lane]);
-            if (lane < G.count) {
-              const int ss = G.first + lane;
-              const int orig = a.perm[ss];
-              const int lo = (int)(int16_t)(m & 0xffff), hi = (int)(int16_t)(m >> 16);
-              if (lo >= a.thresh) {
-                const int k = atomicAdd(a.ovf_count, 1);
-                if (k < a.ovf_cap) a.ovf[k] = make_int2(P.qa, ss);
-              } else {
-                a.scores[(int64_t)P.qa * a.ndb + orig] = lo - kOff;
-              }
-              if (P.qb >= 0) {
-                if (hi >= a.thresh) {
-                  const int k = atomicAdd(a.ovf_count, 1);
-                  if (k < a.ovf_cap) a.ovf[k] = make_int2(P.qb, ss);
-                } else {
-                  a.scores[(int64_t)P.qb * a.ndb + orig] = hi - kOff;
-                }
-              }
-            }
+          if (lane < G.count) {   // end of the group: flush both halves
+            const int ss = G.first + lane, orig = a.perm[ss];
+            flush_half(cq_lo, lo16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap);
+            flush_half(cq_hi, hi16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap);
           }
+          best = koff;
+          cq_lo = cq_hi = -1;
           gk++;
           g += gstride;
           if (g < gend) {
@@ -442,8 +478,9 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
   if (block_aborted(a.abort_flag)) return;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const QueryPair P = a.pairs[a.pair];
-  const int rows = P.la > P.lb ? P.la : P.lb;
+  const int rows = P.rows;
   const int nch = (rows + CH - 1) / CH;
+  const int nslices = P.rows_padded / 16;
   const int s = a.l0 + blockIdx.x * kK3Warps + warp;
   const bool valid = s < a.l1;
   const int len = valid ? a.sorted_len[s] : 0;
@@ -455,7 +492,9 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
   const uint32_t padw = 0x01010101u * kPadCode;
   const int32_t *gprof = a.prof + P.prof_off;
   const int ntile = (len + T - 1) / T;   // columns up to ntile*T <= G.ncols carry pad codes
+  const int orig = valid ? a.perm[s] : 0;
   uint32_t best = koff;
+  int cq_lo = -1, cq_hi = -1;   // queries of this lane's slice (per half)
 
   for (int ch = 0; ch < nch; ch++) {
     __syncthreads();
@@ -465,7 +504,26 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
       smem[(c * K + i) * 32 + l] = (uint32_t)__ldg(gprof + (int64_t)c * P.rows_padded + ch * CH + r);
     }
     __syncthreads();
-    if (!valid || len == 0) continue;
+    if (!valid) continue;
+    // lane l's rows of this chunk are slice ch*32 + l: flush a half whose query changed;
+    // the start mask of the slice below applies to what this lane hands down
+    uint32_t omask = 0;
+    {
+      const int sidx = ch * 32 + lane;
+      const SliceInfo si = a.slices[P.slice_off + sidx];
+      if (si.q_lo != cq_lo) {
+        flush_half(cq_lo, lo16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap);
+        best = (best & 0xffff0000u) | (koff & 0xffffu);
+        cq_lo = si.q_lo;
+      }
+      if (si.q_hi != cq_hi) {
+        flush_half(cq_hi, hi16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap);
+        best = (best & 0x0000ffffu) | (koff & 0xffff0000u);
+        cq_hi = si.q_hi;
+      }
+      if (sidx + 1 < nslices) omask = start_mask(a.slices[P.slice_off + sidx + 1]);
+    }
+    if (len == 0) continue;
     uint32_t H[K], E[K];
 #pragma unroll
     for (int i = 0; i < K; i++) { H[i] = koff; E[i] = koff; }
@@ -537,6 +595,11 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
         }
         dp_tile<K, T, 32>(prc, H, E, hdc, out_f, out_h, best, na, nbeta, koff);
 #pragma unroll
+        for (int jj = 0; jj < T; jj++) {   // bit-select: 0 except above a query start
+          out_h[jj] = (out_h[jj] & ~omask) | (koff & omask);
+          out_f[jj] = (out_f[jj] & ~omask) | (koff & omask);
+        }
+#pragma unroll
         for (int q = 0; q < NW; q++) out_c[q] = in_c[q];
         if (lane == 31 && ch < nch - 1)
 #pragma unroll
@@ -544,26 +607,9 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
       }
     }
   }
-  // warp max of best, then the two halves
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) best = __vmaxs2(best, __shfl_xor_sync(0xffffffffu, best, o));
-  if (valid && lane == 0) {
-    const int orig = a.perm[s];
-    const int lo = (int)(int16_t)(best & 0xffff), hi = (int)(int16_t)(best >> 16);
-    if (lo >= a.thresh) {
-      const int k = atomicAdd(a.ovf_count, 1);
-      if (k < a.ovf_cap) a.ovf[k] = make_int2(P.qa, s);
-    } else {
-      a.scores[(int64_t)P.qa * a.ndb + orig] = lo - kOff;
-    }
-    if (P.qb >= 0) {
-      if (hi >= a.thresh) {
-        const int k = atomicAdd(a.ovf_count, 1);
-        if (k < a.ovf_cap) a.ovf[k] = make_int2(P.qb, s);
-      } else {
-        a.scores[(int64_t)P.qb * a.ndb + orig] = hi - kOff;
-      }
-    }
+  if (valid) {   // every lane flushes what it holds
+    flush_half(cq_lo, lo16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap);
+    flush_half(cq_hi, hi16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap);
   }
 }
 

@@ -59,19 +59,30 @@ struct Unit {
   int64_t work;          // padded lane-cells (balancing)
 };
 
-// ---- query pairs ----------------------------------------------------------------------
-struct QueryPair {
-  int32_t qa, qb;        // query indices (qb = -1 if absent)
-  int32_t la, lb;        // lengths
-  int32_t rows_padded;   // rows in the profile (multiple of kProfileRowAlign, >= 1 band)
-  int64_t prof_off;      // offset (in int32) of this pair's profile [kNCodes][rows_padded]
+// ---- query packs ------------------------------------------------------------------------
+// The s16x2 kernels run two query "halves" per 32-bit lane word.  A pack fills each half
+// with a run of queries, every query starting on a 16-row slice boundary (16 = the rows of
+// one K1 warp / one K3 lane), so a short query does not leave the other half idle.  At a
+// slice that starts a query the producer of the row above hands down H = F = 0 for that
+// half, and a warp (K1) or lane (K3) flushes its running maximum of a half whenever the
+// query of its slice changes (atomicMax into the score matrix).
+struct SliceInfo {       // 16 consecutive pack rows
+  int32_t q_lo, off_lo;  // query of the low half (-1 none) and the row of that query at the
+  int32_t q_hi, off_hi;  // slice's first row (0 = the slice starts the query)
+};
+struct QueryPair {       // a pack
+  int32_t rows;          // rows to compute: the longer half (16-aligned)
+  int32_t rows_padded;   // profile rows (multiple of kProfileRowAlign)
+  int64_t prof_off;      // offset (in int32) of this pack's profile [kNCodes][rows_padded]
+  int32_t slice_off;     // first SliceInfo of the pack (rows_padded / 16 entries)
+  int32_t pad_;
 };
 
 // ---- kernel launchers (kernels.cu) -------------------------------------------------------
 struct K1Args {
   const uint4 *packed; const GroupInfo *groups; const int32_t *perm;
-  const int32_t *prof; const QueryPair *pairs;
-  int32_t pair; int32_t g0;          // unit: pair, first group
+  const int32_t *prof; const QueryPair *pairs; const SliceInfo *slices;
+  int32_t pair; int32_t g0;          // unit: pack, first group
   int32_t n_groups;                  // groups [g0, g0 + n_groups) (set by launch_k1)
   int32_t *scores; int64_t ndb;      // [nq][ndb]
   int32_t thresh;                    // overflow threshold on best~ (offset repr)
@@ -82,7 +93,7 @@ struct K1Args {
 };
 struct K3Args {   // sequences [l0,l1) in sorted order (the long groups)
   const uint4 *packed; const GroupInfo *groups; const int32_t *perm; const int32_t *sorted_len;
-  const int32_t *prof; const QueryPair *pairs;
+  const int32_t *prof; const QueryPair *pairs; const SliceInfo *slices;
   int32_t pair; int32_t l0, l1;
   int32_t *scores; int64_t ndb;
   int32_t thresh;
@@ -119,7 +130,8 @@ struct TbArgs {
 void launch_traceback(const TbArgs &a, int n_pairs, cudaStream_t st);
 
 void launch_profile(const uint8_t *qcodes, const int64_t *qoff, const QueryPair *pairs, int npairs,
-                    const int8_t *matrix, int32_t *prof, int64_t prof_total, cudaStream_t st);
+                    const SliceInfo *slices, const int8_t *matrix, int32_t *prof, int64_t prof_total,
+                    cudaStream_t st);
 void launch_k1(const K1Args &a, int n_groups, int min_cols, int rows_padded, cudaStream_t st,
                int n_sm);
 void launch_k3(const K3Args &a, int rows_padded, cudaStream_t st);
