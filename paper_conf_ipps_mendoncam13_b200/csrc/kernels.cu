@@ -524,6 +524,7 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
       if (sidx + 1 < nslices) omask = start_mask(a.slices[P.slice_off + sidx + 1]);
     }
     if (len == 0) continue;
+    const bool any_mask = __any_sync(0xffffffffu, omask != 0);   // warp-uniform
     uint32_t H[K], E[K];
 #pragma unroll
     for (int i = 0; i < K; i++) { H[i] = koff; E[i] = koff; }
@@ -594,10 +595,12 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
           hprev_top = in_h[jj];
         }
         dp_tile<K, T, 32>(prc, H, E, hdc, out_f, out_h, best, na, nbeta, koff);
+        if (any_mask) {   // bit-select: omask is 0 except in a lane above a query start
 #pragma unroll
-        for (int jj = 0; jj < T; jj++) {   // bit-select: 0 except above a query start
-          out_h[jj] = (out_h[jj] & ~omask) | (koff & omask);
-          out_f[jj] = (out_f[jj] & ~omask) | (koff & omask);
+          for (int jj = 0; jj < T; jj++) {
+            out_h[jj] = (out_h[jj] & ~omask) | (koff & omask);
+            out_f[jj] = (out_f[jj] & ~omask) | (koff & omask);
+          }
         }
 #pragma unroll
         for (int q = 0; q < NW; q++) out_c[q] = in_c[q];
