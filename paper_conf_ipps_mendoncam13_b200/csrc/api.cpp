@@ -107,8 +107,11 @@ struct DevSearch {
   DBuf<int32_t> prof;
   DBuf<int32_t> scores_own;
   int32_t *scores = nullptr;
-  DBuf<int2> ovf;
-  DBuf<int32_t> ovf_count;
+  DBuf<int2> ovf;              // [streams][kOvfCap] saturated pairs, one list per stream
+  DBuf<int32_t> ovf_count;     // [streams]
+  DBuf<int32_t> ovf_cursor;    // [streams] entries taken by the int32 re-run
+  DBuf<uint32_t> ovf_bits;     // [nq*ndb] bits: pair already listed
+  int32_t ovf_cap = 0;         // entries per stream list
   DBuf<uint2> k3_border;   // [streams][max_k3_seqs][max_len]
   DBuf<int32_t> k2_border;
   DBuf<int32_t> abort_dev;      // per-unit WA cancellation flags (device memory)
@@ -359,6 +362,26 @@ struct UnitLog {
 
 static const int kOvfCap = 1 << 20;
 
+static const int kK2BlocksPerUnit = 8;   // 32 warps per stream for the int32 re-run
+
+// K2 arguments for the saturated-pair list of one stream
+static K2Args k2_args(const Plan &P, const PackedDB &db, DevSearch &S, int stream_idx, int32_t alpha,
+                      int32_t beta) {
+  Device &D = *S.D;
+  K2Args a;
+  a.qcodes = S.qcodes.p; a.qoff = S.qoff.p;
+  a.packed = D.packed.p; a.groups = D.groups.p; a.sorted_len = D.sorted_len.p; a.perm = D.perm.p;
+  a.matrix = S.matrix.p;
+  a.ovf = S.ovf.p + (size_t)stream_idx * S.ovf_cap; a.ovf_count = S.ovf_count.p + stream_idx;
+  a.ovf_cap = S.ovf_cap; a.ovf_cursor = S.ovf_cursor.p + stream_idx;
+  a.scores = S.scores; a.ndb = db.n; a.alpha = alpha; a.beta = beta;
+  const int64_t stride = std::max<int64_t>(P.max_len, 1);
+  a.border = S.k2_border.p + (size_t)stream_idx * kK2BlocksPerUnit * 4 * stride * 2;
+  a.border_stride = stride;
+  a.n_warps_total = kK2BlocksPerUnit * 4;
+  return a;
+}
+
 static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const Unit &U, int uidx,
                         int stream_idx, int32_t alpha, int32_t beta, int32_t thresh) {
   Device &D = *S.D;
@@ -372,7 +395,8 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     a.pair = U.pair; a.g0 = U.b0;
     a.scores = S.scores; a.ndb = db.n;
     a.thresh = thresh;
-    a.ovf = S.ovf.p; a.ovf_count = S.ovf_count.p; a.ovf_cap = kOvfCap;
+    a.ovf = S.ovf.p + (size_t)stream_idx * S.ovf_cap; a.ovf_count = S.ovf_count.p + stream_idx;
+    a.ovf_cap = S.ovf_cap; a.ovf_bits = S.ovf_bits.p;
     a.border = D.k1_border.p; a.border_slot_cols = D.slot_cols; a.slots_per_sm = D.slots_per_sm;
     a.slot_busy = D.slot_busy.p;
     a.abort_flag = S.abort_d + uidx;
@@ -385,7 +409,8 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     a.pair = U.pair; a.l0 = U.b0; a.l1 = U.b1;
     a.scores = S.scores; a.ndb = db.n;
     a.thresh = thresh;
-    a.ovf = S.ovf.p; a.ovf_count = S.ovf_count.p; a.ovf_cap = kOvfCap;
+    a.ovf = S.ovf.p + (size_t)stream_idx * S.ovf_cap; a.ovf_count = S.ovf_count.p + stream_idx;
+    a.ovf_cap = S.ovf_cap; a.ovf_bits = S.ovf_bits.p;
     const int64_t stride = (std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16;  // >= tiles * T
     a.border = S.k3_border.p + (size_t)stream_idx * P.max_k3_seqs * stride;
     a.border_stride = stride;
@@ -393,6 +418,9 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     a.na = na; a.nb = nbm;
     launch_k3(a, P.pairs[U.pair].rows_padded, st);
   }
+  S.launches++;
+  // int32 re-run of the pairs this unit saturated, on its stream (overlaps other units)
+  launch_k2(k2_args(P, db, S, stream_idx, alpha, beta), kK2BlocksPerUnit, st);
   S.launches++;
 }
 
@@ -556,8 +584,14 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       const size_t nsc = (size_t)nq * nd;
       if (w == 0 && o.outputs_on_device && scores && !dist) X.scores = scores;
       else { X.scores_own.ensure(D.id, nsc); X.scores = X.scores_own.p; }
-      X.ovf.ensure(D.id, kOvfCap);
-      X.ovf_count.ensure(D.id, 1);
+      // saturated-pair lists: 2^20 per stream, or every pair when the s16x2 path is not
+      // usable (alpha + beta > 16384: all pairs are re-scored in int32)
+      X.ovf_cap = s16_ok ? kOvfCap : (int32_t)std::min<int64_t>((int64_t)nq * nd + 1, INT32_MAX / 2);
+      X.ovf.ensure(D.id, (size_t)depth * X.ovf_cap);
+      X.ovf_count.ensure(D.id, depth);
+      X.ovf_cursor.ensure(D.id, depth);
+      X.ovf_bits.ensure(D.id, ((size_t)nq * nd + 31) / 32);
+      X.k2_border.ensure(D.id, (size_t)depth * kK2BlocksPerUnit * 4 * std::max<int64_t>(P.max_len, 1) * 2);
       const size_t k3b = (size_t)depth * std::max(P.max_k3_seqs, 1) *
                          ((std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16);
       if (P.n_long_seqs > 0) X.k3_border.ensure(D.id, k3b);
@@ -646,7 +680,9 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         while (ready.load() < nW) std::this_thread::yield();
         CK(cudaEventRecord(X.ev_start, s0));
         launch_fill(X.scores, (int64_t)nq * nd, -1, s0);
-        CK(cudaMemsetAsync(X.ovf_count.p, 0, sizeof(int32_t), s0));
+        CK(cudaMemsetAsync(X.ovf_count.p, 0, sizeof(int32_t) * depth, s0));
+        CK(cudaMemsetAsync(X.ovf_cursor.p, 0, sizeof(int32_t) * depth, s0));
+        CK(cudaMemsetAsync(X.ovf_bits.p, 0, sizeof(uint32_t) * (((size_t)nq * nd + 31) / 32), s0));
         launch_profile(X.qcodes.p, X.qoff.p, X.pairs.p, (int)P.pairs.size(), X.slices.p, X.matrix.p,
                        X.prof.p, P.prof_total, s0);
         X.launches += 2 + (P.pairs.empty() ? 0 : 1);
@@ -743,25 +779,16 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
           if (!progressed)
             std::this_thread::sleep_for(std::chrono::microseconds(n_inflight > 0 ? 20 : 100));
         }
-        // int32 re-run of saturated pairs (K2), on this device's own list
+        // the per-unit int32 re-runs ran on each stream after its units; check the lists
         for (int k = 0; k < depth; k++) CK(cudaStreamSynchronize(D.streams[k]));
-        int32_t novf = 0;
-        CK(cudaMemcpy(&novf, X.ovf_count.p, sizeof(int32_t), cudaMemcpyDeviceToHost));
-        if (novf > kOvfCap) throw Error(SW_ENOMEM, "overflow list capacity exceeded");
-        X.n_ovf = novf;
-        if (novf > 0) {
-          const int blocks = std::min(1024, (novf + 3) / 4);
-          const int64_t stride = std::max<int64_t>(H.max_len, 1);
-          X.k2_border.ensure(D.id, (size_t)blocks * 4 * stride * 2);
-          K2Args a;
-          a.qcodes = X.qcodes.p; a.qoff = X.qoff.p;
-          a.packed = D.packed.p; a.groups = D.groups.p; a.sorted_len = D.sorted_len.p; a.perm = D.perm.p;
-          a.matrix = X.matrix.p; a.ovf = X.ovf.p; a.ovf_count = X.ovf_count.p;
-          a.scores = X.scores; a.ndb = nd; a.alpha = alpha; a.beta = beta;
-          a.border = X.k2_border.p; a.border_stride = stride; a.n_warps_total = blocks * 4;
-          launch_k2(a, blocks, s0);
-          X.launches++;
-          CK(cudaGetLastError());
+        std::vector<int32_t> novf(depth, 0), ncur(depth, 0);
+        CK(cudaMemcpy(novf.data(), X.ovf_count.p, sizeof(int32_t) * depth, cudaMemcpyDeviceToHost));
+        CK(cudaMemcpy(ncur.data(), X.ovf_cursor.p, sizeof(int32_t) * depth, cudaMemcpyDeviceToHost));
+        X.n_ovf = 0;
+        for (int k = 0; k < depth; k++) {
+          if (novf[k] > X.ovf_cap) throw Error(SW_ENOMEM, "overflow list capacity exceeded");
+          X.n_ovf += novf[k];
+          if (ncur[k] < novf[k]) throw Error(SW_ECUDA, "int32 re-run left saturated pairs");
         }
         CK(cudaEventRecord(X.ev_end, s0));
         CK(cudaEventSynchronize(X.ev_end));

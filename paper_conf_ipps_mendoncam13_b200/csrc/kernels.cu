@@ -115,11 +115,15 @@ struct Cell {
 // spans several warps / lanes / bands, each contributes the maximum over its rows).
 __device__ __forceinline__ void flush_half(int q, int v, int ss, int orig, int32_t *scores,
                                            int64_t ndb, int thresh, int2 *ovf, int32_t *ovf_count,
-                                           int ovf_cap) {
+                                           int ovf_cap, uint32_t *ovf_bits) {
   if (q < 0) return;
-  if (v >= thresh) {
-    const int k = atomicAdd(ovf_count, 1);
-    if (k < ovf_cap) ovf[k] = make_int2(q, ss);
+  if (v >= thresh) {   // several warps / lanes may saturate on one pair: list it once
+    const int64_t bit = (int64_t)q * ndb + orig;
+    const uint32_t m = 1u << (bit & 31);
+    if (!(atomicOr(ovf_bits + (bit >> 5), m) & m)) {
+      const int k = atomicAdd(ovf_count, 1);
+      if (k < ovf_cap) ovf[k] = make_int2(q, ss);
+    }
   } else {
     atomicMax(scores + (int64_t)q * ndb + orig, v - kOff);
   }
@@ -270,9 +274,9 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
           if (lane < G.count) {
             const int ss = G.first + lane, orig = a.perm[ss];
             if (si.q_lo != cq_lo)
-              flush_half(cq_lo, lo16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap);
+              flush_half(cq_lo, lo16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
             if (si.q_hi != cq_hi)
-              flush_half(cq_hi, hi16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap);
+              flush_half(cq_hi, hi16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
           }
           if (si.q_lo != cq_lo) best = (best & 0xffff0000u) | (koff & 0xffffu);
           if (si.q_hi != cq_hi) best = (best & 0x0000ffffu) | (koff & 0xffff0000u);
@@ -357,8 +361,8 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
           band = 0;
           if (lane < G.count) {   // end of the group: flush both halves
             const int ss = G.first + lane, orig = a.perm[ss];
-            flush_half(cq_lo, lo16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap);
-            flush_half(cq_hi, hi16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap);
+            flush_half(cq_lo, lo16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
+            flush_half(cq_hi, hi16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
           }
           best = koff;
           cq_lo = cq_hi = -1;
@@ -512,12 +516,12 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
       const int sidx = ch * 32 + lane;
       const SliceInfo si = a.slices[P.slice_off + sidx];
       if (si.q_lo != cq_lo) {
-        flush_half(cq_lo, lo16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap);
+        flush_half(cq_lo, lo16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
         best = (best & 0xffff0000u) | (koff & 0xffffu);
         cq_lo = si.q_lo;
       }
       if (si.q_hi != cq_hi) {
-        flush_half(cq_hi, hi16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap);
+        flush_half(cq_hi, hi16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
         best = (best & 0x0000ffffu) | (koff & 0xffff0000u);
         cq_hi = si.q_hi;
       }
@@ -611,8 +615,8 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
     }
   }
   if (valid) {   // every lane flushes what it holds
-    flush_half(cq_lo, lo16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap);
-    flush_half(cq_hi, hi16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap);
+    flush_half(cq_lo, lo16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
+    flush_half(cq_hi, hi16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
   }
 }
 
@@ -657,10 +661,23 @@ __global__ void __launch_bounds__(128) k2_kernel(const K2Args a) {
   __syncthreads();
   const int lane = threadIdx.x & 31;
   const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int count = *a.ovf_count;
+  const int count = min(*a.ovf_count, a.ovf_cap);
   const uint8_t *bytes = reinterpret_cast<const uint8_t *>(a.packed);
   constexpr int NEG = -(1 << 29);
-  for (int p = gw; p < count; p += a.n_warps_total) {
+  while (true) {
+    // claim the next entry; the cursor never passes the count (a later re-run on this
+    // stream must still find the entries appended after this one)
+    int p = count;
+    if (lane == 0) {
+      int cur = *(volatile int32_t *)a.ovf_cursor;
+      while (cur < count) {
+        const int seen = atomicCAS(a.ovf_cursor, cur, cur + 1);
+        if (seen == cur) { p = cur; break; }
+        cur = seen;
+      }
+    }
+    p = __shfl_sync(0xffffffffu, p, 0);
+    if (p >= count) break;
     const int q = a.ovf[p].x, s = a.ovf[p].y;
     const int m = (int)(a.qoff[q + 1] - a.qoff[q]);
     const uint8_t *qc = a.qcodes + a.qoff[q];

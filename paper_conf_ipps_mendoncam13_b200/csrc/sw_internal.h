@@ -86,7 +86,7 @@ struct K1Args {
   int32_t n_groups;                  // groups [g0, g0 + n_groups) (set by launch_k1)
   int32_t *scores; int64_t ndb;      // [nq][ndb]
   int32_t thresh;                    // overflow threshold on best~ (offset repr)
-  int2 *ovf; int32_t *ovf_count; int32_t ovf_cap;
+  int2 *ovf; int32_t *ovf_count; int32_t ovf_cap; uint32_t *ovf_bits;
   uint2 *border; int32_t border_slot_cols; int32_t slots_per_sm; int32_t *slot_busy;
   const volatile int32_t *abort_flag;
   uint32_t na, nb;                   // packed -alpha, -beta
@@ -97,7 +97,7 @@ struct K3Args {   // sequences [l0,l1) in sorted order (the long groups)
   int32_t pair; int32_t l0, l1;
   int32_t *scores; int64_t ndb;
   int32_t thresh;
-  int2 *ovf; int32_t *ovf_count; int32_t ovf_cap;
+  int2 *ovf; int32_t *ovf_count; int32_t ovf_cap; uint32_t *ovf_bits;
   uint2 *border; int64_t border_stride;   // per-warp border (>= max long len)
   const volatile int32_t *abort_flag;
   uint32_t na, nb;
@@ -106,7 +106,8 @@ struct K2Args {   // int32 re-run of saturated pairs (warp per pair)
   const uint8_t *qcodes; const int64_t *qoff;
   const uint4 *packed; const GroupInfo *groups; const int32_t *sorted_len; const int32_t *perm;
   const int8_t *matrix;                   // 24x24 (device)
-  const int2 *ovf; const int32_t *ovf_count;
+  const int2 *ovf; const int32_t *ovf_count; int32_t ovf_cap;
+  int32_t *ovf_cursor;                    // warps take entries with atomicAdd
   int32_t *scores; int64_t ndb;
   int32_t alpha, beta;
   int32_t *border; int64_t border_stride; int32_t n_warps_total;

@@ -17,6 +17,7 @@ ap.add_argument("--n-db", type=int, default=None)
 ap.add_argument("--n-queries", type=int, default=None)
 ap.add_argument("--streams", type=int, default=3)
 ap.add_argument("--long-threshold", type=int, default=0)
+ap.add_argument("--unit-cells", type=int, default=0)
 ap.add_argument("--dump-log", default=None)
 ap.add_argument("--print-k1", type=int, default=0, help="print the first N K1 units (launch order)")
 args = ap.parse_args()
@@ -25,7 +26,7 @@ D = Database(w.db)
 for s in range(args.steps):
     t = time.perf_counter()
     r = D.search(w.queries, top_k=10, outputs_on_device=True, streams=args.streams,
-                 long_threshold=args.long_threshold)
+                 long_threshold=args.long_threshold, target_unit_cells=args.unit_cells)
     st = r.stats
     print(f"step {s}: {st['gcups']:.1f} GCUPS dev {st['seconds_device']:.3f}s wall {time.perf_counter()-t:.3f}s "
           f"k1 {st['kernel_seconds_k1']:.3f}s/{st['cells_k1']:.3e} k3 {st['kernel_seconds_k3']:.3f}s/{st['cells_k3']:.3e} "
