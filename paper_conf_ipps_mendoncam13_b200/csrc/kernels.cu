@@ -322,8 +322,10 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
       // rows of the last band past the longer query are padding: skip them (nobody reads
       // their output; the last band writes no border)
       const bool live = band < nb - 1 || warp * K < rows - (nb - 1) * BAND;
-      constexpr int GS = (UQ == 8) ? 8 : 4;   // columns interleaved in one skewed tile
-#pragma unroll
+      // UQ: 8 = skewed tiles of 8 columns, 4 = of 4 columns, 81 = tiles of 8 columns with the
+      // tile loop kept rolled (half the code of T = 16: the step fits the instruction cache)
+      constexpr int GS = (UQ == 8 || UQ == 81) ? 8 : 4;
+#pragma unroll(UQ == 81 ? 1 : T / GS)
       for (int q = 0; q < T / GS && live; q++) {
         const uint32_t *prc[GS];
         uint32_t hdc[GS], fc[GS], oh[GS];
@@ -428,6 +430,15 @@ int k1_blocks_per_sm() {
   return v;
 }
 int k1_band_rows() { return k1_variant() == 4 ? kK1Rows * 4 : kK1Rows * 8; }
+static bool k1_wide_rolled() {   // SW_K1_WIDE_ROLLED=1: 16-column steps with a rolled tile loop
+  static int v = -1;
+  if (v < 0) {
+    const char *e = getenv("SW_K1_WIDE_ROLLED");
+    v = (e && atoi(e) == 1) ? 1 : 0;
+    if (v) k1_occ<8, 16, 2, 81>();
+  }
+  return v == 1;
+}
 static bool k1_wide_enabled() {
   static int v = -1;
   if (v < 0) {
@@ -446,7 +457,8 @@ void launch_k1(const K1Args &a_in, int n_groups, int min_cols, int, cudaStream_t
   const int cap = std::max(1, n_sm) * k1_blocks_per_sm();
   const dim3 g(std::min(n_groups, cap));
   if (min_cols >= kWideCols && k1_variant() == 3 && k1_wide_enabled()) {
-    k1_kernel<kK1Rows, 8, 16, 2, 8><<<g, 256, k1_smem<8, 16>(), st>>>(a);
+    if (k1_wide_rolled()) k1_kernel<kK1Rows, 8, 16, 2, 81><<<g, 256, k1_smem<8, 16>(), st>>>(a);
+    else k1_kernel<kK1Rows, 8, 16, 2, 8><<<g, 256, k1_smem<8, 16>(), st>>>(a);
     return;
   }
   switch (k1_variant()) {

@@ -346,3 +346,22 @@ def test_traceback_long_and_asymmetric():
         assert a["score"] == ref[k]
         _check_alignment(qs.seq(int(qi[k])).decode(), db.seq(int(di[k])).decode(), a, M, 4, 3)
     D.close()
+
+
+def test_unusual_inputs():
+    """Ambiguity codes B/Z/X and '*', lower case, a query longer than the database
+    sequences (12,000 aa; several K1 bands of 128 rows and K3 chunks of 512), many short
+    queries (packs of several queries per s16x2 half), and duplicate sequences."""
+    rng = np.random.default_rng(17)
+    alpha = seqgen.AMINO + "BZX*"
+    def rs(n):
+        return "".join(alpha[i] for i in rng.integers(0, len(alpha), n))
+    queries = [rs(12000), rs(5).lower(), rs(1)] + [rs(int(x)) for x in rng.integers(10, 300, 61)]
+    db = [rs(int(x)) for x in rng.integers(0, 4000, 300)] + [queries[3], queries[3], "*" * 50, "X" * 3100]
+    qs, dbs = seqgen.SeqSet.from_list(queries), seqgen.SeqSet.from_list(db)
+    ref = oracle.search(seqgen.SeqSet.from_list([q.upper() for q in queries]), dbs)
+    for thr in (0, 1000):
+        r = _search(dbs, qs, top_k=6, long_threshold=thr)
+        bad = np.argwhere(r.scores != ref)
+        assert len(bad) == 0, (thr, bad[:5])
+        _check_topk(r, ref, 6)
