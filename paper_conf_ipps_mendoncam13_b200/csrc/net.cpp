@@ -165,7 +165,8 @@ void SchedClient::connect(const char *host, int port, int rank, double timeout_s
       freeaddrinfo(res);
       throw Error(SW_ENET, "slave: cannot reach the master at " + std::string(host) + ":" + std::to_string(port));
     }
-    std::this_thread::sleep_for(std::chrono::milliseconds(20));
+    // retry quickly: every rank's GPU waits (and is timed) until all slaves registered
+    std::this_thread::sleep_for(std::chrono::microseconds(500));
   }
   freeaddrinfo(res);
   nodelay(fd_);
