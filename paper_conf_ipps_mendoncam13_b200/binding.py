@@ -66,11 +66,11 @@ class sw_stats(ctypes.Structure):
 EXPORTS = ["sw_opts_default", "sw_db_create", "sw_db_destroy", "sw_db_residues", "sw_db_size",
            "sw_db_devices", "sw_search", "sw_topk_device", "sw_last_error", "sw_version",
            "sw_sched_create", "sw_sched_destroy", "sw_sched_report", "sw_sched_request",
-           "sw_sched_complete", "sw_sched_abandon", "sw_sched_is_finished", "sw_sched_state",
+           "sw_sched_complete", "sw_sched_abandon", "sw_sched_start", "sw_sched_is_finished", "sw_sched_state",
            "sw_sched_committed_by", "sw_sched_replicas", "sw_sched_phi", "sw_sched_rate",
            "sw_sched_counter", "sw_sched_log_json", "sw_master_start", "sw_master_stop",
            "sw_slave_connect", "sw_slave_request", "sw_slave_report", "sw_slave_complete",
-           "sw_slave_abandon", "sw_slave_is_finished", "sw_slave_done", "sw_align"]
+           "sw_slave_abandon", "sw_slave_start", "sw_slave_is_finished", "sw_slave_done", "sw_align"]
 
 
 def lib():
@@ -120,6 +120,8 @@ def lib():
     L.sw_sched_complete.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_double]
     L.sw_sched_complete.restype = ctypes.c_int32
     L.sw_sched_abandon.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_double]
+    L.sw_sched_start.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_double]
+    L.sw_sched_start.restype = ctypes.c_int32
     for name in ("sw_sched_is_finished", "sw_sched_state", "sw_sched_committed_by",
                  "sw_sched_replicas"):
         getattr(L, name).argtypes = [ctypes.c_void_p, ctypes.c_int32]
@@ -144,6 +146,8 @@ def lib():
     L.sw_slave_complete.argtypes = [ctypes.c_void_p, ctypes.c_int32]
     L.sw_slave_complete.restype = ctypes.c_int32
     L.sw_slave_abandon.argtypes = [ctypes.c_void_p, ctypes.c_int32]
+    L.sw_slave_start.argtypes = [ctypes.c_void_p, ctypes.c_int32]
+    L.sw_slave_start.restype = ctypes.c_int32
     L.sw_slave_is_finished.argtypes = [ctypes.c_void_p, ctypes.c_int32]
     L.sw_slave_is_finished.restype = ctypes.c_int32
     L.sw_slave_done.argtypes = [ctypes.c_void_p]
@@ -347,6 +351,10 @@ class Scheduler:
     def abandon(self, worker, unit, now):
         lib().sw_sched_abandon(self._h, worker, unit, now)
 
+    def start(self, worker, unit, now) -> bool:
+        """Worker is about to execute `unit`: False if it is finished or was moved away."""
+        return bool(lib().sw_sched_start(self._h, worker, unit, now))
+
     def is_finished(self, unit) -> bool:
         return bool(lib().sw_sched_is_finished(self._h, unit))
 
@@ -414,6 +422,12 @@ class Slave:
 
     def abandon(self, unit):
         lib().sw_slave_abandon(self._h, unit)
+
+    def start(self, unit) -> bool:
+        rc = lib().sw_slave_start(self._h, unit)
+        if rc < 0:
+            raise SwError(SW_ENET, lib().sw_last_error().decode())
+        return rc == 1
 
     def is_finished(self, unit) -> bool:
         return lib().sw_slave_is_finished(self._h, unit) == 1

@@ -654,9 +654,9 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       if (client) return client->is_finished(u);
       return sched ? sw_sched_is_finished(sched, u) : 0;
     };
-    auto saband = [&](int w, int u, double t) {
-      if (client) client->abandon(u, t);
-      else if (sched) sw_sched_abandon(sched, w, u, t);
+    auto sstart = [&](int w, int u, double t) -> int {
+      if (client) return client->start(u, t);
+      return sched ? sw_sched_start(sched, w, u, t) : 1;
     };
 
     // ---------------- workers: one thread per device
@@ -753,7 +753,8 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
             if (inflight[k] >= 0) continue;
             const int u = pending.front();
             pending.pop_front();
-            if (sfin(u)) { saband(wid, u, now_s()); progressed = true; k--; continue; }
+            // finished elsewhere, or moved to an idle worker by WA before it started
+            if (!sstart(wid, u, now_s())) { progressed = true; k--; continue; }
             CK(cudaEventRecord(X.u_start[k], D.streams[k]));
             launch_unit(P, H, X, P.units[u], u, k, alpha, beta, thresh);
             CK(cudaGetLastError());

@@ -23,6 +23,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <algorithm>
+#include <mutex>
 #include "sw_internal.h"
 
 namespace sw {
@@ -400,12 +401,11 @@ static size_t k1_smem() {
 // 4 = (4, 8, 4, 8).  Groups of >= kWideCols columns use (8, 16, 2, 8) unless SW_K1_WIDE=0
 // (half the pipeline steps and barriers; needs nt >= W+1 tiles of 16 columns).
 static int k1_variant() {
-  static int v = -1;
-  if (v < 0) {
+  static const int v = [] {
     const char *e = getenv("SW_K1_VARIANT");
-    v = e ? atoi(e) : 3;
-    if (v < 0 || v > 4) v = 3;
-  }
+    const int x = e ? atoi(e) : 3;
+    return (x < 0 || x > 4) ? 3 : x;
+  }();
   return v;
 }
 template <int W, int T, int MINB, int UQ>
@@ -417,8 +417,9 @@ static int k1_occ() {
   return n > 0 ? n : 1;
 }
 int k1_blocks_per_sm() {
-  static int v = -1;
-  if (v < 0) {
+  static std::once_flag once;
+  static int v = 1;
+  std::call_once(once, [] {
     switch (k1_variant()) {
       case 0: v = k1_occ<8, 8, 2, 4>(); break;
       case 1: v = k1_occ<8, 4, 3, 4>(); break;
@@ -426,27 +427,26 @@ int k1_blocks_per_sm() {
       case 4: v = k1_occ<4, 8, 4, 8>(); break;
       default: v = k1_occ<8, 8, 2, 8>(); break;
     }
-  }
+  });
   return v;
 }
 int k1_band_rows() { return k1_variant() == 4 ? kK1Rows * 4 : kK1Rows * 8; }
 static bool k1_wide_rolled() {   // SW_K1_WIDE_ROLLED=1: 16-column steps with a rolled tile loop
-  static int v = -1;
-  if (v < 0) {
-    const char *e = getenv("SW_K1_WIDE_ROLLED");
-    v = (e && atoi(e) == 1) ? 1 : 0;
-    if (v) k1_occ<8, 16, 2, 81>();
-  }
-  return v == 1;
+  static const bool v = [] { const char *e = getenv("SW_K1_WIDE_ROLLED"); return e && atoi(e) == 1; }();
+  return v;
 }
 static bool k1_wide_enabled() {
-  static int v = -1;
-  if (v < 0) {
-    const char *e = getenv("SW_K1_WIDE");
-    v = (e && atoi(e) == 0) ? 0 : 1;
-    if (v) k1_occ<8, 16, 2, 8>();
-  }
-  return v == 1;
+  static const bool v = [] { const char *e = getenv("SW_K1_WIDE"); return !(e && atoi(e) == 0); }();
+  return v;
+}
+
+// dynamic shared memory above 48 KB needs the function attribute on the launching device;
+// it is set before every launch (cheap, and correct with several devices and threads)
+template <int W, int T, int MINB, int UQ>
+static void k1_go(const K1Args &a, dim3 g, cudaStream_t st) {
+  auto fn = k1_kernel<kK1Rows, W, T, MINB, UQ>;
+  cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem<W, T>());
+  fn<<<g, W * 32, k1_smem<W, T>(), st>>>(a);
 }
 
 void launch_k1(const K1Args &a_in, int n_groups, int min_cols, int, cudaStream_t st, int n_sm) {
@@ -457,16 +457,16 @@ void launch_k1(const K1Args &a_in, int n_groups, int min_cols, int, cudaStream_t
   const int cap = std::max(1, n_sm) * k1_blocks_per_sm();
   const dim3 g(std::min(n_groups, cap));
   if (min_cols >= kWideCols && k1_variant() == 3 && k1_wide_enabled()) {
-    if (k1_wide_rolled()) k1_kernel<kK1Rows, 8, 16, 2, 81><<<g, 256, k1_smem<8, 16>(), st>>>(a);
-    else k1_kernel<kK1Rows, 8, 16, 2, 8><<<g, 256, k1_smem<8, 16>(), st>>>(a);
+    if (k1_wide_rolled()) k1_go<8, 16, 2, 81>(a, g, st);
+    else k1_go<8, 16, 2, 8>(a, g, st);
     return;
   }
   switch (k1_variant()) {
-    case 0: k1_kernel<kK1Rows, 8, 8, 2, 4><<<g, 256, k1_smem<8, 8>(), st>>>(a); break;
-    case 1: k1_kernel<kK1Rows, 8, 4, 3, 4><<<g, 256, k1_smem<8, 4>(), st>>>(a); break;
-    case 2: k1_kernel<kK1Rows, 8, 8, 3, 4><<<g, 256, k1_smem<8, 8>(), st>>>(a); break;
-    case 4: k1_kernel<kK1Rows, 4, 8, 4, 8><<<g, 128, k1_smem<4, 8>(), st>>>(a); break;
-    default: k1_kernel<kK1Rows, 8, 8, 2, 8><<<g, 256, k1_smem<8, 8>(), st>>>(a); break;
+    case 0: k1_go<8, 8, 2, 4>(a, g, st); break;
+    case 1: k1_go<8, 4, 3, 4>(a, g, st); break;
+    case 2: k1_go<8, 8, 3, 4>(a, g, st); break;
+    case 4: k1_go<4, 8, 4, 8>(a, g, st); break;
+    default: k1_go<8, 8, 2, 8>(a, g, st); break;
   }
 }
 
@@ -634,11 +634,7 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
 
 // K3 tile width (tuning; SW_K3_T): 8 columns per lane step (default) or 4
 static int k3_tile() {
-  static int v = -1;
-  if (v < 0) {
-    const char *e = getenv("SW_K3_T");
-    v = (e && atoi(e) == 4) ? 4 : 8;
-  }
+  static const int v = [] { const char *e = getenv("SW_K3_T"); return (e && atoi(e) == 4) ? 4 : 8; }();
   return v;
 }
 void launch_k3(const K3Args &a, int, cudaStream_t st) {
@@ -646,15 +642,14 @@ void launch_k3(const K3Args &a, int, cudaStream_t st) {
   if (n <= 0) return;
   const size_t smem = sizeof(uint32_t) * kNCodes * kK3Rows * 32 + sizeof(uint4) * kK3Warps * 3 +
                       sizeof(uint2) * kK3Warps * 3 * 8;
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(k3_kernel<kK3Rows, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    cudaFuncSetAttribute(k3_kernel<kK3Rows, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    attr = true;
-  }
   const int blocks = (n + kK3Warps - 1) / kK3Warps;
-  if (k3_tile() == 4) k3_kernel<kK3Rows, 4><<<blocks, kK3Warps * 32, smem, st>>>(a);
-  else k3_kernel<kK3Rows, 8><<<blocks, kK3Warps * 32, smem, st>>>(a);
+  if (k3_tile() == 4) {
+    cudaFuncSetAttribute(k3_kernel<kK3Rows, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    k3_kernel<kK3Rows, 4><<<blocks, kK3Warps * 32, smem, st>>>(a);
+  } else {
+    cudaFuncSetAttribute(k3_kernel<kK3Rows, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    k3_kernel<kK3Rows, 8><<<blocks, kK3Warps * 32, smem, st>>>(a);
+  }
 }
 
 // ------------------------------------------------------------------------------------

@@ -18,7 +18,7 @@ namespace sw {
 
 namespace {
 enum Op : int32_t { kHello = 0, kRequest = 1, kReport = 2, kComplete = 3, kAbandon = 4,
-                    kFinishedMap = 5, kDone = 6, kCounters = 7 };
+                    kFinishedMap = 5, kDone = 6, kCounters = 7, kStart = 8 };
 struct Msg {
   int32_t op, worker, unit, cap;
   double t, cells, sec;
@@ -109,6 +109,7 @@ void MasterServer::serve(int fd) {
       case kReport: if (sched_) sw_sched_report(sched_, worker, t, m.cells, m.sec); break;
       case kComplete: h.rc = sched_ ? sw_sched_complete(sched_, worker, m.unit, t) : 1; break;
       case kAbandon: if (sched_) sw_sched_abandon(sched_, worker, m.unit, t); break;
+      case kStart: h.rc = sched_ ? sw_sched_start(sched_, worker, m.unit, t) : 1; break;
       case kFinishedMap: {
         const int32_t n = m.cap;
         buf.assign((n + 31) / 32, 0);
@@ -197,6 +198,7 @@ int32_t SchedClient::request(double t, int32_t *out, int32_t cap) {
 void SchedClient::report(double t, double cells, double sec) { call(kReport, 0, 0, t, cells, sec, nullptr); }
 int32_t SchedClient::complete(int32_t unit, double t) { return call(kComplete, unit, 0, t, 0, 0, nullptr); }
 void SchedClient::abandon(int32_t unit, double t) { call(kAbandon, unit, 0, t, 0, 0, nullptr); }
+int32_t SchedClient::start(int32_t unit, double t) { return call(kStart, unit, 0, t, 0, 0, nullptr); }
 int32_t SchedClient::is_finished(int32_t unit) {
   const double t = now_s();
   if (t - last_refresh_ > 5e-4 || unit / 32 >= (int32_t)finished_.size()) {
@@ -269,6 +271,9 @@ int32_t sw_slave_complete(sw_slave *c, int32_t unit) {
 }
 void sw_slave_abandon(sw_slave *c, int32_t unit) {
   try { c->c.abandon(unit, clk()); } catch (const std::exception &e) { sw::set_last_error(e.what()); }
+}
+int32_t sw_slave_start(sw_slave *c, int32_t unit) {
+  try { return c->c.start(unit, clk()); } catch (const std::exception &e) { sw::set_last_error(e.what()); return -2; }
 }
 int32_t sw_slave_is_finished(sw_slave *c, int32_t unit) {
   try { return c->c.is_finished(unit); } catch (const std::exception &e) { sw::set_last_error(e.what()); return -2; }

@@ -43,6 +43,7 @@ class SchedClient {
   void report(double t, double cells, double sec);
   int32_t complete(int32_t unit, double t);
   void abandon(int32_t unit, double t);
+  int32_t start(int32_t unit, double t);   // 1 = run it, 0 = finished or moved away
   int32_t is_finished(int32_t unit);   // cached bitmap, refreshed at most every 0.5 ms
   void done();
   int32_t wa_grants() const { return wa_; }

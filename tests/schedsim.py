@@ -27,8 +27,7 @@ def simulate(speeds, unit_cells, policy="pss", wa=True, omega=4, heartbeat=0.5, 
     def start_next(w, t):
         while queue[w]:
             u = queue[w].pop(0)
-            if S.is_finished(u):
-                S.abandon(w, u, t)
+            if not S.start(w, u, t):   # finished elsewhere or moved away by WA
                 continue
             dur = unit_cells[u] / speed[w]
             current[w] = (u, t, t + dur)

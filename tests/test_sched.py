@@ -104,6 +104,38 @@ def test_states_and_first_result_wins():
     assert S.counter(2) == 4                   # duplicated cells
 
 
+def test_wa_moves_a_queued_task_instead_of_duplicating():
+    """A task still queued (un-started) in the holder's PSS package is moved to the idle PE
+    (reading R11): one replica, the old holder's start() is refused, no duplicated cells.
+    A started task (here the head of the queue) is duplicated as in Fig. 5."""
+    S = Scheduler(2, [100] * 6)
+    assert S.request(0, 0.0) == [0] and S.request(1, 0.0) == [1]
+    S.report(0, 1.0, 300.0, 1.0)
+    S.report(1, 1.0, 100.0, 1.0)
+    assert S.complete(0, 0, 1.0)
+    assert S.request(0, 1.0) == [2, 3, 4]              # Phi = 3
+    assert S.start(0, 2, 1.0)
+    assert S.complete(1, 1, 1.0)
+    assert S.request(1, 1.0) == [5]
+    assert S.start(1, 5, 1.0)
+    S.report(0, 1.5, 10.0, 1.0)                        # worker 0 slows down (local load)
+    assert S.complete(1, 5, 2.0)
+    assert S.request(1, 2.0) == [4]                    # latest ETA: the tail of w0's package
+    assert S.replicas(4) == 1                          # moved, not duplicated
+    assert S.start(1, 4, 2.0)
+    assert S.complete(1, 4, 3.0)
+    assert S.request(1, 3.0) == [3]                    # next latest, also un-started
+    assert S.replicas(3) == 1
+    assert S.start(1, 3, 3.0) and S.complete(1, 3, 4.0)
+    assert S.request(1, 4.0) == [2]                    # w0's started head: duplicated
+    assert S.replicas(2) == 2
+    assert S.complete(1, 2, 5.0) and not S.complete(0, 2, 9.0)
+    assert not S.start(0, 3, 9.0) and not S.start(0, 4, 9.0)   # w0 skips the moved ones
+    assert S.request(0, 9.0) is None
+    assert S.counter(2) == 100                         # only the started head was duplicated
+    assert [S.committed_by(u) for u in range(6)] == [0, 1, 1, 1, 1, 1]
+
+
 def test_wa_only_when_strictly_earlier():
     S = Scheduler(2, [6])
     S.report(0, 0.0, 1.0, 1.0)
