@@ -175,6 +175,8 @@ def main():
     ap.add_argument("--streams", type=int, default=4)
     ap.add_argument("--unit-cells", type=int, default=0)
     ap.add_argument("--top-k", type=int, default=10)
+    ap.add_argument("--long-threshold", type=int, default=0,
+                    help="DB length routed to the intra-task kernel K3 (0 = libsw's auto)")
     args = ap.parse_args()
     if args.impl == "reference":
         return reference_arm(args)
@@ -205,7 +207,8 @@ def main():
     db_create_s = time.perf_counter() - t
     cells = int(w.meta["cells"])
     kw = dict(policy=args.policy, workload_adjust=not args.no_wa, streams=args.streams,
-              target_unit_cells=args.unit_cells, straggler_mask=args.straggler_mask)
+              target_unit_cells=args.unit_cells, straggler_mask=args.straggler_mask,
+              long_threshold=args.long_threshold)
 
     def step():
         if world > 1:

@@ -15,7 +15,7 @@ __device__ __forceinline__ uint32_t pk(int v) { return ((uint32_t)(v & 0xffff)) 
 
 // profile entries: P[c][i] s16x2 (natural), Pa = S + alpha (s16x2), V = signed-packed int32 S
 template <int K, int VAR>
-__global__ void __launch_bounds__(256, (VAR == 11 ? 2 : 1)) dp(const uint4 *__restrict__ db, const uint32_t *__restrict__ gprof,
+__global__ void __launch_bounds__(256, (VAR >= 11 ? 2 : 1)) dp(const uint4 *__restrict__ db, const uint32_t *__restrict__ gprof,
                                           int alpha, int beta, uint32_t *out, int reps) {
   __shared__ uint32_t P[NC * (K + 1)];
   for (int k = threadIdx.x; k < NC * (K + 1); k += blockDim.x) P[k] = gprof[k];
@@ -33,7 +33,9 @@ __global__ void __launch_bounds__(256, (VAR == 11 ? 2 : 1)) dp(const uint4 *__re
       else { H[i] = Kp; E[i] = Kp; }                    // offset repr, floored E
     }
     const uint4 *p = db + tid;
-    if (VAR == 11) {   // VAR2 cell, 8 columns per tile with explicit row skew (ILP 8)
+    if (VAR == 11 || VAR == 13 || VAR == 14) {   // 8 columns per tile with explicit row skew (ILP 8)
+      // 11: VAR2 cell; 13: t = max(h - alpha, Koff) by 32-bit IADD + 2-input VIMNMX (one
+      // DPX fewer, one issue more); 14: 13 with the H floor on h (vmaxs2) and unfloored t
       uint32_t hprev = Kp;
       for (int w = 0; w < NCOL / 16; w++) {
         uint4 r4 = p[(size_t)w * gridDim.x * blockDim.x];
@@ -56,8 +58,10 @@ __global__ void __launch_bounds__(256, (VAR == 11 ? 2 : 1)) dp(const uint4 *__re
               const int i = k - g;
               if (i >= 0 && i < K) {
                 uint32_t x = hdc[g] + prc[g][i];
-                uint32_t h = __vimax3_s16x2(x, E[i], fc[g]);
-                uint32_t t = __viaddmax_s16x2(h, na, Kp);
+                uint32_t h, t;
+                if (VAR == 11) { h = __vimax3_s16x2(x, E[i], fc[g]); t = __viaddmax_s16x2(h, na, Kp); }
+                else if (VAR == 13) { h = __vimax3_s16x2(x, E[i], fc[g]); t = __vmaxs2(h - A32, Kp); }
+                else { h = __vmaxs2(__vimax3_s16x2(x, E[i], fc[g]), Kp); t = h - A32; }
                 E[i] = __viaddmax_s16x2(E[i], nb, t);
                 fc[g] = __viaddmax_s16x2(fc[g], nb, t);
                 hdc[g] = H[i]; H[i] = h;
@@ -301,9 +305,13 @@ int main() {
   int reps = 2;
   std::vector<uint32_t> r11;
   for (int pass = 0; pass < 2; pass++) {
+    std::vector<uint32_t> r13, r14, r12;
     run<16, 2>(nthreads, ddb, 12, 2, dout, r2, reps, ghz, nsm);
     run<16, 11>(nthreads, ddb, 12, 2, dout, r11, reps, ghz, nsm);
-    printf("agree16: %d\n", r2 == r11);
+    run<16, 13>(nthreads, ddb, 12, 2, dout, r13, reps, ghz, nsm);
+    run<16, 14>(nthreads, ddb, 12, 2, dout, r14, reps, ghz, nsm);
+    run<16, 12>(nthreads, ddb, 12, 2, dout, r12, reps, ghz, nsm);
+    printf("agree16: %d %d %d %d\n", r2 == r11, r2 == r13, r2 == r14, r2 == r12);
   }
   return 0;
 }
