@@ -564,6 +564,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       int32_t need_cols = 0;
       for (int32_t g = P.first_short_group; g < (int32_t)H.groups.size(); g++)
         need_cols = std::max(need_cols, H.groups[g].ncols);
+      need_cols = (need_cols + kWordCols - 1) / kWordCols * kWordCols;   // whole 16-column tiles
       if (need_cols > D.slot_cols) {
         D.k1_border.alloc(D.id, (size_t)D.sm_slots * D.slots_per_sm * need_cols * 32);
         D.slot_busy.alloc(D.id, (size_t)D.sm_slots * D.slots_per_sm);

@@ -194,7 +194,7 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   // draining the warp pipeline between them
   const int gfirst = a.g0 + blockIdx.x, gend = a.g0 + a.n_groups, gstride = gridDim.x;
   int total = 0;
-  for (int g = gfirst; g < gend; g += gstride) total += nb * (a.groups[g].ncols / T);
+  for (int g = gfirst; g < gend; g += gstride) total += nb * ((a.groups[g].ncols + T - 1) / T);
 
   uint2 *border = nullptr;
   if (nb > 1 && threadIdx.x == 0) {   // a border-row slot of this SM (released at exit)
@@ -220,7 +220,7 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   // block-uniform tracker of warp 0's band starts: the profile of global band B+1 is
   // loaded into slot (B+1)&1 when warp W-1 leaves band B-1, i.e. W-1 steps after warp 0
   // starts band B (every band has nt >= W+1 steps, so warp 0 needs it later)
-  int t_g = gfirst, t_band = 0, t_nt = a.groups[gfirst].ncols / T, t_start = 0, t_B = 0;
+  int t_g = gfirst, t_band = 0, t_nt = (a.groups[gfirst].ncols + T - 1) / T, t_start = 0, t_B = 0;
   int rl_step = -1, rl_band = 0, rl_slot = 0;
 
   // per-warp iterator over (group, band, tile); the queries of this warp's current slice
@@ -230,7 +230,7 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   uint32_t omask = 0;
   const int nslices = P.rows_padded / 16;
   GroupInfo G = a.groups[g];
-  int nt = G.ncols / T, nwords = (G.ncols + kWordCols - 1) / kWordCols, wnext = nwords > 1 ? 1 : 0;
+  int nt = (G.ncols + T - 1) / T, nwords = (G.ncols + kWordCols - 1) / kWordCols, wnext = nwords > 1 ? 1 : 0;
   const uint4 *wp = a.packed + G.word_off + lane;
   uint4 r4 = wp[0], r4n = wp[(size_t)wnext * 32];
   uint32_t H[K], E[K];
@@ -245,7 +245,7 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
         if (++t_band == nb) {
           t_band = 0;
           t_g += gstride;
-          if (t_g < gend) t_nt = a.groups[t_g].ncols / T;
+          if (t_g < gend) t_nt = (a.groups[t_g].ncols + T - 1) / T;
         }
         // the band after this one: rows (t_band+1) mod nb, slot (t_B+1)&1
         if (t_B + 1 >= 2) {
@@ -326,8 +326,12 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
       // UQ: 8 = skewed tiles of 8 columns, 4 = of 4 columns, 81 = tiles of 8 columns with the
       // tile loop kept rolled (half the code of T = 16: the step fits the instruction cache)
       constexpr int GS = (UQ == 8 || UQ == 81) ? 8 : 4;
+      // group columns are a multiple of 8: with 16-column tiles the last tile of a band
+      // may hold 8 real columns; its second half (pad codes) is skipped (outputs unused)
+      const int nq_tile = (T == 16 && tile == nt - 1 && (G.ncols & 15)) ? T / GS / 2 : T / GS;
 #pragma unroll(UQ == 81 ? 1 : T / GS)
       for (int q = 0; q < T / GS && live; q++) {
+        if (q >= nq_tile) break;
         const uint32_t *prc[GS];
         uint32_t hdc[GS], fc[GS], oh[GS];
 #pragma unroll
@@ -373,7 +377,7 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
           g += gstride;
           if (g < gend) {
             G = a.groups[g];
-            nt = G.ncols / T;
+            nt = (G.ncols + T - 1) / T;
             nwords = (G.ncols + kWordCols - 1) / kWordCols;
             wnext = nwords > 1 ? 1 : 0;
             wp = a.packed + G.word_off + lane;

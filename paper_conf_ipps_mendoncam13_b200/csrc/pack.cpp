@@ -135,8 +135,6 @@ int pack_database(const int64_t *offsets, const char *residues, int32_t n, Packe
     G.count = std::min(kGroup, n - G.first);
     int32_t l = out.sorted_len[G.first];
     int32_t cols = (l + kColAlign - 1) / kColAlign * kColAlign;
-    // groups wide enough for the 16-column-step K1 instance are rounded to its tile
-    if (cols >= kWideCols) cols = (cols + kWordCols - 1) / kWordCols * kWordCols;
     G.ncols = std::max(cols, kMinCols);
     G.word_off = words;
     G.pad_ = 0;
