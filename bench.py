@@ -114,6 +114,17 @@ def oracle_rate(w, seconds_target=15.0, seed=99, max_threads=None):
     return cells / dt / 1e9, cores, desc, cells, dt
 
 
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
 def reference_arm(args):
     rank, world, _ = env_rank()
     if rank != 0:
@@ -137,7 +148,7 @@ def reference_arm(args):
                        "note": "oracle (plain C Gotoh, OpenMP over pairs) on host cores; each step a "
                                "bounded random sample of the workload's pairs"},
             "cpu_baseline": {"value": value, "unit": "GCUPS", "cores": cores, "kind": "oracle",
-                             "sample": desc},
+                             "sample": desc, "cpu_model": cpu_model()},
             "e2e": {"value": value, "unit": "GCUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
             "context": PAPER_CONTEXT}
     print(json.dumps(line), flush=True)
@@ -333,7 +344,9 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         g, cores, desc, _, _ = oracle_rate(w, seconds_target=args.cpu_seconds)
-        cpu = {"value": g, "unit": "GCUPS", "cores": cores, "kind": "oracle", "sample": desc}
+        g1, _, desc1, _, _ = oracle_rate(w, seconds_target=3.0, seed=7, max_threads=1)
+        cpu = {"value": g, "unit": "GCUPS", "cores": cores, "kind": "oracle", "sample": desc,
+               "single_core": {"value": g1, "sample": desc1}, "cpu_model": cpu_model()}
 
     if rank == 0:
         line = {"metric": "GCUPS", "value": value, "unit": "GCUPS", "n_gpus": world,
