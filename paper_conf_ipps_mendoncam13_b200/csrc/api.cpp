@@ -362,7 +362,6 @@ struct UnitLog {
 
 static const int kOvfCap = 1 << 20;
 
-static const int kK2BlocksPerUnit = 8;   // 32 warps per stream for the int32 re-run
 
 // K2 arguments for the saturated-pair list of one stream
 static K2Args k2_args(const Plan &P, const PackedDB &db, DevSearch &S, int stream_idx, int32_t alpha,
@@ -374,11 +373,10 @@ static K2Args k2_args(const Plan &P, const PackedDB &db, DevSearch &S, int strea
   a.matrix = S.matrix.p;
   a.ovf = S.ovf.p + (size_t)stream_idx * S.ovf_cap; a.ovf_count = S.ovf_count.p + stream_idx;
   a.ovf_cap = S.ovf_cap; a.ovf_cursor = S.ovf_cursor.p + stream_idx;
-  a.scores = S.scores; a.ndb = db.n; a.alpha = alpha; a.beta = beta;
+  a.scores = S.scores; a.ndb = db.n; a.alpha = alpha; a.beta = beta; a.one = 1;
   const int64_t stride = std::max<int64_t>(P.max_len, 1);
-  a.border = S.k2_border.p + (size_t)stream_idx * kK2BlocksPerUnit * 4 * stride * 2;
+  a.border = S.k2_border.p + (size_t)stream_idx * kK2Blocks * stride * 2;
   a.border_stride = stride;
-  a.n_warps_total = kK2BlocksPerUnit * 4;
   return a;
 }
 
@@ -420,7 +418,7 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
   }
   S.launches++;
   // int32 re-run of the pairs this unit saturated, on its stream (overlaps other units)
-  launch_k2(k2_args(P, db, S, stream_idx, alpha, beta), kK2BlocksPerUnit, st);
+  launch_k2(k2_args(P, db, S, stream_idx, alpha, beta), kK2Blocks, st);
   S.launches++;
 }
 
@@ -592,7 +590,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       X.ovf_count.ensure(D.id, depth);
       X.ovf_cursor.ensure(D.id, depth);
       X.ovf_bits.ensure(D.id, ((size_t)nq * nd + 31) / 32);
-      X.k2_border.ensure(D.id, (size_t)depth * kK2BlocksPerUnit * 4 * std::max<int64_t>(P.max_len, 1) * 2);
+      X.k2_border.ensure(D.id, (size_t)depth * kK2Blocks * std::max<int64_t>(P.max_len, 1) * 2);
       const size_t k3b = (size_t)depth * std::max(P.max_k3_seqs, 1) *
                          ((std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16);
       if (P.n_long_seqs > 0) X.k3_border.ensure(D.id, k3b);

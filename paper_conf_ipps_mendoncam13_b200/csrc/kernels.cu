@@ -657,37 +657,55 @@ void launch_k3(const K3Args &a, int, cudaStream_t st) {
 }
 
 // ------------------------------------------------------------------------------------
-// K2: int32 re-run of saturated (query, sequence) pairs.  Plain int32 Gotoh with the
-// zero floor, one warp per pair, lane l owning rows [l*K2R, (l+1)*K2R) of each chunk of
-// 32*K2R rows (same wavefront as K3); scores read from the 24x24 matrix in shared
-// memory.  Rare (only near-identical long pairs saturate int16), so kept simple.
+// K2: int32 re-run of saturated (query, sequence) pairs.  Same recurrence as K1/K3 in
+// plain int32 (E and F floored at 0, exact for H: DESIGN.md §6), one BLOCK per pair:
+// thread L owns rows [L*K2R, (L+1)*K2R) of each chunk of kK2Threads*K2R query rows and
+// runs the wavefront of P14 §II.B (Fig. 3a) across the whole block -- at step t thread L
+// updates the K2C-column tile t - L and hands its bottom row (H, F) to thread L+1 through
+// a double-buffered shared-memory slot (one __syncthreads per step); the last active
+// thread writes the chunk's bottom row to a global border read by thread 0 in the next
+// chunk.  A single long saturated pair (C5: a 5,000-aa query inside a 10k-35k sequence)
+// therefore runs on a whole SM instead of one warp.  Scores come from the 25x25 matrix
+// replicated per lane in shared memory ([query code][db code][lane]: bank = lane, no
+// conflicts although every thread is at a different row and column).
 // ------------------------------------------------------------------------------------
-constexpr int K2R = 8;
-__global__ void __launch_bounds__(128) k2_kernel(const K2Args a) {
-  __shared__ int32_t Ms[kNCodes * 32];  // [query code][db code], pad row/col = kPadScore
-  for (int k = threadIdx.x; k < kNCodes * 32; k += blockDim.x) {
-    const int r = k / 32, c = k % 32;
+constexpr int K2R = 16;          // rows per thread
+constexpr int K2C = 4;           // columns per tile (one aligned 32-bit word of codes)
+constexpr int kK2Threads = 512;  // threads per block (chunk = 8,192 rows)
+constexpr size_t kK2Smem = sizeof(int32_t) * kNCodes * kNCodes * 32 + sizeof(int2) * 2 * kK2Threads * K2C;
+
+__global__ void __launch_bounds__(kK2Threads, 1) k2_kernel(const K2Args a) {
+  extern __shared__ __align__(16) int32_t k2s[];
+  int32_t *Ms = k2s;                                              // [qc][dc][lane]
+  int2 *hand = reinterpret_cast<int2 *>(k2s + kNCodes * kNCodes * 32);  // [2][K2C][threads]
+  __shared__ int claim_s;
+  __shared__ int red_s[kK2Threads / 32];
+  const int count = min(*a.ovf_count, a.ovf_cap);
+  if (*(volatile int32_t *)a.ovf_cursor >= count) return;   // nothing saturated (the usual case)
+  for (int k = threadIdx.x; k < kNCodes * kNCodes * 32; k += kK2Threads) {
+    const int r = k / (kNCodes * 32), c = (k / 32) % kNCodes;
     Ms[k] = (r < 24 && c < 24) ? (int32_t)a.matrix[r * 24 + c] : kPadScore;
   }
-  __syncthreads();
-  const int lane = threadIdx.x & 31;
-  const int gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int count = min(*a.ovf_count, a.ovf_cap);
-  const uint8_t *bytes = reinterpret_cast<const uint8_t *>(a.packed);
-  constexpr int NEG = -(1 << 29);
+  const int L = threadIdx.x, lane = L & 31;
+  const uint32_t *words = reinterpret_cast<const uint32_t *>(a.packed);
+  int32_t *border = a.border + (size_t)blockIdx.x * a.border_stride * 2;
+  const int na = -a.alpha, nb = -a.beta, one = a.one;
+  constexpr int CH = kK2Threads * K2R;
   while (true) {
     // claim the next entry; the cursor never passes the count (a later re-run on this
     // stream must still find the entries appended after this one)
-    int p = count;
-    if (lane == 0) {
+    if (L == 0) {
+      int p = count;
       int cur = *(volatile int32_t *)a.ovf_cursor;
       while (cur < count) {
         const int seen = atomicCAS(a.ovf_cursor, cur, cur + 1);
         if (seen == cur) { p = cur; break; }
         cur = seen;
       }
+      claim_s = p;
     }
-    p = __shfl_sync(0xffffffffu, p, 0);
+    __syncthreads();
+    const int p = claim_s;
     if (p >= count) break;
     const int q = a.ovf[p].x, s = a.ovf[p].y;
     const int m = (int)(a.qoff[q + 1] - a.qoff[q]);
@@ -695,55 +713,115 @@ __global__ void __launch_bounds__(128) k2_kernel(const K2Args a) {
     const int len = a.sorted_len[s];
     const GroupInfo G = a.groups[s / kGroup];
     const int gl = s % kGroup;
-    int32_t *border = a.border + (size_t)gw * a.border_stride * 2;
+    // the 32-bit word of codes of tile tt (columns tt*4 .. tt*4+3 of this lane's sequence)
+    auto codes_of = [&](int tt) -> uint32_t {
+      const int col = tt * K2C;
+      return __ldg(words + ((G.word_off + (int64_t)(col >> 4) * kGroup + gl) * 4 + ((col & 15) >> 2)));
+    };
+    const int ntile = (len + K2C - 1) / K2C;   // columns up to ntile*4 <= G.ncols are pad codes
+    const int nch = (m + CH - 1) / CH;
     int best = 0;
-    const int nch = (m + 32 * K2R - 1) / (32 * K2R);
-    for (int ch = 0; ch < nch; ch++) {
-      int qr[K2R];
+    for (int ch = 0; ch < nch && len > 0; ch++) {
+      const int r0 = ch * CH;
+      const int nact = min(kK2Threads, (m - r0 + K2R - 1) / K2R);   // threads with real rows
+      const bool active = L < nact;
+      int rowoff[K2R];
 #pragma unroll
       for (int i = 0; i < K2R; i++) {
-        const int row = ch * 32 * K2R + lane * K2R + i;
-        qr[i] = row < m ? qc[row] : kPadCode;
+        const int row = r0 + L * K2R + i;
+        rowoff[i] = (row < m ? (int)qc[row] : kPadCode) * (kNCodes * 32) + lane;
       }
       int H[K2R], E[K2R];
 #pragma unroll
-      for (int i = 0; i < K2R; i++) { H[i] = 0; E[i] = NEG; }
-      int hprev_top = 0, out_h = 0, out_f = NEG, out_c = kPadCode;
-      for (int t = 0; t < len + 31; t++) {
-        int in_h = __shfl_up_sync(0xffffffffu, out_h, 1);
-        int in_f = __shfl_up_sync(0xffffffffu, out_f, 1);
-        int in_c = __shfl_up_sync(0xffffffffu, out_c, 1);
-        if (lane == 0 && t < len) {
-          in_c = bytes[(G.word_off + (int64_t)(t >> 4) * kGroup + gl) * 16 + (t & 15)];
-          if (ch == 0) { in_h = 0; in_f = NEG; }
-          else { in_h = border[2 * t]; in_f = border[2 * t + 1]; }
-        }
-        const int col = t - lane;
-        if (col >= 0 && col < len) {
-          int hd = hprev_top, hup = in_h, f = in_f;
-          hprev_top = in_h;
+      for (int i = 0; i < K2R; i++) { H[i] = 0; E[i] = 0; }
+      int hprev_top = 0;
+      const int steps = ntile + nact - 1;
+      // register prefetch, one step ahead: this thread's next codes word and (thread 0 of
+      // a later chunk) the next border entries
+      uint32_t cw_next = (active && L == 0 && ntile > 0) ? codes_of(0) : 0u;
+      int2 bnext[K2C];
 #pragma unroll
-          for (int i = 0; i < K2R; i++) {
-            const int e = max(E[i] - a.beta, H[i] - a.alpha);      // E(i,j)
-            f = max(f - a.beta, hup - a.alpha);                     // F(i,j)
-            int h = hd + Ms[qr[i] * 32 + in_c];                     // diagonal
-            h = max(max(h, e), max(f, 0));                          // H(i,j)
-            hd = H[i]; H[i] = h; E[i] = e; hup = h;
-            best = max(best, h);
+      for (int g = 0; g < K2C; g++)
+        bnext[g] = (L == 0 && ch > 0) ? make_int2(border[2 * g], border[2 * g + 1]) : make_int2(0, 0);
+      for (int t = 0; t < steps; t++) {
+        const int tile = t - L;
+        if (active && tile >= 0 && tile < ntile) {
+          const uint32_t cw = cw_next;
+          if (tile + 1 < ntile) cw_next = codes_of(tile + 1);
+          int2 in[K2C];
+          if (L == 0) {
+#pragma unroll
+            for (int g = 0; g < K2C; g++) in[g] = bnext[g];
+            if (ch > 0 && tile + 1 < ntile)
+#pragma unroll
+              for (int g = 0; g < K2C; g++) {
+                const int col = (tile + 1) * K2C + g;
+                bnext[g] = make_int2(border[2 * col], border[2 * col + 1]);
+              }
+          } else {
+#pragma unroll
+            for (int g = 0; g < K2C; g++) in[g] = hand[(((t - 1) & 1) * K2C + g) * kK2Threads + L - 1];
           }
-          out_h = H[K2R - 1]; out_f = f; out_c = in_c;
-          if (lane == 31 && ch < nch - 1) { border[2 * col] = out_h; border[2 * col + 1] = out_f; }
+          int coff[K2C], hd[K2C], f[K2C], oh[K2C];
+#pragma unroll
+          for (int g = 0; g < K2C; g++) {
+            coff[g] = (int)((cw >> (8 * g)) & 0xffu) * 32;
+            hd[g] = hprev_top;
+            f[g] = in[g].y;
+            hprev_top = in[g].x;
+          }
+          // skewed tile: at sub-step k column g updates row k - g (K2C independent chains)
+#pragma unroll
+          for (int k = 0; k < K2R + K2C - 1; k++) {
+#pragma unroll
+            for (int g = 0; g < K2C; g++) {
+              const int i = k - g;
+              if (i >= 0 && i < K2R) {
+                // x on the FMA pipe (IMAD by an opaque 1): a plain add would be fused by
+                // ptxas into a VIADDMNMX + VIMNMX pair, one more ALU op per cell
+                const int x = Ms[rowoff[i] + coff[g]] * one + hd[g];
+                const int h = __vimax3_s32(x, E[i], f[g]);      // >= 0: E, F floored at 0
+                const int tt = __viaddmax_s32(h, na, 0);        // max(H - alpha, 0)
+                E[i] = __viaddmax_s32(E[i], nb, tt);            // E(i, j+1)
+                f[g] = __viaddmax_s32(f[g], nb, tt);            // F(i+1, j)
+                hd[g] = H[i];
+                H[i] = h;
+                best = max(best, h);
+                if (i == K2R - 1) oh[g] = h;
+              }
+            }
+          }
+#pragma unroll
+          for (int g = 0; g < K2C; g++) hand[((t & 1) * K2C + g) * kK2Threads + L] = make_int2(oh[g], f[g]);
+          if (L == nact - 1 && ch < nch - 1)
+#pragma unroll
+            for (int g = 0; g < K2C; g++) {
+              const int col = tile * K2C + g;
+              border[2 * col] = oh[g];
+              border[2 * col + 1] = f[g];
+            }
+        } else if (active && L > 0 && tile == -1 && ntile > 0) {
+          cw_next = codes_of(0);   // first tile of this thread starts next step
         }
+        __syncthreads();
       }
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) best = max(best, __shfl_xor_sync(0xffffffffu, best, o));
-    if (lane == 0) a.scores[(int64_t)q * a.ndb + a.perm[s]] = best;
+    if (lane == 0) red_s[L >> 5] = best;
+    __syncthreads();
+    if (L == 0) {
+      int b = 0;
+      for (int w = 0; w < kK2Threads / 32; w++) b = max(b, red_s[w]);
+      a.scores[(int64_t)q * a.ndb + a.perm[s]] = b;
+    }
+    __syncthreads();   // claim_s / red_s / hand reused by the next pair
   }
 }
 
 void launch_k2(const K2Args &a, int blocks, cudaStream_t st) {
-  k2_kernel<<<blocks, 128, 0, st>>>(a);
+  cudaFuncSetAttribute(k2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kK2Smem);
+  k2_kernel<<<blocks, kK2Threads, kK2Smem, st>>>(a);
 }
 
 // ------------------------------------------------------------------------------------

@@ -102,15 +102,17 @@ struct K3Args {   // sequences [l0,l1) in sorted order (the long groups)
   const volatile int32_t *abort_flag;
   uint32_t na, nb;
 };
-struct K2Args {   // int32 re-run of saturated pairs (warp per pair)
+constexpr int kK2Blocks = 16;      // K2 blocks per launch (one block per saturated pair at a time)
+struct K2Args {   // int32 re-run of saturated pairs (block per pair)
   const uint8_t *qcodes; const int64_t *qoff;
   const uint4 *packed; const GroupInfo *groups; const int32_t *sorted_len; const int32_t *perm;
   const int8_t *matrix;                   // 24x24 (device)
   const int2 *ovf; const int32_t *ovf_count; int32_t ovf_cap;
-  int32_t *ovf_cursor;                    // warps take entries with atomicAdd
+  int32_t *ovf_cursor;                    // blocks take entries with atomicCAS
   int32_t *scores; int64_t ndb;
   int32_t alpha, beta;
-  int32_t *border; int64_t border_stride; int32_t n_warps_total;
+  int32_t one;                              // = 1 (opaque to the compiler, see k2_kernel)
+  int32_t *border; int64_t border_stride;   // per-block border row (2 x int32 per column)
 };
 
 struct TbPair {     // one pair of a traceback batch
