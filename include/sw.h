@@ -78,7 +78,7 @@ typedef struct {
   int32_t policy;            /* SW_POLICY_SS | SW_POLICY_PSS (default PSS) */
   int32_t workload_adjust;   /* 1 = WA on (default, P20 "always activated"), 0 = off */
   int32_t omega;             /* PSS history length (Omega, P18 §IV.A.2); default 4 (reading R10) */
-  int32_t streams_per_device;/* units in flight per GPU (default 4) */
+  int32_t streams_per_device;/* units in flight per GPU (default 4, at most 64) */
   int64_t target_unit_cells; /* cells per work unit; 0 = auto; INT64_MAX = one unit per
                                 query pair and kernel kind (the paper's very coarse
                                 "comparison of one query sequence to one genomic database",

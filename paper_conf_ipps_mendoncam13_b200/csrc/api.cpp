@@ -117,6 +117,7 @@ struct DevSearch {
   DBuf<int32_t> abort_dev;      // per-unit WA cancellation flags (device memory)
   int32_t *abort_d = nullptr;
   int32_t *one_h = nullptr;      // pinned constant 1, source of the cancellation copies
+  int32_t *ovf_seen_h = nullptr; // pinned [kMaxStreams]: ovf_count copied after each unit
   cudaStream_t cancel_st = nullptr;
   std::vector<char> cancelled;
   cudaEvent_t ev_start = nullptr, ev_end = nullptr;
@@ -153,6 +154,7 @@ struct Device {
 };
 inline DevSearch::~DevSearch() {
   if (one_h) cudaFreeHost(one_h);
+  if (ovf_seen_h) cudaFreeHost(ovf_seen_h);
   if (cancel_st) cudaStreamDestroy(cancel_st);
   if (ev_start) cudaEventDestroy(ev_start);
   if (ev_end) cudaEventDestroy(ev_end);
@@ -410,16 +412,19 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     a.ovf = S.ovf.p + (size_t)stream_idx * S.ovf_cap; a.ovf_count = S.ovf_count.p + stream_idx;
     a.ovf_cap = S.ovf_cap; a.ovf_bits = S.ovf_bits.p;
     const int64_t stride = (std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16;  // >= tiles * T
-    a.border = S.k3_border.p + (size_t)stream_idx * P.max_k3_seqs * stride;
+    a.border = S.k3_border.p + (size_t)stream_idx * P.max_k3_seqs * k3_phases() * stride;
     a.border_stride = stride;
     a.abort_flag = S.abort_d + uidx;
     a.na = na; a.nb = nbm;
     launch_k3(a, P.pairs[U.pair].rows_padded, st);
   }
   S.launches++;
-  // int32 re-run of the pairs this unit saturated, on its stream (overlaps other units)
-  launch_k2(k2_args(P, db, S, stream_idx, alpha, beta), kK2Blocks, st);
-  S.launches++;
+  // saturated pairs listed so far on this stream -> host (4 bytes): the worker launches
+  // the int32 re-run (K2) on this stream when the unit completes and the list grew.  K2's
+  // blocks need a whole SM's worth of shared memory, so an empty K2 launched after every
+  // unit would wait for a K1 block to leave and stall the stream.
+  CK(cudaMemcpyAsync(S.ovf_seen_h + stream_idx, S.ovf_count.p + stream_idx, sizeof(int32_t),
+                     cudaMemcpyDeviceToHost, st));
 }
 
 }  // namespace sw
@@ -517,6 +522,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
     if (opts_in) o = *opts_in;
     if (o.omega < 1) o.omega = 4;
     if (o.streams_per_device <= 0) o.streams_per_device = 4;
+    if (o.streams_per_device > kMaxStreams) throw Error(SW_EINVAL, "streams_per_device must be <= 64");
     if (o.policy != SW_POLICY_SS && o.policy != SW_POLICY_PSS) throw Error(SW_EINVAL, "bad policy");
     const bool dist = o.dist_world > 1;
     if (dist && (o.dist_rank < 0 || o.dist_rank >= o.dist_world || !o.dist_host || o.dist_port <= 0))
@@ -591,7 +597,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       X.ovf_cursor.ensure(D.id, depth);
       X.ovf_bits.ensure(D.id, ((size_t)nq * nd + 31) / 32);
       X.k2_border.ensure(D.id, (size_t)depth * kK2Blocks * std::max<int64_t>(P.max_len, 1) * 2);
-      const size_t k3b = (size_t)depth * std::max(P.max_k3_seqs, 1) *
+      const size_t k3b = (size_t)depth * std::max(P.max_k3_seqs, 1) * k3_phases() *
                          ((std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16);
       if (P.n_long_seqs > 0) X.k3_border.ensure(D.id, k3b);
       const size_t nu = std::max<size_t>(P.units.size(), 1);
@@ -602,6 +608,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       if (!X.one_h) {
         CK(cudaHostAlloc((void **)&X.one_h, sizeof(int32_t), cudaHostAllocDefault));
         *X.one_h = 1;
+        CK(cudaHostAlloc((void **)&X.ovf_seen_h, sizeof(int32_t) * kMaxStreams, cudaHostAllocDefault));
       }
       if (!X.cancel_st) CK(cudaStreamCreateWithFlags(&X.cancel_st, cudaStreamNonBlocking));
       if (!X.ev_start) CK(cudaEventCreate(&X.ev_start));
@@ -697,6 +704,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         std::vector<double> t_grant(P.units.size(), 0), t_launch(depth, 0);
         std::vector<double> hold_until(depth, 0);
         std::vector<int> completed_wait(depth, 0);
+        std::vector<int32_t> k2_upto(depth, 0);   // saturated pairs handed to K2 per stream
         bool done = false;
         double last_report = now_s();
         int32_t buf[64];
@@ -739,6 +747,15 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
             inflight[k] = -1;
             completed_wait[k] = 0;
             progressed = true;
+            // int32 re-run of what this unit saturated, on its stream before the next unit
+            // (overlaps the units in flight on the other streams)
+            const int32_t seen = ((volatile int32_t *)X.ovf_seen_h)[k];
+            if (seen > k2_upto[k]) {
+              launch_k2(k2_args(P, H, X, k, alpha, beta), kK2Blocks, D.streams[k]);
+              CK(cudaGetLastError());
+              X.launches++;
+              k2_upto[k] = seen;
+            }
           }
           // cancel in-flight replicas whose task finished elsewhere (WA loser)
           for (int k = 0; k < depth; k++)
@@ -779,7 +796,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
           if (!progressed)
             std::this_thread::sleep_for(std::chrono::microseconds(n_inflight > 0 ? 20 : 100));
         }
-        // the per-unit int32 re-runs ran on each stream after its units; check the lists
+        // the int32 re-runs ran on each stream after the units that saturated; check the lists
         for (int k = 0; k < depth; k++) CK(cudaStreamSynchronize(D.streams[k]));
         std::vector<int32_t> novf(depth, 0), ncur(depth, 0);
         CK(cudaMemcpy(novf.data(), X.ovf_count.p, sizeof(int32_t) * depth, cudaMemcpyDeviceToHost));

@@ -476,54 +476,83 @@ void launch_k1(const K1Args &a_in, int n_groups, int min_cols, int, cudaStream_t
 
 // ------------------------------------------------------------------------------------
 // K3: intra-task kernel for long DB sequences (P14 §II.B fine-grained approach, Fig. 3a:
-// "the calculations that can be done in parallel evolve as waves on diagonals").  One
-// warp per (query pair, long sequence); lane l owns rows [l*K, (l+1)*K) of each chunk of
-// 32*K query rows.  At step t lane l updates the T-column tile t - l (T columns give the
-// lane T independent dependency chains); it receives the bottom row (H, F) of that tile
-// and its 4 residue codes from lane l-1 by __shfl_up_sync, lane 0 takes them from the
-// previous chunk's border row (prefetched one step ahead) and the packed database, and
-// lane 31 writes the chunk's bottom row to the border.  Block = kK3Warps sequences that
-// share the chunk profile in shared memory laid out [code][row-in-lane][lane] (bank =
-// lane: conflict-free although every lane reads a different code).
+// "the calculations that can be done in parallel evolve as waves on diagonals").  A warp
+// works on one (query pack, long sequence) pair; lane l owns rows [l*K, (l+1)*K) of each
+// chunk of 32*K query rows.  At step t lane l updates the T-column tile t - l (T columns
+// give the lane T independent dependency chains); it receives the bottom row (H, F) of
+// that tile and its residue codes from lane l-1 by __shfl_up_sync, lane 0 takes them from
+// the previous chunk's border row and the packed database (streamed by cp.async through a
+// 3-deep shared-memory ring, two tiles ahead), and lane 31 writes the chunk's bottom row
+// to the border.
+//
+// Chunk phases (PH): the chunks of a pair are dealt round-robin to PH warps, chunk c to
+// phase c % PH, and phase p+1 runs chunk c+1 while phase p is still on chunk c (it reads
+// the border tile by tile, behind a per-warp progress counter in shared memory), so one
+// long pair takes about 1/PH of the single-warp latency: the fine-grained wavefront of
+// Fig. 3a applied once more, across warps ("it sends its border column to P1", P14).
+// Block = kK3Warps sequences x PH phases; the kK3Warps warps of a phase share that
+// phase's chunk profile in shared memory, laid out [code][row-in-lane][lane] (bank =
+// lane: conflict-free although every lane reads a different code).  Every dependency
+// points to a lower chunk (progress: chunk c waits for c-1; the phase barrier before
+// chunk c waits for c-PH), so the warps of a block cannot deadlock.
 // ------------------------------------------------------------------------------------
-template <int K, int T>
-__global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
+__device__ __forceinline__ void named_barrier(int id, int threads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(threads) : "memory");
+}
+
+template <int K, int T, int PH>
+__global__ void __launch_bounds__(kK3Warps * PH * 32) k3_kernel(const K3Args a) {
   static_assert(T == 4 || T == 8, "tile = one or two 32-bit words of packed residues");
   constexpr int NW = T / 4;          // 32-bit residue words per tile
   constexpr int TPU = 4 / NW;        // tiles per 128-bit word
   constexpr int CH = 32 * K;
-  extern __shared__ __align__(16) uint32_t smem[];  // [kNCodes][K][32], then the rings
-  uint4 *ring4 = reinterpret_cast<uint4 *>(smem + kNCodes * K * 32);   // [warps][3]
-  uint2 *ring2 = reinterpret_cast<uint2 *>(ring4 + kK3Warps * 3);      // [warps][3][T]
+  constexpr int NWARP = kK3Warps * PH;
+  constexpr int PROF = kNCodes * K * 32;   // words of one chunk profile
+  extern __shared__ __align__(16) uint32_t smem[];  // [PH][kNCodes][K][32], then the rings
+  uint4 *ring4 = reinterpret_cast<uint4 *>(smem + PH * PROF);      // [warps][3]
+  uint2 *ring2 = reinterpret_cast<uint2 *>(ring4 + NWARP * 3);    // [warps][3][T]
+  __shared__ int prog_s[NWARP];   // tiles of border published by each warp (all its chunks)
   if (block_aborted(a.abort_flag)) return;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int sw = warp % kK3Warps, ph = warp / kK3Warps;   // sequence slot, phase
+  if (threadIdx.x < NWARP) prog_s[threadIdx.x] = 0;
   const QueryPair P = a.pairs[a.pair];
   const int rows = P.rows;
   const int nch = (rows + CH - 1) / CH;
   const int nslices = P.rows_padded / 16;
-  const int s = a.l0 + blockIdx.x * kK3Warps + warp;
+  const int s = a.l0 + blockIdx.x * kK3Warps + sw;
   const bool valid = s < a.l1;
   const int len = valid ? a.sorted_len[s] : 0;
   const GroupInfo G = a.groups[valid ? s / kGroup : 0];
   const int gl = s % kGroup;
   const uint4 *wp = a.packed + G.word_off + gl;
-  uint2 *border = a.border + (size_t)(blockIdx.x * kK3Warps + warp) * a.border_stride;
+  // border rows: this warp writes its own (phase ph of sequence slot), reads the previous
+  // phase's (the previous chunk)
+  const size_t bslot = (size_t)(blockIdx.x * kK3Warps + sw) * PH;
+  uint2 *border_out = a.border + (bslot + ph) * a.border_stride;
+  const int pph = ph == 0 ? PH - 1 : ph - 1;
+  const uint2 *border_in = a.border + (bslot + pph) * a.border_stride;
+  const volatile int *prog_in = prog_s + pph * kK3Warps + sw;
   const uint32_t koff = pk2(kOff), na = a.na, nbeta = a.nb;
   const uint32_t padw = 0x01010101u * kPadCode;
   const int32_t *gprof = a.prof + P.prof_off;
+  uint32_t *prof_s = smem + ph * PROF;
   const int ntile = (len + T - 1) / T;   // columns up to ntile*T <= G.ncols carry pad codes
   const int orig = valid ? a.perm[s] : 0;
   uint32_t best = koff;
   int cq_lo = -1, cq_hi = -1;   // queries of this lane's slice (per half)
+  int published = 0;            // border tiles this warp has published (lane 31's count)
+  __syncthreads();              // prog_s initialised
 
-  for (int ch = 0; ch < nch; ch++) {
-    __syncthreads();
-    for (int idx = threadIdx.x; idx < kNCodes * CH; idx += kK3Warps * 32) {
+  for (int ch = ph; ch < nch; ch += PH) {
+    // the kK3Warps warps of this phase reload its chunk profile (all done with chunk ch-PH)
+    if (PH == 1) __syncthreads(); else named_barrier(1 + ph, kK3Warps * 32);
+    for (int idx = threadIdx.x - ph * kK3Warps * 32; idx < kNCodes * CH; idx += kK3Warps * 32) {
       const int c = idx / CH, r = idx - c * CH;     // r = l*K + i
       const int l = r / K, i = r - l * K;
-      smem[(c * K + i) * 32 + l] = (uint32_t)__ldg(gprof + (int64_t)c * P.rows_padded + ch * CH + r);
+      prof_s[(c * K + i) * 32 + l] = (uint32_t)__ldg(gprof + (int64_t)c * P.rows_padded + ch * CH + r);
     }
-    __syncthreads();
+    if (PH == 1) __syncthreads(); else named_barrier(1 + ph, kK3Warps * 32);
     if (!valid) continue;
     // lane l's rows of this chunk are slice ch*32 + l: flush a half whose query changed;
     // the start mask of the slice below applies to what this lane hands down
@@ -545,6 +574,9 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
     }
     if (len == 0) continue;
     const bool any_mask = __any_sync(0xffffffffu, omask != 0);   // warp-uniform
+    // border tiles of chunk ch-1 are published by phase pph as tiles
+    // base_in .. base_in + ntile - 1 of its running count
+    const int base_in = (ch - 1 - pph) / PH * ntile;
     uint32_t H[K], E[K];
 #pragma unroll
     for (int i = 0; i < K; i++) { H[i] = koff; E[i] = koff; }
@@ -561,9 +593,14 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
     auto fetch = [&](int tt) {             // lane 0: inputs of tile tt into slot tt % 3
       if (tt < ntile) {
         const int sl = tt % 3;
-        if (ch > 0)
+        if (ch > 0) {
+          if (PH > 1) {   // wait until the previous chunk's warp has published tile tt
+            while (*prog_in < base_in + tt + 1) __nanosleep(64);
+            __threadfence_block();
+          }
 #pragma unroll
-          for (int jj = 0; jj < T; jj++) cp_async8(&bring[sl * T + jj], &border[tt * T + jj]);
+          for (int jj = 0; jj < T; jj += 2) cp_async16(&bring[sl * T + jj], &border_in[tt * T + jj]);
+        }
         if (tt % TPU == 0) cp_async16(&wring[(tt / TPU) % 3], &wp[(size_t)(tt / TPU) * kGroup]);
       }
     };
@@ -609,7 +646,7 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
 #pragma unroll
         for (int jj = 0; jj < T; jj++) {
           const uint32_t c = (in_c[jj / 4] >> (8 * (jj % 4))) & 0xffu;
-          prc[jj] = smem + c * K * 32 + lane;
+          prc[jj] = prof_s + c * K * 32 + lane;
           hdc[jj] = hprev_top;
           out_f[jj] = in_f[jj];
           hprev_top = in_h[jj];
@@ -624,9 +661,14 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
         }
 #pragma unroll
         for (int q = 0; q < NW; q++) out_c[q] = in_c[q];
-        if (lane == 31 && ch < nch - 1)
+        if (lane == 31 && ch < nch - 1) {
 #pragma unroll
-          for (int jj = 0; jj < T; jj++) border[tile * T + jj] = make_uint2(out_h[jj], out_f[jj]);
+          for (int jj = 0; jj < T; jj++) border_out[tile * T + jj] = make_uint2(out_h[jj], out_f[jj]);
+          if (PH > 1) {   // publish: the border stores are ordered before the counter
+            __threadfence_block();
+            *(volatile int *)&prog_s[warp] = ++published;
+          }
+        }
       }
     }
   }
@@ -636,24 +678,32 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
   }
 }
 
-// K3 tile width (tuning; SW_K3_T): 8 columns per lane step (default) or 4
+// K3 tile width (tuning; SW_K3_T): 8 columns per lane step (default) or 4.  Chunk phases
+// (SW_K3_PHASES): 1 (default) or 2 -- measured slower on C4 (-2.7 %) and C5 (-11 %, also at
+// 1/8 of its database): with 16 warps per SM the SM is already busy, and the phase
+// barriers and the consumer's wait at each chunk start only add idle time.
 static int k3_tile() {
   static const int v = [] { const char *e = getenv("SW_K3_T"); return (e && atoi(e) == 4) ? 4 : 8; }();
   return v;
 }
+int k3_phases() {
+  static const int v = [] { const char *e = getenv("SW_K3_PHASES"); return (e && atoi(e) == 2) ? 2 : 1; }();
+  return v;
+}
+template <int T, int PH>
+static void k3_go(const K3Args &a, int n, cudaStream_t st) {
+  const size_t smem = sizeof(uint32_t) * PH * kNCodes * kK3Rows * 32 + sizeof(uint4) * kK3Warps * PH * 3 +
+                      sizeof(uint2) * kK3Warps * PH * 3 * T;
+  const int blocks = (n + kK3Warps - 1) / kK3Warps;
+  cudaFuncSetAttribute(k3_kernel<kK3Rows, T, PH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  k3_kernel<kK3Rows, T, PH><<<blocks, kK3Warps * PH * 32, smem, st>>>(a);
+}
 void launch_k3(const K3Args &a, int, cudaStream_t st) {
   const int n = a.l1 - a.l0;
   if (n <= 0) return;
-  const size_t smem = sizeof(uint32_t) * kNCodes * kK3Rows * 32 + sizeof(uint4) * kK3Warps * 3 +
-                      sizeof(uint2) * kK3Warps * 3 * 8;
-  const int blocks = (n + kK3Warps - 1) / kK3Warps;
-  if (k3_tile() == 4) {
-    cudaFuncSetAttribute(k3_kernel<kK3Rows, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    k3_kernel<kK3Rows, 4><<<blocks, kK3Warps * 32, smem, st>>>(a);
-  } else {
-    cudaFuncSetAttribute(k3_kernel<kK3Rows, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    k3_kernel<kK3Rows, 8><<<blocks, kK3Warps * 32, smem, st>>>(a);
-  }
+  const bool two = k3_phases() == 2;
+  if (k3_tile() == 4) { if (two) k3_go<4, 2>(a, n, st); else k3_go<4, 1>(a, n, st); }
+  else { if (two) k3_go<8, 2>(a, n, st); else k3_go<8, 1>(a, n, st); }
 }
 
 // ------------------------------------------------------------------------------------

@@ -98,10 +98,11 @@ struct K3Args {   // sequences [l0,l1) in sorted order (the long groups)
   int32_t *scores; int64_t ndb;
   int32_t thresh;
   int2 *ovf; int32_t *ovf_count; int32_t ovf_cap; uint32_t *ovf_bits;
-  uint2 *border; int64_t border_stride;   // per-warp border (>= max long len)
+  uint2 *border; int64_t border_stride;   // per (sequence, phase) border (>= max long len)
   const volatile int32_t *abort_flag;
   uint32_t na, nb;
 };
+constexpr int kMaxStreams = 64;    // sw_opts.streams_per_device limit
 constexpr int kK2Blocks = 16;      // K2 blocks per launch (one block per saturated pair at a time)
 struct K2Args {   // int32 re-run of saturated pairs (block per pair)
   const uint8_t *qcodes; const int64_t *qoff;
@@ -144,6 +145,7 @@ void launch_max_merge(int32_t *dst, const int32_t *src, int64_t n, cudaStream_t 
 void launch_topk(const int32_t *scores, int32_t nq, int64_t ndb, int32_t k, int2 *hits,
                  cudaStream_t st);
 int k1_blocks_per_sm();
+int k3_phases();   // warps per long pair (chunk phases of K3)
 int k1_band_rows();   // rows per K1 band (W*K of the selected variant)
 
 // ---- host packing (pack.cpp) ----------------------------------------------------------------

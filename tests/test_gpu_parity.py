@@ -107,6 +107,29 @@ def test_big_matrix_forces_many_overflows():
     assert r.stats["n_overflow_pairs"] >= 2
 
 
+def test_overflow_rerun_multi_chunk():
+    """K2 runs one block per saturated pair with 8,192-row chunks: a 9,500-aa overflowing
+    query crosses a chunk border (border row handed from the last active thread to thread
+    0), with its best cell below the border, and a gapped copy in a second sequence."""
+    q = b"W" * 3000 + seqgen.residues(21, 0, 6000).tobytes() + b"W" * 500
+    gapped = q[:8000] + b"PG" + q[8000:9000] + q[9003:]
+    base = seqgen.random_seqset(22, 40, 100, 3000)
+    seqs = [base.seq(i) for i in range(base.n)]
+    seqs[3] = b"KK" + q + b"EE"
+    seqs[17] = gapped
+    db = seqgen.SeqSet.from_list(seqs)
+    qs = seqgen.SeqSet.from_list([q, seqgen.residues(23, 0, 900).tobytes()])
+    ref = oracle.search(qs, db)
+    assert ref[0, 3] > 32767 and ref[0, 17] > 32767
+    r = _search(db, qs, top_k=3)
+    assert (r.scores == ref).all()
+    assert r.stats["n_overflow_pairs"] >= 2
+    # every pair through K2 (alpha + beta > 16384), several chunks, no saturation needed
+    ref2 = oracle.search(qs, db, gap_open=20000, gap_extend=3)
+    r2 = _search(db, qs, gap_open=20000, gap_extend=3, top_k=3)
+    assert (r2.scores == ref2).all()
+
+
 def test_precision_routing_large_gaps():
     """alpha + beta > 16384: every pair goes to the int32 kernel."""
     qs, db = _mixed_case(5, nq=4, nd=100, max_len=500)
