@@ -283,3 +283,22 @@ def test_topk_definition():
     assert i.tolist() == [[1, 2, 0], [0, 1, 2]]
     s, i = oracle.topk(scores, 7)
     assert i[0].tolist() == [1, 2, 0, 3, 4, -1, -1] and s[0, 5:].tolist() == [0, 0]
+
+
+def test_golden_digests_are_the_oracles():
+    """tests/golden/oracle_digests.json (used by the full-matrix GPU parity test) holds the
+    oracle's own digests: recompute the small config here and check the file's format."""
+    import hashlib
+    import json
+    import os
+    path = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden", "oracle_digests.json")
+    with open(path) as f:
+        g = json.load(f)
+    w = seqgen.make_workload("C1")
+    sc = oracle.search(w.queries, w.db)
+    assert g["C1"]["sha256_scores"] == hashlib.sha256(np.ascontiguousarray(sc, dtype="<i4").tobytes()).hexdigest()
+    s, i = oracle.topk(sc, 10)
+    assert g["C1"]["top10_scores"] == s.tolist() and g["C1"]["top10_index"] == i.tolist()
+    for cfg, e in g.items():
+        assert len(e["sha256_scores"]) == 64 and e["n_queries"] > 0 and e["n_db"] > 0
+        assert len(e["top10_index"]) == e["n_queries"]
