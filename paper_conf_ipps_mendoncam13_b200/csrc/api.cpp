@@ -1011,6 +1011,9 @@ int sw_align(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t 
       CK(cudaMemcpy(dp.p, batch.data(), sizeof(TbPair) * nb, cudaMemcpyHostToDevice));
       DBuf<uint8_t> ddir; ddir.alloc(D.id, std::max<int64_t>(dir_total, 1));
       DBuf<char> dops; dops.alloc(D.id, std::max<int64_t>(ops_total, 1));
+      // the kernel writes only the last n_ops bytes of each pair's area; the whole area is
+      // copied back, so clear it (compute-sanitizer initcheck clean)
+      CK(cudaMemset(dops.p, 0, std::max<int64_t>(ops_total, 1)));
       DBuf<TbResult> dres; dres.alloc(D.id, nb);
       DBuf<int32_t> dborder; dborder.alloc(D.id, (size_t)nb * max_n * 2);
       TbArgs a;
