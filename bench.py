@@ -186,6 +186,8 @@ def main():
     ap.add_argument("--streams", type=int, default=4)
     ap.add_argument("--unit-cells", type=int, default=0)
     ap.add_argument("--top-k", type=int, default=10)
+    ap.add_argument("--trace", default=None,
+                    help="write the last timed step's unit log as a Chrome trace (JSON) to this path")
     ap.add_argument("--long-threshold", type=int, default=0,
                     help="DB length routed to the intra-task kernel K3 (0 = libsw's auto)")
     args = ap.parse_args()
@@ -260,6 +262,10 @@ def main():
         stats.append(st)
     wall = time.perf_counter() - wall0
     clocks = sampler.stop()
+    if args.trace and rank == 0:
+        from paper_conf_ipps_mendoncam13_b200 import chrome_trace
+        with open(args.trace, "w") as f:
+            json.dump(chrome_trace(stats[-1].get("unit_log", []), name=f"{args.config} step"), f)
     if world > 1:
         tt = torch.tensor([dev_s], device="cuda", dtype=torch.float64)
         tdist.all_reduce(tt, op=tdist.ReduceOp.MAX)

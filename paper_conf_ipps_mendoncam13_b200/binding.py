@@ -180,6 +180,29 @@ class SearchResult:
     stats: dict
 
 
+def chrome_trace(unit_log, name="sw_search") -> dict:
+    """The per-unit event log of a search (stats["unit_log"]) as a Chrome-trace / Perfetto
+    JSON object (SURVEY §5 tracing): one process per worker (GPU), one thread per stream, a
+    complete event per unit replica (host clock from launch to observed completion; args:
+    cells, device_ms, committed, pack) and an instant event at each grant on a "master"
+    thread -- the analogue of the paper's per-interaction marks (P24 Figs. 7/8)."""
+    ev = []
+    workers = sorted({e["worker"] for e in unit_log})
+    for w in workers:
+        ev.append({"ph": "M", "name": "process_name", "pid": w, "args": {"name": f"{name}: worker {w}"}})
+        ev.append({"ph": "M", "name": "thread_name", "pid": w, "tid": -1, "args": {"name": "master grants"}})
+    for e in unit_log:
+        kind = "K1 inter-task" if e["kind"] == 0 else "K3 intra-task"
+        ev.append({"ph": "X", "name": f"unit {e['unit']} ({kind})", "cat": "unit",
+                   "pid": e["worker"], "tid": e.get("stream", 0),
+                   "ts": 1e6 * e["t_start"], "dur": max(0.0, 1e6 * (e["t_end"] - e["t_start"])),
+                   "args": {"cells": e["cells"], "pack": e["pair"], "committed": e["committed"],
+                            "device_ms": e.get("device_ms")}})
+        ev.append({"ph": "i", "name": f"grant unit {e['unit']}", "cat": "grant", "s": "t",
+                   "pid": e["worker"], "tid": -1, "ts": 1e6 * e["t_grant"]})
+    return {"traceEvents": ev, "displayTimeUnit": "ms"}
+
+
 def _stats_dict(st: sw_stats) -> dict:
     d = {k: getattr(st, k) for k, _ in sw_stats._fields_ if k != "unit_log_json"}
     d["unit_log"] = json.loads(st.unit_log_json.decode()) if st.unit_log_json else []

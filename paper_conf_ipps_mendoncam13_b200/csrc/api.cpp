@@ -356,10 +356,11 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
 
 // ---------------------------------------------------------------- per-search device state
 struct UnitLog {
-  int32_t unit, worker;
-  double t_grant, t_start, t_end;
+  int32_t unit, worker, stream;
+  double t_grant, t_start, t_end;   // host clock (s since the search start)
   int64_t cells;
   int committed;
+  float device_ms;                  // CUDA events around the unit's kernels on its stream
 };
 
 static const int kOvfCap = 1 << 20;
@@ -742,7 +743,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
             if (!committed) X.dup_cells += U.cells;
             {
               std::lock_guard<std::mutex> g(ulog_mu);
-              ulog.push_back({u, wid, t_grant[u] - t0, t_launch[k] - t0, tn - t0, U.cells, committed});
+              ulog.push_back({u, wid, k, t_grant[u] - t0, t_launch[k] - t0, tn - t0, U.cells, committed, ms});
             }
             inflight[k] = -1;
             completed_wait[k] = 0;
@@ -925,7 +926,8 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         const Unit &U = P.units[L.unit];
         js << (k ? "," : "") << "{\"unit\":" << L.unit << ",\"kind\":" << U.kind << ",\"pair\":" << U.pair
            << ",\"worker\":" << L.worker << ",\"t_grant\":" << L.t_grant << ",\"t_start\":" << L.t_start
-           << ",\"t_end\":" << L.t_end << ",\"cells\":" << L.cells << ",\"committed\":" << L.committed << "}";
+           << ",\"t_end\":" << L.t_end << ",\"cells\":" << L.cells << ",\"committed\":" << L.committed
+           << ",\"stream\":" << L.stream << ",\"device_ms\":" << L.device_ms << "}";
       }
       js << "]";
       db->unit_log = js.str();

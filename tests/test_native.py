@@ -1,6 +1,7 @@
 """Host-side native checks (no GPU): libsw loads and exports every symbol include/*.h
 declares; its BLOSUM62 transcription matches the checksums and the oracle's copy; the
 multi-process master/slave protocol (TCP) and the cross-rank merge (gloo, world 2)."""
+import json
 import multiprocessing as mp
 import os
 import re
@@ -167,3 +168,21 @@ def test_gloo_world2_merge():
     for p in procs:
         p.join(timeout=60)
     assert all(o[1] and o[2] for o in out), out
+
+
+def test_chrome_trace_of_a_unit_log():
+    """The per-unit event log exports as a Chrome trace: one complete event per unit replica
+    on (worker, stream), one grant mark per unit, process/thread names."""
+    from paper_conf_ipps_mendoncam13_b200 import chrome_trace
+    log = [dict(unit=0, kind=0, pair=0, worker=0, stream=1, t_grant=0.0, t_start=0.001, t_end=0.011,
+                cells=10**9, committed=1, device_ms=9.5),
+           dict(unit=1, kind=1, pair=2, worker=1, stream=0, t_grant=0.002, t_start=0.003, t_end=0.04,
+                cells=3 * 10**9, committed=0, device_ms=36.0)]
+    tr = chrome_trace(log)
+    ev = tr["traceEvents"]
+    units = [e for e in ev if e["ph"] == "X"]
+    assert len(units) == 2 and len([e for e in ev if e["ph"] == "i"]) == 2
+    assert units[0]["pid"] == 0 and units[0]["tid"] == 1 and abs(units[0]["dur"] - 1e4) < 1e-6
+    assert units[1]["args"]["committed"] == 0 and "K3" in units[1]["name"]
+    assert {e["pid"] for e in ev if e["ph"] == "M"} == {0, 1}
+    json.dumps(tr)
