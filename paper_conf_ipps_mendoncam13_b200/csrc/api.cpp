@@ -312,11 +312,27 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
   for (int32_t p = 0; p < (int32_t)P.pairs.size(); p++) {
     const QueryPair &qp = P.pairs[p];
     const int64_t rows_eff = P.real_rows[p];
-    // K3 units over the long sequences (multiples of kK3Warps)
+    // K3 units over the long sequences (multiples of kK3Warps), cut greedily at k3_target
+    // cells (the last unit of a pack is the remainder: a short unit that fills the tail).
+    // A K3 launch runs one warp per sequence, so a unit needs many sequences to cover the
+    // SMs: k3_target is at least 4x the unit target and at least the cells of kK3UnitSeqs
+    // average sequences (one block per B200 SM); with several workers it is capped so that
+    // every stream of every worker gets a unit of each pack's long work.  (An explicit
+    // target_unit_cells is taken as given: 4x it per K3 unit.)
+    int64_t long_cells = 0;
+    for (int32_t s = 0; s < P.n_long_seqs; s++) long_cells += rows_eff * db.sorted_len[s];
+    const int64_t n_packs = (int64_t)P.pairs.size();
+    const int64_t t4 = target > INT64_MAX / 4 ? INT64_MAX : 4 * target;   // INT64_MAX: very coarse
+    int64_t k3_target = t4;
+    if (P.n_long_seqs > 0 && o.target_unit_cells <= 0) {   // auto sizing only
+      k3_target = std::max<int64_t>(t4, long_cells / P.n_long_seqs * kK3UnitSeqs);
+      const int64_t per_pack = ((int64_t)n_workers * depth + n_packs - 1) / n_packs;
+      if (per_pack > 1) k3_target = std::max<int64_t>(1, std::min<int64_t>(k3_target, (long_cells + per_pack - 1) / per_pack));
+    }
     for (int32_t s = 0; s < P.n_long_seqs;) {
       int32_t e = s;
       int64_t cells = 0, work = 0;
-      while (e < P.n_long_seqs && (cells < 4 * target || e == s || (e - s) % kK3Warps)) {
+      while (e < P.n_long_seqs && (cells < k3_target || e == s || (e - s) % kK3Warps)) {
         cells += rows_eff * db.sorted_len[e];
         work += (int64_t)qp.rows_padded * db.sorted_len[e];
         e++;

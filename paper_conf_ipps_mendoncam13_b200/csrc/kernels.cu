@@ -514,7 +514,10 @@ __global__ void __launch_bounds__(kK3Warps * PH * 32) k3_kernel(const K3Args a) 
   __shared__ int prog_s[NWARP];   // tiles of border published by each warp (all its chunks)
   if (block_aborted(a.abort_flag)) return;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int sw = warp % kK3Warps, ph = warp / kK3Warps;   // sequence slot, phase
+  // sequence slot, phase: the PH warps of a sequence are consecutive, so producer and
+  // consumer sit on different SM sub-partitions (warp % 4) and a waiting consumer does
+  // not take issue slots from its own producer
+  const int sw = warp / PH, ph = warp % PH;
   if (threadIdx.x < NWARP) prog_s[threadIdx.x] = 0;
   const QueryPair P = a.pairs[a.pair];
   const int rows = P.rows;
@@ -532,7 +535,7 @@ __global__ void __launch_bounds__(kK3Warps * PH * 32) k3_kernel(const K3Args a) 
   uint2 *border_out = a.border + (bslot + ph) * a.border_stride;
   const int pph = ph == 0 ? PH - 1 : ph - 1;
   const uint2 *border_in = a.border + (bslot + pph) * a.border_stride;
-  const volatile int *prog_in = prog_s + pph * kK3Warps + sw;
+  const volatile int *prog_in = prog_s + sw * PH + pph;
   const uint32_t koff = pk2(kOff), na = a.na, nbeta = a.nb;
   const uint32_t padw = 0x01010101u * kPadCode;
   const int32_t *gprof = a.prof + P.prof_off;
@@ -547,7 +550,7 @@ __global__ void __launch_bounds__(kK3Warps * PH * 32) k3_kernel(const K3Args a) 
   for (int ch = ph; ch < nch; ch += PH) {
     // the kK3Warps warps of this phase reload its chunk profile (all done with chunk ch-PH)
     if (PH == 1) __syncthreads(); else named_barrier(1 + ph, kK3Warps * 32);
-    for (int idx = threadIdx.x - ph * kK3Warps * 32; idx < kNCodes * CH; idx += kK3Warps * 32) {
+    for (int idx = sw * 32 + lane; idx < kNCodes * CH; idx += kK3Warps * 32) {
       const int c = idx / CH, r = idx - c * CH;     // r = l*K + i
       const int l = r / K, i = r - l * K;
       prof_s[(c * K + i) * 32 + l] = (uint32_t)__ldg(gprof + (int64_t)c * P.rows_padded + ch * CH + r);
@@ -595,7 +598,7 @@ __global__ void __launch_bounds__(kK3Warps * PH * 32) k3_kernel(const K3Args a) 
         const int sl = tt % 3;
         if (ch > 0) {
           if (PH > 1) {   // wait until the previous chunk's warp has published tile tt
-            while (*prog_in < base_in + tt + 1) __nanosleep(64);
+            while (*prog_in < base_in + tt + 1) {}
             __threadfence_block();
           }
 #pragma unroll

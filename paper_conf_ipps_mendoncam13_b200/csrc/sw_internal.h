@@ -34,6 +34,7 @@ constexpr int kK1Band = kK1Rows * kK1Warps;
 constexpr int kK3Rows = 16;        // rows per lane
 constexpr int kK3Chunk = 32 * kK3Rows;   // rows per warp chunk
 constexpr int kK3Warps = 4;        // long sequences per block (share the chunk profile)
+constexpr int kK3UnitSeqs = 148 * kK3Warps;   // long sequences that give each B200 SM one K3 block
 constexpr int kProfileRowAlign = 512;    // lcm(kK1Band, kK3Chunk)
 
 // ---- packed database (device) -------------------------------------------------------
