@@ -362,11 +362,30 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
   // so that every pair gets written, but they must have cells > 0 for the scheduler)
   for (auto &u : P.units) u.cells = std::max<int64_t>(u.cells, 1);
   // LPT by expected duration: intra-task (long-sequence) units first -- each warp walks a
-  // whole long pair, so they have the longest latency -- then inter-task units by work
-  std::stable_sort(P.units.begin(), P.units.end(), [](const Unit &a, const Unit &b) {
-    if (a.kind != b.kind) return a.kind == kUnitIntra;
+  // whole long pair, so they have the longest latency -- then inter-task units by work.
+  // A small K3 unit (fewer sequences than one block per SM) is interleaved with the largest
+  // K1 units instead (K3, K1, K3, K1, ...): small K3 units alone on every stream would
+  // leave SMs idle at the start of the step (C4 at 1/8 of its database: 140 ms of 447)
+  auto small3 = [](const Unit &u) { return u.kind == kUnitIntra && u.b1 - u.b0 < kK3UnitSeqs; };
+  std::stable_sort(P.units.begin(), P.units.end(), [&](const Unit &a, const Unit &b) {
+    const int ra = a.kind == kUnitIntra ? (small3(a) ? 1 : 0) : 2;
+    const int rb = b.kind == kUnitIntra ? (small3(b) ? 1 : 0) : 2;
+    if (ra != rb) return ra < rb;
     return a.work > b.work;
   });
+  {
+    size_t nb = 0, ns = 0;
+    while (nb < P.units.size() && P.units[nb].kind == kUnitIntra && !small3(P.units[nb])) nb++;
+    ns = nb;
+    while (ns < P.units.size() && small3(P.units[ns])) ns++;
+    std::vector<Unit> order(P.units.begin(), P.units.begin() + nb);
+    size_t i3 = nb, i1 = ns;
+    while (i3 < ns || i1 < P.units.size()) {
+      if (i3 < ns) order.push_back(P.units[i3++]);
+      if (i1 < P.units.size()) order.push_back(P.units[i1++]);
+    }
+    P.units.swap(order);
+  }
   return P;
 }
 
