@@ -388,3 +388,22 @@ def test_unusual_inputs():
         bad = np.argwhere(r.scores != ref)
         assert len(bad) == 0, (thr, bad[:5])
         _check_topk(r, ref, 6)
+
+
+def test_extreme_lengths():
+    """Beyond the paper's shapes: database sequences of 120,000 and 70,000 residues and a
+    60,000-aa query (118 K3 chunks, 469 K1 bands), through K3 (auto threshold) and through
+    K1 alone (threshold above every length: 120,000-column groups and border rows)."""
+    q_short = seqgen.residues(31, 0, 300).tobytes()
+    long1 = seqgen.residues(32, 0, 120000).tobytes()
+    long1 = long1[:50000] + q_short + long1[50300:]
+    db = [long1, seqgen.residues(33, 0, 70000).tobytes()] + \
+         [seqgen.residues(34, k * 1000, 200 + 13 * k).tobytes() for k in range(40)]
+    qs = seqgen.SeqSet.from_list([seqgen.residues(35, 0, 2000).tobytes(), q_short,
+                                  seqgen.residues(36, 0, 60000).tobytes()])
+    dbs = seqgen.SeqSet.from_list(db)
+    ref = oracle.search(qs, dbs)
+    for thr in (0, 1 << 20):
+        r = _search(dbs, qs, top_k=4, long_threshold=thr)
+        assert (r.scores == ref).all(), (thr, np.argwhere(r.scores != ref)[:5])
+        _check_topk(r, ref, 4)
