@@ -21,7 +21,7 @@ import numpy as np  # noqa: E402
 import oracle  # noqa: E402
 import seqgen  # noqa: E402
 
-OUT = os.path.join(ROOT, "tests", "golden", "oracle_digests.json")
+OUT = os.environ.get("GOLDEN_OUT") or os.path.join(ROOT, "tests", "golden", "oracle_digests.json")
 
 
 def digest(scores: np.ndarray) -> str:
