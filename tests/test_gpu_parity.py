@@ -407,3 +407,33 @@ def test_extreme_lengths():
         r = _search(dbs, qs, top_k=4, long_threshold=thr)
         assert (r.scores == ref).all(), (thr, np.argwhere(r.scores != ref)[:5])
         _check_topk(r, ref, 4)
+
+
+_PHASES_SCRIPT = r"""
+import sys; sys.path.insert(0, %r)
+import numpy as np, oracle, seqgen
+from paper_conf_ipps_mendoncam13_b200 import Database
+qs = seqgen.SeqSet.from_list([seqgen.residues(41, 0, L).tobytes() for L in (1300, 600, 17, 3000)])
+db = seqgen.random_seqset(42, 300, 0, 4000)
+db = seqgen.SeqSet.from_list([db.seq(i) for i in range(db.n)] + [b"W" * 3000])
+ref = oracle.search(qs, db)
+D = Database(db, devices=[0])
+for thr in (0, 500):
+    r = D.search(qs, top_k=3, long_threshold=thr)
+    assert (r.scores == ref).all(), np.argwhere(r.scores != ref)[:5]
+D.close()
+print("ok")
+"""
+
+
+def test_k3_chunk_phases_option():
+    """SW_K3_PHASES=2 (two warps per long pair, pipelined over chunks behind a progress
+    counter; an option, not the default): bit-exact, several chunks per phase, K2 re-run."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, SW_K3_PHASES="2")
+    out = subprocess.run([sys.executable, "-c", _PHASES_SCRIPT % root], env=env, capture_output=True,
+                         text=True, timeout=600)
+    assert out.returncode == 0 and out.stdout.strip().endswith("ok"), out.stderr[-2000:]
