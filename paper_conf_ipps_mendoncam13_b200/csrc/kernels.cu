@@ -28,6 +28,8 @@
 
 namespace sw {
 
+constexpr bool kK1PairLoads = true;   // K1 reads two profile rows per LDS.64
+__constant__ uint8_t c_code_of_slot[kNCodes] = SW_CODE_OF_SLOT_INIT;   // database slot -> code
 __device__ __forceinline__ uint32_t pk2(int v) { return ((uint32_t)(v & 0xffff)) * 0x10001u; }
 __device__ __forceinline__ void cp_async8(void *smem_dst, const void *gsrc) {
   const unsigned d = (unsigned)__cvta_generic_to_shared(smem_dst);
@@ -58,8 +60,8 @@ __device__ __forceinline__ uint32_t smid() {
 }
 
 // ------------------------------------------------------------------------------------
-// K4: query-pair profiles.  prof[pair][c][row] = S_b*65536 + S_a (signed-packed int32),
-// S_a = S[qa_row][c] (kPadScore past the end of qa or for the pad code), same for qb.
+// K4: query-pair profiles.  prof[pair][c][row] = S_b*65536 + S_a (signed-packed int32), c = database slot,
+// S_a = S[qa_row][code of slot c] (kPadScore past the end of qa or for the pad code), same for qb.
 // ------------------------------------------------------------------------------------
 __global__ void profile_kernel(const uint8_t *__restrict__ qcodes, const int64_t *__restrict__ qoff,
                                const QueryPair *__restrict__ pairs, const SliceInfo *__restrict__ slices,
@@ -71,14 +73,15 @@ __global__ void profile_kernel(const uint8_t *__restrict__ qcodes, const int64_t
     const int c = (int)(k / P.rows_padded), row = (int)(k % P.rows_padded);
     const SliceInfo si = slices[P.slice_off + row / 16];
     int sa = kPadScore, sb = kPadScore;
-    if (c < 24) {
+    if (c < 24) {   // c = database slot
+      const int dc = c_code_of_slot[c];
       if (si.q_lo >= 0) {
         const int64_t r = si.off_lo + row % 16;
-        if (r < qoff[si.q_lo + 1] - qoff[si.q_lo]) sa = M[qcodes[qoff[si.q_lo] + r] * 24 + c];
+        if (r < qoff[si.q_lo + 1] - qoff[si.q_lo]) sa = M[qcodes[qoff[si.q_lo] + r] * 24 + dc];
       }
       if (si.q_hi >= 0) {
         const int64_t r = si.off_hi + row % 16;
-        if (r < qoff[si.q_hi + 1] - qoff[si.q_hi]) sb = M[qcodes[qoff[si.q_hi] + r] * 24 + c];
+        if (r < qoff[si.q_hi + 1] - qoff[si.q_hi]) sb = M[qcodes[qoff[si.q_hi] + r] * 24 + dc];
       }
     }
     prof[P.prof_off + k] = sb * 65536 + sa;
@@ -141,18 +144,28 @@ __device__ __forceinline__ uint32_t start_mask(const SliceInfo &n) {
 // are interleaved explicitly: at step k column g updates row k - g.  Column g starts with
 // diagonal hdc[g] and top F fc[g]; on return out_h[g] / fc[g] hold its bottom-row H and
 // the F passed down.  PS = profile stride between consecutive rows.
-template <int K, int G, int PS>
+// PAIR (PS == 1, 8-byte aligned rows): the profile of rows i, i+1 is read with one LDS.64.
+template <int K, int G, int PS, bool PAIR = false>
 __device__ __forceinline__ void dp_tile(const uint32_t *const (&prc)[G], uint32_t (&H)[K],
                                         uint32_t (&E)[K], uint32_t (&hdc)[G], uint32_t (&fc)[G],
                                         uint32_t (&out_h)[G], uint32_t &best, uint32_t na, uint32_t nb,
                                         uint32_t koff) {
+  static_assert(!PAIR || (PS == 1 && K % 2 == 0), "pair loads need consecutive rows");
+  uint2 pv[G];
 #pragma unroll
   for (int k = 0; k < K + G - 1; k++) {
 #pragma unroll
     for (int g = 0; g < G; g++) {
       const int i = k - g;
       if (i >= 0 && i < K) {
-        Cell::row(prc[g][i * PS], hdc[g], H[i], E[i], fc[g], best, na, nb, koff);
+        uint32_t v;
+        if (PAIR) {
+          if ((i & 1) == 0) pv[g] = *reinterpret_cast<const uint2 *>(prc[g] + i);
+          v = (i & 1) ? pv[g].y : pv[g].x;
+        } else {
+          v = prc[g][i * PS];
+        }
+        Cell::row(v, hdc[g], H[i], E[i], fc[g], best, na, nb, koff);
         if (i == K - 1) out_h[g] = H[K - 1];
       }
     }
@@ -172,8 +185,9 @@ template <int K, int W, int T, int MINB, int UQ>
 __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   static_assert(T == 4 || T == 8 || T == 16, "tile = 1, 2 or 4 32-bit words of residues");
   constexpr int BAND = W * K;
-  constexpr int S = BAND + 1;  // odd stride: lanes reading one row with different codes hit
-                               // different banks
+  // profile stride: odd (lanes reading one row with different codes hit different banks),
+  // or even with pair loads (rows i, i+1 of one code in one LDS.64)
+  constexpr int S = kK1PairLoads ? BAND + 2 : BAND + 1;
   constexpr int TPW = kWordCols / T;   // tiles per 16-column residue word
   extern __shared__ __align__(16) uint32_t smem[];
   uint32_t *prof_s = smem;                                            // [2][kNCodes][S]
@@ -345,7 +359,7 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
           fc[j] = v.y;
           hprev_top = v.x;
         }
-        dp_tile<K, GS, 1>(prc, H, E, hdc, fc, oh, best, na, nbeta, koff);
+        dp_tile<K, GS, 1, kK1PairLoads>(prc, H, E, hdc, fc, oh, best, na, nbeta, koff);
         if (omask) {   // the slice below starts a query: it sees H = F = 0 above
 #pragma unroll
           for (int j = 0; j < GS; j++) {
@@ -395,7 +409,7 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
 
 template <int W, int T>
 static size_t k1_smem() {
-  constexpr int S = kK1Rows * W + 1;
+  constexpr int S = kK1PairLoads ? kK1Rows * W + 2 : kK1Rows * W + 1;
   return sizeof(uint32_t) * 2 * kNCodes * S + sizeof(uint2) * W * 2 * T * 32 +
          sizeof(uint32_t) * 2 * W * 32 + sizeof(uint2) * 3 * T * 32;
 }
@@ -736,8 +750,8 @@ __global__ void __launch_bounds__(kK2Threads, 1) k2_kernel(const K2Args a) {
   const int count = min(*a.ovf_count, a.ovf_cap);
   if (*(volatile int32_t *)a.ovf_cursor >= count) return;   // nothing saturated (the usual case)
   for (int k = threadIdx.x; k < kNCodes * kNCodes * 32; k += kK2Threads) {
-    const int r = k / (kNCodes * 32), c = (k / 32) % kNCodes;
-    Ms[k] = (r < 24 && c < 24) ? (int32_t)a.matrix[r * 24 + c] : kPadScore;
+    const int r = k / (kNCodes * 32), c = (k / 32) % kNCodes;   // query code, database slot
+    Ms[k] = (r < 24 && c < 24) ? (int32_t)a.matrix[r * 24 + c_code_of_slot[c]] : kPadScore;
   }
   const int L = threadIdx.x, lane = L & 31;
   const uint32_t *words = reinterpret_cast<const uint32_t *>(a.packed);
@@ -889,8 +903,8 @@ constexpr int K6R = 8;
 __global__ void __launch_bounds__(32) traceback_kernel(const TbArgs a) {
   __shared__ int32_t Ms[kNCodes * 32];
   for (int k = threadIdx.x; k < kNCodes * 32; k += 32) {
-    const int r = k / 32, c = k % 32;
-    Ms[k] = (r < 24 && c < 24) ? (int32_t)a.matrix[r * 24 + c] : kPadScore;
+    const int r = k / 32, c = k % 32;   // query code, database slot
+    Ms[k] = (r < 24 && c < 24) ? (int32_t)a.matrix[r * 24 + c_code_of_slot[c]] : kPadScore;
   }
   __syncwarp();
   const int lane = threadIdx.x;

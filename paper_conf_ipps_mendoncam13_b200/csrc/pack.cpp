@@ -92,6 +92,16 @@ const int8_t *blosum62() {
   return m;
 }
 
+// database residue code -> slot (sw_internal.h: SW_CODE_OF_SLOT_INIT, inverted)
+static const struct SlotTable {
+  uint8_t v[kNCodes];
+  SlotTable() {
+    const uint8_t code_of_slot[kNCodes] = SW_CODE_OF_SLOT_INIT;
+    for (int sl = 0; sl < kNCodes; sl++) v[code_of_slot[sl]] = (uint8_t)sl;
+  }
+} slot_table;
+static const uint8_t *const slot_of_code = slot_table.v;
+
 int pack_database(const int64_t *offsets, const char *residues, int32_t n, PackedDB &out,
                   std::string &err) {
   out = PackedDB();
@@ -154,7 +164,7 @@ int pack_database(const int64_t *offsets, const char *residues, int32_t n, Packe
         uint8_t *dst = bytes + ((G.word_off + (int64_t)w * kGroup + lane) * 16);
         for (int b = 0; b < kWordCols; b++) {
           int32_t j = w * kWordCols + b;
-          dst[b] = (j < l) ? (uint8_t)encode_residue((unsigned char)src[j]) : (uint8_t)kPadCode;
+          dst[b] = (j < l) ? slot_of_code[encode_residue((unsigned char)src[j])] : (uint8_t)kPadCode;
         }
       }
     }

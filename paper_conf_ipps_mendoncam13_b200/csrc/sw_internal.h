@@ -20,6 +20,14 @@ struct Error : std::runtime_error {
 constexpr int kNCodes = 25;        // 24 NCBI letters ARNDCQEGHILKMFPSTWYVBZX* + pad
 constexpr int kPadCode = 24;       // packing pad (DB columns beyond a sequence's end)
 constexpr int kPadScore = -1;      // S[.][pad] and pad query rows: <= 0 (reading R9)
+// Database residues are stored in the packed database as "slots", a permutation of the
+// codes: the K1 profile is read two rows per LDS.64 with a row stride of 65 8-byte words,
+// so the bank pair a lane hits is slot mod 16.  The 16 most frequent amino acids (Swiss-Prot
+// composition) get slots 0..15, one bank pair each; M H C W B Z X * share bank pairs with
+// the 8 least frequent of them (slots 16..23); the pad code keeps slot 24.  Profiles, the
+// K2/K6 matrices and the K3 profile are indexed by slot; query rows stay codes.
+//                                     slot: 0  1  2 3  4  5 6 7  8 9 10 11 12 13 14 15 16 17 18 19 20 21 22 23 24
+#define SW_CODE_OF_SLOT_INIT            {18,13,5,2,14,16,3,1,10,0, 7,19, 6,15, 9,11,12, 8, 4,17,20,21,22,23,24}
 constexpr int kOff = 128;          // offset representation bias of the s16x2 kernels
                                    // (>= -min int8 score so 32-bit adds never borrow)
 constexpr int kWordCols = 16;      // residues per packed 128-bit word
