@@ -144,13 +144,14 @@ __device__ __forceinline__ uint32_t start_mask(const SliceInfo &n) {
 // are interleaved explicitly: at step k column g updates row k - g.  Column g starts with
 // diagonal hdc[g] and top F fc[g]; on return out_h[g] / fc[g] hold its bottom-row H and
 // the F passed down.  PS = profile stride between consecutive rows.
-// PAIR (PS == 1, 8-byte aligned rows): the profile of rows i, i+1 is read with one LDS.64.
-template <int K, int G, int PS, bool PAIR = false>
+// PAIR: the profile of rows i, i+1 (i even) is one 8-byte word at prc + (i/2)*PPS, read
+// with one LDS.64 (K1: consecutive rows, PPS = 2; K3: row pairs interleaved per lane, PPS = 64).
+template <int K, int G, int PS, bool PAIR = false, int PPS = 2>
 __device__ __forceinline__ void dp_tile(const uint32_t *const (&prc)[G], uint32_t (&H)[K],
                                         uint32_t (&E)[K], uint32_t (&hdc)[G], uint32_t (&fc)[G],
                                         uint32_t (&out_h)[G], uint32_t &best, uint32_t na, uint32_t nb,
                                         uint32_t koff) {
-  static_assert(!PAIR || (PS == 1 && K % 2 == 0), "pair loads need consecutive rows");
+  static_assert(!PAIR || K % 2 == 0, "pair loads need an even row count");
   uint2 pv[G];
 #pragma unroll
   for (int k = 0; k < K + G - 1; k++) {
@@ -160,7 +161,7 @@ __device__ __forceinline__ void dp_tile(const uint32_t *const (&prc)[G], uint32_
       if (i >= 0 && i < K) {
         uint32_t v;
         if (PAIR) {
-          if ((i & 1) == 0) pv[g] = *reinterpret_cast<const uint2 *>(prc[g] + i);
+          if ((i & 1) == 0) pv[g] = *reinterpret_cast<const uint2 *>(prc[g] + (i / 2) * PPS);
           v = (i & 1) ? pv[g].y : pv[g].x;
         } else {
           v = prc[g][i * PS];
@@ -567,7 +568,10 @@ __global__ void __launch_bounds__(kK3Warps * PH * 32) k3_kernel(const K3Args a) 
     for (int idx = sw * 32 + lane; idx < kNCodes * CH; idx += kK3Warps * 32) {
       const int c = idx / CH, r = idx - c * CH;     // r = l*K + i
       const int l = r / K, i = r - l * K;
-      prof_s[(c * K + i) * 32 + l] = (uint32_t)__ldg(gprof + (int64_t)c * P.rows_padded + ch * CH + r);
+      // [slot][row pair][lane][2]: a lane's rows i, i+1 form one 8-byte word (LDS.64); the
+      // 8-byte bank pair is lane mod 16, so no conflicts although lanes read different slots
+      prof_s[((c * (K / 2) + i / 2) * 32 + l) * 2 + (i & 1)] =
+          (uint32_t)__ldg(gprof + (int64_t)c * P.rows_padded + ch * CH + r);
     }
     if (PH == 1) __syncthreads(); else named_barrier(1 + ph, kK3Warps * 32);
     if (!valid) continue;
@@ -663,12 +667,12 @@ __global__ void __launch_bounds__(kK3Warps * PH * 32) k3_kernel(const K3Args a) 
 #pragma unroll
         for (int jj = 0; jj < T; jj++) {
           const uint32_t c = (in_c[jj / 4] >> (8 * (jj % 4))) & 0xffu;
-          prc[jj] = prof_s + c * K * 32 + lane;
+          prc[jj] = prof_s + (c * (K / 2) * 32 + lane) * 2;
           hdc[jj] = hprev_top;
           out_f[jj] = in_f[jj];
           hprev_top = in_h[jj];
         }
-        dp_tile<K, T, 32>(prc, H, E, hdc, out_f, out_h, best, na, nbeta, koff);
+        dp_tile<K, T, 32, true, 64>(prc, H, E, hdc, out_f, out_h, best, na, nbeta, koff);
         if (any_mask) {   // bit-select: omask is 0 except in a lane above a query start
 #pragma unroll
           for (int jj = 0; jj < T; jj++) {
