@@ -366,7 +366,8 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
   // A small K3 unit (fewer sequences than one block per SM) is interleaved with the largest
   // K1 units instead (K3, K1, K3, K1, ...): small K3 units alone on every stream would
   // leave SMs idle at the start of the step (C4 at 1/8 of its database: 140 ms of 447)
-  auto small3 = [](const Unit &u) { return u.kind == kUnitIntra && u.b1 - u.b0 < kK3UnitSeqs; };
+  static const bool interleave = [] { const char *e = getenv("SW_UNIT_INTERLEAVE"); return !(e && atoi(e) == 0); }();
+  auto small3 = [](const Unit &u) { return interleave && u.kind == kUnitIntra && u.b1 - u.b0 < kK3UnitSeqs; };
   std::stable_sort(P.units.begin(), P.units.end(), [&](const Unit &a, const Unit &b) {
     const int ra = a.kind == kUnitIntra ? (small3(a) ? 1 : 0) : 2;
     const int rb = b.kind == kUnitIntra ? (small3(b) ? 1 : 0) : 2;
@@ -765,7 +766,9 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
                 hold_until[k] = tn;
               }
             }
-            if (tn < hold_until[k]) continue;
+            // an emulated slow PE stops working on a replica whose task finished elsewhere
+            // (WA: the first result wins and the other replicas are cancelled)
+            if (tn < hold_until[k] && !sfin(inflight[k])) continue;
             const int u = inflight[k];
             const Unit &U = P.units[u];
             float ms = 0;

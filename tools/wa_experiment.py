@@ -28,6 +28,8 @@ def main():
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--slowdown", type=int, default=6)
     ap.add_argument("--out", default=None)
+    ap.add_argument("--unit-cells", type=int, default=0,
+                    help="target_unit_cells (0 = auto; 2**62 = the paper's very coarse tasks, one per pack)")
     args = ap.parse_args()
     w = seqgen.make_workload(args.config)
     D = Database(w.db, devices=[0] * args.workers)
@@ -45,7 +47,7 @@ def main():
                 for _ in range(args.reps):
                     r = D.search(w.queries, top_k=10, streams=2, policy=policy, workload_adjust=wa,
                                  straggler_mask=mask, straggler_slowdown=args.slowdown,
-                                 straggler_after_ms=after)
+                                 straggler_after_ms=after, target_unit_cells=args.unit_cells)
                     assert (r.scores == ref).all(), "scores differ across schedules"
                     st = r.stats
                     if best is None or st["seconds_device"] < best["seconds_device"]:
@@ -79,7 +81,7 @@ def main():
                                                makespan_on=on["makespan_s"], makespan_off=off["makespan_s"],
                                                tail_on=on["tail_s"], tail_off=off["tail_s"])
             print(f"WA gain {name}/{policy}: {summary[f'{name}/{policy}']['gcups_gain_pct']:+.1f} % GCUPS")
-    out = dict(config=args.config, workers=args.workers, slowdown=args.slowdown,
+    out = dict(config=args.config, workers=args.workers, slowdown=args.slowdown, unit_cells=args.unit_cells,
                note="P workers share one B200 (separate streams/replicas); the straggler holds each "
                     "completion back by (slowdown-1) x the unit's device time",
                summary=summary, runs=rows)
