@@ -188,6 +188,7 @@ struct Plan {
   int32_t first_short_group = 0;
   int32_t max_k3_seqs = 0;   // largest K3 unit (sequences)
   int32_t max_len = 0;
+  std::vector<uint8_t> pack_may_ovf;   // per pack: a query whose score bound reaches the s16 flag
 };
 
 static void validate_seqset(const sw_seqset *s, const char *what) {
@@ -202,7 +203,8 @@ static void validate_seqset(const sw_seqset *s, const char *what) {
     throw Error(SW_EINVAL, std::string(what) + ": residues is NULL");
 }
 
-static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, int n_workers) {
+static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, int n_workers,
+                      const int8_t *M, int32_t thresh) {
   Plan P;
   const int32_t nq = q->n;
   P.qoff.resize(nq + 1);
@@ -286,6 +288,31 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
   }
   P.prof_total = prof;
   P.max_len = db.max_len;
+  // packs that can saturate int16: a query's score is at most the sum over its residues of
+  // their best substitution score; units of such packs go first, so the int32 re-run of
+  // what they saturate overlaps the rest of the step instead of ending it (C5's planted
+  // W/C/Y-rich query)
+  {
+    int row_best[24];
+    for (int a = 0; a < 24; a++) {
+      row_best[a] = kPadScore;
+      for (int c = 0; c < 24; c++) row_best[a] = std::max(row_best[a], (int)M[a * 24 + c]);
+    }
+    std::vector<uint8_t> q_may(nq, 0);
+    for (int32_t k = 0; k < nq; k++) {
+      int64_t bound = 0;
+      for (int64_t p = P.qoff[k]; p < P.qoff[k + 1]; p++) bound += std::max(0, row_best[P.qcodes[p]]);
+      q_may[k] = bound + kOff >= (int64_t)thresh;
+    }
+    P.pack_may_ovf.assign(P.pairs.size(), 0);
+    for (size_t p = 0; p < P.pairs.size(); p++) {
+      const QueryPair &qp = P.pairs[p];
+      for (int32_t sidx = 0; sidx < qp.rows_padded / 16; sidx++) {
+        const SliceInfo &x = P.slices[qp.slice_off + sidx];
+        if ((x.q_lo >= 0 && q_may[x.q_lo]) || (x.q_hi >= 0 && q_may[x.q_hi])) { P.pack_may_ovf[p] = 1; break; }
+      }
+    }
+  }
   // long sequences -> K3: whole groups whose longest member exceeds the threshold
   int32_t thr = o.long_threshold == 0 ? 3072 : o.long_threshold;
   const int32_t ng = (int32_t)db.groups.size();
@@ -372,6 +399,7 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
     const int ra = a.kind == kUnitIntra ? (small3(a) ? 1 : 0) : 2;
     const int rb = b.kind == kUnitIntra ? (small3(b) ? 1 : 0) : 2;
     if (ra != rb) return ra < rb;
+    if (P.pack_may_ovf[a.pair] != P.pack_may_ovf[b.pair]) return P.pack_may_ovf[a.pair] > P.pack_may_ovf[b.pair];
     return a.work > b.work;
   });
   {
@@ -578,7 +606,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
     const PackedDB &H = db->host;
     const int32_t nq = queries->n, nd = H.n;
     const int nW = dist ? 1 : (int)db->devs.size();
-    Plan P = make_plan(queries, H, o, dist ? o.dist_world : nW);
+    Plan P = make_plan(queries, H, o, dist ? o.dist_world : nW, M, thresh);
     const double wall0 = now_s();
 
     std::vector<DevSearch *> S(nW);
