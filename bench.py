@@ -25,6 +25,7 @@ import time
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")   # before torch creates a context
 
 import numpy as np  # noqa: E402
 
@@ -34,6 +35,7 @@ PAPER_CONTEXT = ("paper: 7,190 s on 1 SSE core (Core i7 3.4 GHz) vs 112 s on 4x 
                  "for 40 queries vs SwissProt (PAPER.md P12); derived ~2.7 and ~174 GCUPS")
 DPX_RATE = 64.0   # measured lane-ops/clk/SM of VIMNMX3.S16x2 / VIADDMNMX.S16x2 (tools/dpx_peak)
 DPX_PER_CELL = 2.0  # K1/K3 inner loop: 4 three-input DPX per s16x2 lane word = 2 per cell
+DPX_FORMULATION = 2.25  # + the running maximum (0.5 VIMNMX3 per word): the kernel's own ALU ops/cell
 
 
 def env_rank():
@@ -273,7 +275,8 @@ def main():
     value = cells * args.steps / dev_s / 1e9
     ms = 1e3 * dev_s / args.steps
 
-    # ---- e2e: host buffers through the C-ABI (queries H2D, scores + hits D2H, pinned)
+    # ---- e2e: host buffers through the C-ABI (queries H2D, scores + hits D2H, pinned).
+    # N > 1: every rank reads back its own committed slice (disjoint), rank 0 the merged hits
     e2e = None
     nq, nd = w.queries.n, w.db.n
     h2d = int(w.queries.total + 8 * (nq + 1) + 576)
@@ -289,10 +292,10 @@ def main():
             t0 = time.perf_counter()
             if world > 1:
                 sc, hs, hi, _ = swdist.search(D, w.queries, rank, world, top_k=args.top_k, **kw)
+                pin_s.copy_(sc, non_blocking=True)
                 if rank == 0:
-                    pin_s.copy_(sc, non_blocking=True)
-                    pin_h[..., 0].copy_(hs)
-                    pin_h[..., 1].copy_(hi)
+                    pin_h[..., 0].copy_(hs, non_blocking=True)
+                    pin_h[..., 1].copy_(hi, non_blocking=True)
                 torch.cuda.synchronize()
             else:
                 D.search(w.queries, top_k=args.top_k, out_scores=pin_s, out_hits=pin_h, **kw)
@@ -305,54 +308,58 @@ def main():
             tsum = float(tt.item())
         e2e = {"value": cells * args.e2e_steps / tsum / 1e9, "unit": "GCUPS",
                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-               "note": "sw_search with host queries and pinned host outputs (scores + hits), host "
-                       "clock around the call; packed DB resident (created once, db_create_s)"}
+               "note": ("sw_search with host queries and pinned host outputs (scores + hits), host "
+                        "clock around the call; packed DB resident (created once, db_create_s)"
+                        + ("; per rank: its committed score slice + (rank 0) the merged hits, max over "
+                           "ranks" if world > 1 else ""))}
 
-    # ---- roofline of the DP kernels (integer/DPX pipe bound)
+    # ---- roofline of the dominant kernel (K1, integer/DPX pipe bound), rank 0 at every N:
+    # one local search with a single stream, so every inter-task (K1) launch runs by itself;
+    # achieved = K1 cells per launch / average K1 launch duration (CUDA events around each
+    # launch on its stream, inside libsw)
     last = stats[-1]
     sm_mhz = clocks["sm_mhz"] or 1965.0
     nsm = torch.cuda.get_device_properties(local).multi_processor_count
     peak = nsm * sm_mhz * 1e6 * DPX_RATE / DPX_PER_CELL / 1e9
     peak_max = nsm * 1965e6 * DPX_RATE / DPX_PER_CELL / 1e9
+    peak_form = nsm * sm_mhz * 1e6 * DPX_RATE / DPX_FORMULATION / 1e9
     per_gpu = value / world
-    # the dominant kernel alone: one search with a single stream, so every inter-task (K1)
-    # launch runs by itself; achieved = K1 cells per launch / average K1 launch duration
-    # (CUDA events around each launch on its stream, inside libsw)
-    flush_l2()
-    alone = D.search(w.queries, top_k=args.top_k, outputs_on_device=True, streams=1,
-                     **{k: v for k, v in kw.items() if k != "streams"}).stats if world == 1 else None
-    k1_launches = sum(1 for e in (alone or {}).get("unit_log", []) if e["kind"] == 0)
-    k1_alone = (alone["cells_k1"] / alone["kernel_seconds_k1"] / 1e9) if alone and alone["kernel_seconds_k1"] > 0 else None
-    k3_alone = (alone["cells_k3"] / alone["kernel_seconds_k3"] / 1e9) if alone and alone["kernel_seconds_k3"] > 0 else None
-    bytes_per_cell, ncu = load_traffic()
-    cells_per_launch = alone["cells_k1"] / k1_launches if k1_launches else None
-    traffic = (bytes_per_cell * cells_per_launch) if (bytes_per_cell and cells_per_launch) else None
-    # achieved: the DP kernels (K1 inter-task + K3 intra-task are the whole step; they run
-    # concurrently on 4 streams, so per-launch durations overlap) -> cells of the timed
-    # steps / device time of the timed steps, per GPU.  The isolated per-launch rate of K1
-    # (1 stream, each launch alone incl. its own wave tail) is reported beside it.
-    achieved = per_gpu
-    roofline = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "GCUPS",
-                "frac": achieved / peak, "traffic": traffic,
-                "kernel": "k1_kernel + k3_kernel (all DP launches of the timed steps, per GPU)",
-                "k1_alone_gcups": k1_alone, "k1_alone_frac": (k1_alone / peak) if k1_alone else None,
-                "k1_launches": k1_launches, "k1_cells_per_launch": cells_per_launch,
-                "k1_avg_launch_ms": (1e3 * alone["kernel_seconds_k1"] / k1_launches) if k1_launches else None,
-                "k3_alone_gcups": k3_alone,
-                "peak_at_max_clock": peak_max,
-                "derivation": f"{nsm} SMs x {sm_mhz:.0f} MHz (median under load) x {DPX_RATE:.0f} "
-                              f"DPX lane-ops/clk/SM (measured, tools/dpx_peak.cu) / "
-                              f"{DPX_PER_CELL:.0f} three-input DPX per cell (4 per s16x2 lane word)",
-                "traffic_note": "dram__bytes_read+write per K1 launch: bytes per cell of the ncu --set full "
-                                "capture (profiles/ncu_k1_summary.json) x the average cells per K1 launch",
-                "k1_cells_share": last["cells_k1"] / max(1, last["cells_k1"] + last["cells_k3"])}
-
-    cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        g, cores, desc, _, _ = oracle_rate(w, seconds_target=args.cpu_seconds)
-        g1, _, desc1, _, _ = oracle_rate(w, seconds_target=3.0, seed=7, max_threads=1)
-        cpu = {"value": g, "unit": "GCUPS", "cores": cores, "kind": "oracle", "sample": desc,
-               "single_core": {"value": g1, "sample": desc1}, "cpu_model": cpu_model()}
+    roofline = cpu = None
+    if rank == 0:
+        flush_l2()
+        alone = D.search(w.queries, top_k=args.top_k, outputs_on_device=True, streams=1,
+                         **{k: v for k, v in kw.items() if k != "streams"}).stats
+        k1_launches = sum(1 for e in alone.get("unit_log", []) if e["kind"] == 0)
+        k1_alone = (alone["cells_k1"] / alone["kernel_seconds_k1"] / 1e9) if alone["kernel_seconds_k1"] > 0 else None
+        k3_alone = (alone["cells_k3"] / alone["kernel_seconds_k3"] / 1e9) if alone["kernel_seconds_k3"] > 0 else None
+        bytes_per_cell, ncu = load_traffic()
+        cells_per_launch = alone["cells_k1"] / k1_launches if k1_launches else None
+        traffic = (bytes_per_cell * cells_per_launch) if (bytes_per_cell and cells_per_launch) else None
+        roofline = {"bound": "alu", "achieved": k1_alone, "peak": peak, "unit": "GCUPS",
+                    "frac": (k1_alone / peak) if k1_alone else None, "traffic": traffic,
+                    "kernel": "k1_kernel (inter-task DP, the dominant kernel): cells per launch / average "
+                              "launch duration, each launch alone on the GPU (1 stream)",
+                    "k1_launches": k1_launches, "k1_cells_per_launch": cells_per_launch,
+                    "k1_avg_launch_ms": (1e3 * alone["kernel_seconds_k1"] / k1_launches) if k1_launches else None,
+                    "k3_alone_gcups": k3_alone,
+                    "step_gcups_per_gpu": per_gpu, "step_frac": per_gpu / peak,
+                    "peak_at_max_clock": peak_max,
+                    "formulation_peak": peak_form,
+                    "k1_frac_of_formulation": (k1_alone / peak_form) if k1_alone else None,
+                    "step_frac_of_formulation": per_gpu / peak_form,
+                    "derivation": f"{nsm} SMs x {sm_mhz:.0f} MHz (median under load) x {DPX_RATE:.0f} "
+                                  f"DPX lane-ops/clk/SM (measured, tools/dpx_peak.cu) / "
+                                  f"{DPX_PER_CELL:.0f} three-input DPX per cell (4 per s16x2 lane word); "
+                                  f"formulation_peak uses the kernel's own {DPX_FORMULATION} ALU-pipe ops per "
+                                  f"cell (4 DPX + 0.5 VIMNMX3 for the running maximum per s16x2 word)",
+                    "traffic_note": "dram__bytes_read+write per K1 launch: bytes per cell of the ncu --set full "
+                                    "capture (profiles/ncu_k1_summary.json) x the average cells per K1 launch",
+                    "k1_cells_share": last["cells_k1"] / max(1, last["cells_k1"] + last["cells_k3"])}
+        if not args.no_cpu_baseline:
+            g, cores, desc, _, _ = oracle_rate(w, seconds_target=args.cpu_seconds)
+            g1, _, desc1, _, _ = oracle_rate(w, seconds_target=3.0, seed=7, max_threads=1)
+            cpu = {"value": g, "unit": "GCUPS", "cores": cores, "kind": "oracle", "sample": desc,
+                   "single_core": {"value": g1, "sample": desc1}, "cpu_model": cpu_model()}
 
     if rank == 0:
         line = {"metric": "GCUPS", "value": value, "unit": "GCUPS", "n_gpus": world,
@@ -370,6 +377,11 @@ def main():
                            "units_per_step": last["n_units"],
                            "overflow_pairs": last["n_overflow_pairs"],
                            "wa_grants": last["n_wa_grants"],
+                           "wa_cancelled": last["n_cancelled"],
+                           "request_messages": last["n_requests"],
+                           "data_plane": ({"hits_allgather_bytes_per_rank": last.get("gather_bytes", 0),
+                                           "scores": "rank-local committed slices (no collective)"}
+                                          if world > 1 else {"peer_bytes": last["peer_bytes"]}),
                            "db_create_s": db_create_s, "generate_s": gen_s,
                            "wall_s_timed": wall, "parallelism": f"dp{world} (PSS/WA units)"},
                 "gpu_launches": launches, "clocks": clocks, "e2e": e2e, "roofline": roofline,

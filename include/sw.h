@@ -51,6 +51,25 @@ enum {
   SW_EBUSY = -6     /* a search is already running on this sw_db */
 };
 
+/* Limits (checked; SW_EINVAL beyond them).  The s16x2 kernels keep a query row index in 16
+ * bits of their slice tables, and K5's per-thread lists hold at most 64 hits. */
+#define SW_MAX_QUERY_LEN 65535 /* residues per query */
+#define SW_MAX_TOP_K 64        /* hits per query */
+
+/* Slower-PE emulation for the workload-adjustment experiments (P24 §V.C
+ * "introduced local load"), applied to the workers in sw_opts.straggler_mask from
+ * straggler_after_ms on, with factor straggler_slowdown (s): */
+enum {
+  SW_STRAGGLER_HOLD = 0,   /* host-side: each completion is held back (s-1) x the unit's device
+                              time (the GPU itself runs at full speed) */
+  SW_STRAGGLER_SM_CAP = 1, /* GPU-side (default): the worker's DP kernels together get
+                              ceil(n_SM / s) SMs' worth of resident blocks (split over its
+                              streams; persistent grids), so its GPU really runs ~s x slower */
+  SW_STRAGGLER_NOISE = 2   /* GPU-side local load: a high-priority kernel occupies all but
+                              ceil(n_SM / s) SMs of the worker's GPU (one SM-filling block each)
+                              until the worker's last unit ends */
+};
+
 /* Task allocation policies (P18 §IV.A). */
 enum {
   SW_POLICY_SS = 0, /* Self-Scheduling: Allocate(N, p_i) = 1 (P18 §IV.A.1) */
@@ -87,9 +106,8 @@ typedef struct {
                                 (warp wavefront) kernel; 0 = auto (3072), <0 = never */
   int32_t outputs_on_device; /* 1: `scores` / `hits` are device pointers on the first
                                 device of the sw_db (inputs-resident timing mode) */
-  uint64_t straggler_mask;   /* experiments: worker w emulates a slower PE if bit w is set:
-                                each completion is held back by (slowdown-1) x the unit's
-                                device time (SURVEY §8(d) WA experiment, P24 §V.C) */
+  uint64_t straggler_mask;   /* experiments: worker w emulates a slower PE if bit w is set
+                                (how: straggler_mode; SURVEY §8(d) WA experiment, P24 §V.C) */
   int32_t straggler_slowdown;/* slowdown factor (default 6, Fig. 5's GPU:SSE ratio) */
   /* multi-process mode (one process per GPU, torchrun): world > 1 makes every rank a
      worker of one master, run as a thread of rank 0 and reached over TCP */
@@ -99,7 +117,8 @@ typedef struct {
   const char *dist_host;     /* master address, e.g. "127.0.0.1" */
   int32_t straggler_after_ms;/* the straggler slows down only after this many ms (local
                                 load introduced mid-run, P24 §V.C); 0 = from the start */
-  int32_t reserved[7];
+  int32_t straggler_mode;    /* SW_STRAGGLER_* (default SW_STRAGGLER_SM_CAP) */
+  int32_t reserved[6];
 } sw_opts;
 
 typedef struct {
@@ -113,16 +132,28 @@ typedef struct {
   int32_t n_units;          /* work units in the plan */
   int32_t n_overflow_pairs; /* pairs re-scored by the int32 kernel after saturation */
   int32_t n_wa_grants;      /* duplicates granted by workload adjustment */
-  int32_t n_requests;       /* master interactions (task requests) */
+  int32_t n_requests;       /* task-request messages to the master (an idle worker's request
+                               waits at the master: one message, not a poll loop) */
   int32_t kernel_launches;  /* CUDA kernels launched by this process for the search */
   int32_t n_devices;        /* devices (in-process) or 1 (per rank) */
   double kernel_seconds_k1; /* summed device time of the inter-task kernel launches */
   double kernel_seconds_k3; /* summed device time of the intra-task kernel launches */
   int64_t cells_k1;         /* real cells computed by inter-task launches (incl. duplicates) */
   int64_t cells_k3;         /* real cells computed by intra-task launches (incl. duplicates) */
-  double tail_seconds;      /* makespan minus the median per-worker finish time */
-  const char *unit_log_json;/* per-unit log (worker, replica, t_grant, t_start, t_end, cells,
-                               committed); owned by the sw_db, valid until its next search */
+  double tail_seconds;      /* tail: the last worker's last unit completion minus the (lower)
+                               median over workers of their last unit completion (device clocks,
+                               each worker's own start event after a common host barrier) */
+  const char *unit_log_json;/* per-replica log: unit, kind, pack, worker, stream, host times
+                               (t_grant, t_start, t_end), device times (dev_t0, dev_t1 ms since
+                               the worker's start; device_ms), cells, cells_done, committed,
+                               cancelled, slowed; owned by the sw_db, valid until its next search */
+  int32_t n_grant_messages; /* request messages that granted at least one task */
+  int32_t n_cancelled;      /* WA replicas stopped early by their abort flag */
+  double seconds_last_unit; /* device time of this process's last unit completion (for the
+                               cross-rank tail in multi-process mode) */
+  int64_t peer_bytes;       /* bytes copied between GPUs by the in-process merge */
+  const char *sched_log_json;/* the master's event log with Φ and v̄ per grant (sw_sched.h);
+                               in-process, or rank 0 in multi-process mode; owned by the sw_db */
 } sw_stats;
 
 typedef struct sw_db sw_db; /* opaque: host index + packed replica on each device */
@@ -143,16 +174,23 @@ int32_t sw_db_size(const sw_db *db);
 int32_t sw_db_devices(const sw_db *db);
 
 /* Compare every query with every database sequence.
+ *   queries     at most SW_MAX_QUERY_LEN residues each
  *   matrix      24x24 int8, row-major, query residue = row; NULL = BLOSUM62
  *   gap_open, gap_extend  >= 0, gap_open + 2*gap_extend <= 2^20
- *   top_k       >= 0 hits per query under (score desc, db_index asc)
+ *   top_k       0 .. SW_MAX_TOP_K hits per query under (score desc, db_index asc)
  *   scores      [nq][ndb] int32 in the ORIGINAL orders, or NULL
  *   hits        [nq][top_k] sw_hit, or NULL
  *   (host pointers, or device pointers on the sw_db's first device when
  *    opts->outputs_on_device)
+ * Data plane (P16 §IV "the slaves send their results to the master, that merges them"):
+ * every committed work unit's top-k is computed on its GPU right after it (K5u); each GPU
+ * merges the lists of the units it committed (K5m).  In-process with several GPUs, the
+ * other GPUs' committed scores (dense, only their units) and top-k lists are copied to the
+ * first GPU over NVLink and merged there -- no full-matrix transfer or reduction.
  * In multi-process mode every rank passes the same inputs; each rank's `scores` then
- * holds the pairs of the units it committed (others = -1) and `hits` the top-k over
- * those; the binding merges them across ranks (NCCL).
+ * holds exactly the pairs of the units it committed (others = -1: the ranks' slices are
+ * disjoint) and `hits` the top-k over those; the binding all-gathers the hits (NCCL,
+ * nq*top_k*8 bytes per rank) and merges them with sw_merge_hits.
  * Results are bit-identical for every GPU count, policy and WA setting. */
 int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t gap_open,
               int32_t gap_extend, int32_t top_k, int32_t *scores, sw_hit *hits,
@@ -163,6 +201,15 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
  * cross-rank reduction.  */
 int sw_topk_device(sw_db *db, const int32_t *scores_dev, int32_t nq, int32_t ndb, int32_t top_k,
                    sw_hit *hits_dev);
+
+/* Merge per-source top-k lists into the global top-k (the master's merge, P16 §IV).
+ *   lists_dev  [n_sources][nq][k_in] sw_hit on the sw_db's first device ({x, -1} = empty)
+ *   hits_dev   [nq][top_k] sw_hit, device memory
+ * Order (score desc, db_index asc); a db_index appearing in several sources with the same
+ * score is kept once (sources are expected to be disjoint, e.g. ranks' committed units).
+ * top_k <= SW_MAX_TOP_K.  Synchronous. */
+int sw_merge_hits(sw_db *db, const sw_hit *lists_dev, int32_t n_sources, int32_t nq, int32_t k_in,
+                  int32_t top_k, sw_hit *hits_dev);
 
 /* ---- Phase 2: the alignments of selected pairs (NEXT-3) ---------------------------------
  * P12 §II.A.2: "In order to obtain the optimal local alignment, the algorithm starts from

@@ -15,11 +15,18 @@ import numpy as np
 
 from . import _build
 
+# several workers' streams on one GPU exceed CUDA's default 8 hardware work queues and would
+# falsely serialize; must be set before the process creates its CUDA context
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
+
 _lib = None
 
 SW_OK, SW_EINVAL, SW_ERESIDUE, SW_ENOMEM, SW_ECUDA, SW_ENET, SW_EBUSY = 0, -1, -2, -3, -4, -5, -6
 SW_POLICY_SS, SW_POLICY_PSS = 0, 1
 SW_TASK_READY, SW_TASK_EXECUTING, SW_TASK_FINISHED = 0, 1, 2
+SW_STRAGGLER_HOLD, SW_STRAGGLER_SM_CAP, SW_STRAGGLER_NOISE = 0, 1, 2
+_STRAGGLER_MODES = {"hold": SW_STRAGGLER_HOLD, "sm_cap": SW_STRAGGLER_SM_CAP, "noise": SW_STRAGGLER_NOISE}
+SW_MAX_TOP_K, SW_MAX_QUERY_LEN = 64, 65535
 
 
 class SwError(RuntimeError):
@@ -41,7 +48,7 @@ class sw_opts(ctypes.Structure):
                 ("straggler_slowdown", ctypes.c_int32), ("dist_rank", ctypes.c_int32),
                 ("dist_world", ctypes.c_int32), ("dist_port", ctypes.c_int32),
                 ("dist_host", ctypes.c_char_p), ("straggler_after_ms", ctypes.c_int32),
-                ("reserved", ctypes.c_int32 * 7)]
+                ("straggler_mode", ctypes.c_int32), ("reserved", ctypes.c_int32 * 6)]
 
 
 class sw_alignment(ctypes.Structure):
@@ -59,18 +66,22 @@ class sw_stats(ctypes.Structure):
                 ("n_devices", ctypes.c_int32), ("kernel_seconds_k1", ctypes.c_double),
                 ("kernel_seconds_k3", ctypes.c_double), ("cells_k1", ctypes.c_int64),
                 ("cells_k3", ctypes.c_int64), ("tail_seconds", ctypes.c_double),
-                ("unit_log_json", ctypes.c_char_p)]
+                ("unit_log_json", ctypes.c_char_p), ("n_grant_messages", ctypes.c_int32),
+                ("n_cancelled", ctypes.c_int32), ("seconds_last_unit", ctypes.c_double),
+                ("peer_bytes", ctypes.c_int64), ("sched_log_json", ctypes.c_char_p)]
 
 
 # every symbol include/*.h declares (tests check the library exports all of them)
 EXPORTS = ["sw_opts_default", "sw_db_create", "sw_db_destroy", "sw_db_residues", "sw_db_size",
-           "sw_db_devices", "sw_search", "sw_topk_device", "sw_last_error", "sw_version",
+           "sw_db_devices", "sw_search", "sw_topk_device", "sw_merge_hits", "sw_last_error", "sw_version",
            "sw_sched_create", "sw_sched_destroy", "sw_sched_report", "sw_sched_request",
-           "sw_sched_complete", "sw_sched_abandon", "sw_sched_start", "sw_sched_is_finished", "sw_sched_state",
+           "sw_sched_request_wait", "sw_sched_complete", "sw_sched_abandon", "sw_sched_fail_worker",
+           "sw_sched_start", "sw_sched_is_finished", "sw_sched_state",
            "sw_sched_committed_by", "sw_sched_replicas", "sw_sched_phi", "sw_sched_rate",
            "sw_sched_counter", "sw_sched_log_json", "sw_master_start", "sw_master_stop",
-           "sw_slave_connect", "sw_slave_request", "sw_slave_report", "sw_slave_complete",
-           "sw_slave_abandon", "sw_slave_start", "sw_slave_is_finished", "sw_slave_done", "sw_align"]
+           "sw_slave_connect", "sw_slave_request", "sw_slave_request_wait", "sw_slave_report",
+           "sw_slave_complete", "sw_slave_abandon", "sw_slave_start", "sw_slave_is_finished",
+           "sw_slave_done", "sw_slave_counter", "sw_align"]
 
 
 def lib():
@@ -106,6 +117,9 @@ def lib():
     L.sw_topk_device.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32,
                                  ctypes.c_int32, ctypes.c_void_p]
     L.sw_topk_device.restype = ctypes.c_int
+    L.sw_merge_hits.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32,
+                                ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p]
+    L.sw_merge_hits.restype = ctypes.c_int
     L.sw_last_error.restype = ctypes.c_char_p
     L.sw_version.restype = ctypes.c_char_p
     L.sw_sched_create.argtypes = [ctypes.c_int32, ctypes.c_int32, P(ctypes.c_int64), ctypes.c_int32,
@@ -117,6 +131,10 @@ def lib():
     L.sw_sched_request.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_double,
                                    P(ctypes.c_int32), ctypes.c_int32]
     L.sw_sched_request.restype = ctypes.c_int32
+    L.sw_sched_request_wait.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_double,
+                                        P(ctypes.c_int32), ctypes.c_int32, ctypes.c_double]
+    L.sw_sched_request_wait.restype = ctypes.c_int32
+    L.sw_sched_fail_worker.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_double]
     L.sw_sched_complete.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_double]
     L.sw_sched_complete.restype = ctypes.c_int32
     L.sw_sched_abandon.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_double]
@@ -135,13 +153,18 @@ def lib():
     L.sw_sched_log_json.argtypes = [ctypes.c_void_p]
     L.sw_sched_log_json.restype = ctypes.c_char_p
     L.sw_master_start.argtypes = [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, P(ctypes.c_int64),
-                                  ctypes.c_int32, ctypes.c_int32, ctypes.c_int32]
+                                  ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, ctypes.c_uint64]
     L.sw_master_start.restype = ctypes.c_void_p
     L.sw_master_stop.argtypes = [ctypes.c_void_p]
-    L.sw_slave_connect.argtypes = [ctypes.c_char_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_double]
+    L.sw_slave_connect.argtypes = [ctypes.c_char_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_double,
+                                   ctypes.c_uint64]
     L.sw_slave_connect.restype = ctypes.c_void_p
     L.sw_slave_request.argtypes = [ctypes.c_void_p, P(ctypes.c_int32), ctypes.c_int32]
     L.sw_slave_request.restype = ctypes.c_int32
+    L.sw_slave_request_wait.argtypes = [ctypes.c_void_p, P(ctypes.c_int32), ctypes.c_int32, ctypes.c_double]
+    L.sw_slave_request_wait.restype = ctypes.c_int32
+    L.sw_slave_counter.argtypes = [ctypes.c_void_p, ctypes.c_int32]
+    L.sw_slave_counter.restype = ctypes.c_int64
     L.sw_slave_report.argtypes = [ctypes.c_void_p, ctypes.c_double, ctypes.c_double]
     L.sw_slave_complete.argtypes = [ctypes.c_void_p, ctypes.c_int32]
     L.sw_slave_complete.restype = ctypes.c_int32
@@ -180,32 +203,56 @@ class SearchResult:
     stats: dict
 
 
-def chrome_trace(unit_log, name="sw_search") -> dict:
+def grant_timeline(sched_log):
+    """The master's grants (sched_log of a search) with times relative to the first event:
+    [{"t_rel", "worker", "unit", "phi", "rate", "wa"}] -- the per-interaction marks of the
+    paper's Figs. 7/8 (package weight Φ and mean rate v̄ of the requesting PE)."""
+    if not sched_log:
+        return []
+    t0 = min(e["t"] for e in sched_log)
+    return [dict(t_rel=e["t"] - t0, worker=e["worker"], unit=e["unit"], phi=e.get("phi", 0),
+                 rate=e.get("rate", 0.0), wa=e["ev"] == "W", ev=e["ev"])
+            for e in sched_log if e["ev"] in ("G", "W")]
+
+
+def chrome_trace(unit_log, name="sw_search", sched_log=None) -> dict:
     """The per-unit event log of a search (stats["unit_log"]) as a Chrome-trace / Perfetto
     JSON object (SURVEY §5 tracing): one process per worker (GPU), one thread per stream, a
     complete event per unit replica (host clock from launch to observed completion; args:
     cells, device_ms, committed, pack) and an instant event at each grant on a "master"
     thread -- the analogue of the paper's per-interaction marks (P24 Figs. 7/8)."""
     ev = []
+    sched_log = grant_timeline(sched_log) if sched_log and "t_rel" not in sched_log[0] else sched_log
     workers = sorted({e["worker"] for e in unit_log})
     for w in workers:
         ev.append({"ph": "M", "name": "process_name", "pid": w, "args": {"name": f"{name}: worker {w}"}})
         ev.append({"ph": "M", "name": "thread_name", "pid": w, "tid": -1, "args": {"name": "master grants"}})
     for e in unit_log:
         kind = "K1 inter-task" if e["kind"] == 0 else "K3 intra-task"
-        ev.append({"ph": "X", "name": f"unit {e['unit']} ({kind})", "cat": "unit",
+        tag = " cancelled" if e.get("cancelled") else (" lost" if not e["committed"] else "")
+        ev.append({"ph": "X", "name": f"unit {e['unit']} ({kind}){tag}", "cat": "unit",
                    "pid": e["worker"], "tid": e.get("stream", 0),
                    "ts": 1e6 * e["t_start"], "dur": max(0.0, 1e6 * (e["t_end"] - e["t_start"])),
-                   "args": {"cells": e["cells"], "pack": e["pair"], "committed": e["committed"],
-                            "device_ms": e.get("device_ms")}})
+                   "args": {"cells": e["cells"], "cells_done": e.get("cells_done", e["cells"]),
+                            "pack": e["pair"], "committed": e["committed"],
+                            "cancelled": e.get("cancelled", 0), "slowed": e.get("slowed", 0),
+                            "device_ms": e.get("device_ms"), "dev_t0_ms": e.get("dev_t0"),
+                            "dev_t1_ms": e.get("dev_t1")}})
         ev.append({"ph": "i", "name": f"grant unit {e['unit']}", "cat": "grant", "s": "t",
                    "pid": e["worker"], "tid": -1, "ts": 1e6 * e["t_grant"]})
+    for g in sched_log or []:
+        if g.get("ev") in ("G", "W"):   # Φ and v̄ of the requesting worker at each grant
+            ev.append({"ph": "C", "name": "PSS package weight phi", "pid": g["worker"],
+                       "ts": 1e6 * g["t_rel"], "args": {"phi": g.get("phi", 0)}})
+            ev.append({"ph": "C", "name": "rate v (GCUPS)", "pid": g["worker"],
+                       "ts": 1e6 * g["t_rel"], "args": {"v": 1e-9 * g.get("rate", 0.0)}})
     return {"traceEvents": ev, "displayTimeUnit": "ms"}
 
 
 def _stats_dict(st: sw_stats) -> dict:
-    d = {k: getattr(st, k) for k, _ in sw_stats._fields_ if k != "unit_log_json"}
+    d = {k: getattr(st, k) for k, _ in sw_stats._fields_ if k not in ("unit_log_json", "sched_log_json")}
     d["unit_log"] = json.loads(st.unit_log_json.decode()) if st.unit_log_json else []
+    d["sched_log"] = json.loads(st.sched_log_json.decode()) if st.sched_log_json else []
     return d
 
 
@@ -244,9 +291,12 @@ class Database:
     def search(self, queries, matrix=None, gap_open=10, gap_extend=2, top_k=10, want_scores=True,
                policy="pss", workload_adjust=True, omega=4, streams=4, target_unit_cells=0,
                long_threshold=0, outputs_on_device=False, straggler_mask=0, straggler_slowdown=6,
-               straggler_after_ms=0, dist=None, out_scores=None, out_hits=None) -> SearchResult:
+               straggler_after_ms=0, straggler_mode="sm_cap", dist=None, out_scores=None,
+               out_hits=None) -> SearchResult:
         """sw_search.  Host outputs are numpy arrays (pinned buffers may be passed via
-        out_scores / out_hits); with outputs_on_device the outputs are torch CUDA tensors."""
+        out_scores / out_hits); with outputs_on_device the outputs are torch CUDA tensors.
+        straggler_mode: "sm_cap" (GPU-side, default), "noise" (GPU-side local load) or
+        "hold" (host-side) -- see SW_STRAGGLER_* in include/sw.h."""
         keep = []
         qs = _seqset(queries, keep)
         nq, nd = int(queries.n), int(self.n)
@@ -262,6 +312,7 @@ class Database:
         o.straggler_mask = straggler_mask
         o.straggler_slowdown = straggler_slowdown
         o.straggler_after_ms = straggler_after_ms
+        o.straggler_mode = _STRAGGLER_MODES[straggler_mode]
         if dist is not None:
             o.dist_rank, o.dist_world, o.dist_port = dist["rank"], dist["world"], dist["port"]
             host = dist.get("host", "127.0.0.1").encode()
@@ -322,6 +373,16 @@ class Database:
                             d_end=a.d_end, ops=raw[a.ops_offset:a.ops_offset + a.n_ops].decode()))
         return res
 
+    def merge_hits(self, lists_dev, top_k):
+        """sw_merge_hits: lists_dev is a torch CUDA int32 tensor [n_sources, nq, k_in, 2]
+        (score, db_index); returns the merged (scores, index) [nq, top_k] on the device."""
+        import torch
+        n_src, nq, k_in, _ = lists_dev.shape
+        lists_dev = lists_dev.contiguous()
+        out = torch.empty((nq, top_k, 2), dtype=torch.int32, device=lists_dev.device)
+        _check(lib().sw_merge_hits(self._h, lists_dev.data_ptr(), n_src, nq, k_in, top_k, out.data_ptr()))
+        return out[..., 0], out[..., 1]
+
     def topk_device(self, scores_dev, top_k):
         """Top-k of a torch CUDA score matrix (entries < 0 ignored) -> (scores, index)."""
         import torch
@@ -368,6 +429,16 @@ class Scheduler:
             return None  # every task finished
         return [buf[i] for i in range(n)]
 
+    def request_wait(self, worker, now, timeout, cap=64):
+        buf = (ctypes.c_int32 * cap)()
+        n = lib().sw_sched_request_wait(self._h, worker, now, buf, cap, timeout)
+        if n < 0:
+            return None
+        return [buf[i] for i in range(n)]
+
+    def fail_worker(self, worker, now):
+        lib().sw_sched_fail_worker(self._h, worker, now)
+
     def complete(self, worker, unit, now) -> bool:
         return bool(lib().sw_sched_complete(self._h, worker, unit, now))
 
@@ -406,11 +477,12 @@ class Scheduler:
 class Master:
     """The multi-process master (sw_master_start): serves `world` slaves over TCP."""
 
-    def __init__(self, port, world, unit_cells, policy="pss", wa=True, omega=4):
+    def __init__(self, port, world, unit_cells, policy="pss", wa=True, omega=4, plan_hash=0):
         cells = np.ascontiguousarray(unit_cells, dtype=np.int64)
         h = lib().sw_master_start(port, world, len(cells),
                                   cells.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)),
-                                  SW_POLICY_SS if policy == "ss" else SW_POLICY_PSS, int(wa), omega)
+                                  SW_POLICY_SS if policy == "ss" else SW_POLICY_PSS, int(wa), omega,
+                                  plan_hash)
         if not h:
             raise SwError(SW_ENET, lib().sw_last_error().decode())
         self._h = h
@@ -424,8 +496,8 @@ class Master:
 class Slave:
     """A slave's connection to the master (sw_slave_*)."""
 
-    def __init__(self, host, port, rank, timeout=30.0):
-        h = lib().sw_slave_connect(host.encode(), port, rank, timeout)
+    def __init__(self, host, port, rank, timeout=30.0, plan_hash=0):
+        h = lib().sw_slave_connect(host.encode(), port, rank, timeout, plan_hash)
         if not h:
             raise SwError(SW_ENET, lib().sw_last_error().decode())
         self._h = h
@@ -436,6 +508,17 @@ class Slave:
         if n == -2:
             raise SwError(SW_ENET, lib().sw_last_error().decode())
         return None if n < 0 else [buf[i] for i in range(n)]
+
+    def request_wait(self, timeout=0.05, cap=64):
+        """One request that waits at the master (long poll) while nothing can be granted."""
+        buf = (ctypes.c_int32 * cap)()
+        n = lib().sw_slave_request_wait(self._h, buf, cap, timeout)
+        if n == -2:
+            raise SwError(SW_ENET, lib().sw_last_error().decode())
+        return None if n < 0 else [buf[i] for i in range(n)]
+
+    def counter(self, which):
+        return lib().sw_slave_counter(self._h, which)
 
     def report(self, cells, seconds):
         lib().sw_slave_report(self._h, float(cells), float(seconds))

@@ -11,6 +11,7 @@
 #include <climits>
 #include <cmath>
 #include <condition_variable>
+#include <cstdlib>
 #include <cstring>
 #include <deque>
 #include <memory>
@@ -55,6 +56,14 @@ static int guarded(F &&f) {
     g_err = e.what();
     return SW_EINVAL;
   }
+}
+
+// Each worker keeps up to 64 streams in flight, plus its cancellation and local-load
+// streams; with several workers on one GPU these exceed the default 8 hardware work queues
+// and unrelated streams would serialize (a fast worker's unit waiting behind a straggler's
+// kernel).  Raise the limit before the first CUDA context is created (no effect after).
+__attribute__((constructor)) static void sw_raise_connections() {
+  setenv("CUDA_DEVICE_MAX_CONNECTIONS", "32", 0);
 }
 
 static double now_s() {
@@ -115,22 +124,39 @@ struct DevSearch {
   DBuf<uint2> k3_border;   // [streams][max_k3_seqs][max_len]
   DBuf<int32_t> k2_border;
   DBuf<int32_t> abort_dev;      // per-unit WA cancellation flags (device memory)
+  DBuf<int32_t> progress;       // per-unit progress counters (K1 groups / K3 sequence-chunks)
   int32_t *abort_d = nullptr;
   int32_t *one_h = nullptr;      // pinned constant 1, source of the cancellation copies
   int32_t *ovf_seen_h = nullptr; // pinned [kMaxStreams]: ovf_count copied after each unit
+  int32_t *prog_h = nullptr;     // pinned [kMaxStreams]: the unit's progress after it ran
   cudaStream_t cancel_st = nullptr;
+  cudaStream_t noise_st = nullptr;   // high priority: the local-load kernel (straggler mode 2)
+  DBuf<int32_t> noise_flag;
+  DBuf<uint32_t> noise_sink;
   std::vector<char> cancelled;
-  cudaEvent_t ev_start = nullptr, ev_end = nullptr;
+  // data plane: per-unit top-k of committed units, merged per worker
+  DBuf<int32_t> pack_q;          // queries of each pack (flattened, Plan::pack_q_off)
+  DBuf<int2> unit_hits;          // [units][max_pack_q][k]
+  DBuf<int2> worker_hits;        // [nq][k] top-k over this worker's committed units
+  DBuf<int2> all_hits;           // device 0: [workers][nq][k]
+  DBuf<int32_t> list_tab;        // merge tables: list_off[nq+1] then list_idx
+  DBuf<SegInfo> segs;            // committed-unit segments (scores data plane)
+  DBuf<int32_t> compact;         // this worker's committed scores, dense
+  DBuf<int32_t> out_stage;       // multi-process: committed-only score matrix
+  std::vector<int32_t> committed;   // units this worker committed
+  cudaEvent_t ev_start = nullptr, ev_end = nullptr, ev_data = nullptr;
   std::vector<cudaEvent_t> u_start, u_end;  // per stream
   int launches = 0;
   double k1_sec = 0, k3_sec = 0;
   int64_t k1_cells = 0, k3_cells = 0;
   int64_t dup_cells = 0;
+  int32_t n_cancelled = 0;
   double finish_wall = 0;
+  double last_dev = 0;           // device time of this worker's last unit completion (s)
   int32_t n_ovf = 0;
   void reset_counters() {
-    launches = 0; k1_sec = k3_sec = 0; k1_cells = k3_cells = 0; dup_cells = 0;
-    finish_wall = 0; n_ovf = 0; scores = nullptr;
+    launches = 0; k1_sec = k3_sec = 0; k1_cells = k3_cells = 0; dup_cells = 0; n_cancelled = 0;
+    finish_wall = 0; last_dev = 0; n_ovf = 0; scores = nullptr; committed.clear();
   }
   ~DevSearch();
 };
@@ -155,9 +181,12 @@ struct Device {
 inline DevSearch::~DevSearch() {
   if (one_h) cudaFreeHost(one_h);
   if (ovf_seen_h) cudaFreeHost(ovf_seen_h);
+  if (prog_h) cudaFreeHost(prog_h);
   if (cancel_st) cudaStreamDestroy(cancel_st);
+  if (noise_st) cudaStreamDestroy(noise_st);
   if (ev_start) cudaEventDestroy(ev_start);
   if (ev_end) cudaEventDestroy(ev_end);
+  if (ev_data) cudaEventDestroy(ev_data);
   for (auto e : u_start) cudaEventDestroy(e);
   for (auto e : u_end) cudaEventDestroy(e);
 }
@@ -170,6 +199,7 @@ struct sw_db {
   std::vector<std::unique_ptr<sw::Device>> devs;
   std::atomic<int> busy{0};
   std::string unit_log;
+  std::string sched_log;
 };
 
 namespace sw {
@@ -189,7 +219,16 @@ struct Plan {
   int32_t max_k3_seqs = 0;   // largest K3 unit (sequences)
   int32_t max_len = 0;
   std::vector<uint8_t> pack_may_ovf;   // per pack: a query whose score bound reaches the s16 flag
+  std::vector<int32_t> pack_q;         // queries of each pack, flattened (ascending ids)
+  std::vector<int32_t> pack_q_off;     // [packs + 1]
+  int32_t max_pack_q = 1;              // most queries in one pack
+  uint64_t hash = 0;                   // FNV-1a of the unit table (multi-process handshake)
 };
+// sorted-sequence range [s0, s1) of a unit's pairs (K1: whole groups; K3: long sequences)
+static inline void unit_seq_range(const Unit &U, int32_t n, int32_t &s0, int32_t &s1) {
+  if (U.kind == kUnitInter) { s0 = U.b0 * kGroup; s1 = std::min(n, U.b1 * kGroup); }
+  else { s0 = U.b0; s1 = U.b1; }
+}
 
 static void validate_seqset(const sw_seqset *s, const char *what) {
   if (!s) throw Error(SW_EINVAL, std::string(what) + " is NULL");
@@ -211,7 +250,8 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
   P.qoff[0] = 0;
   for (int32_t k = 0; k < nq; k++) {
     const int64_t l = q->offsets[k + 1] - q->offsets[k];
-    if (l > 65535) throw Error(SW_EINVAL, "query " + std::to_string(k) + " longer than 65535");
+    if (l > SW_MAX_QUERY_LEN)
+      throw Error(SW_EINVAL, "query " + std::to_string(k) + " longer than 65535 residues (SW_MAX_QUERY_LEN)");
     P.qoff[k + 1] = P.qoff[k] + l;
   }
   P.qcodes.resize(P.qoff[nq]);
@@ -415,6 +455,31 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
     }
     P.units.swap(order);
   }
+  // the queries of each pack (a query lives in one half-run of one pack)
+  P.pack_q_off.assign(P.pairs.size() + 1, 0);
+  for (size_t p = 0; p < P.pairs.size(); p++) {
+    std::vector<int32_t> qs;
+    const QueryPair &qp = P.pairs[p];
+    for (int32_t sidx = 0; sidx < qp.rows_padded / 16; sidx++) {
+      const SliceInfo &x = P.slices[qp.slice_off + sidx];
+      if (x.q_lo >= 0) qs.push_back(x.q_lo);
+      if (x.q_hi >= 0) qs.push_back(x.q_hi);
+    }
+    std::sort(qs.begin(), qs.end());
+    qs.erase(std::unique(qs.begin(), qs.end()), qs.end());
+    P.pack_q.insert(P.pack_q.end(), qs.begin(), qs.end());
+    P.pack_q_off[p + 1] = (int32_t)P.pack_q.size();
+    P.max_pack_q = std::max<int32_t>(P.max_pack_q, (int32_t)qs.size());
+  }
+  // unit-table hash: ranks of one multi-process search must agree on it (net.cpp handshake)
+  uint64_t h = 1469598103934665603ull;
+  auto mix = [&](int64_t v) {
+    for (int b = 0; b < 8; b++) { h ^= (uint64_t)((v >> (8 * b)) & 0xff); h *= 1099511628211ull; }
+  };
+  mix(nq); mix(db.n); mix(db.residues); mix((int64_t)P.units.size());
+  for (const Unit &u : P.units) { mix(u.kind); mix(u.pair); mix(u.b0); mix(u.b1); mix(u.cells); }
+  for (int32_t q : P.pack_q) mix(q);
+  P.hash = h;
   return P;
 }
 
@@ -422,9 +487,13 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
 struct UnitLog {
   int32_t unit, worker, stream;
   double t_grant, t_start, t_end;   // host clock (s since the search start)
-  int64_t cells;
-  int committed;
+  int64_t cells;                    // the unit's cells
+  int64_t cells_done;               // cells this replica computed (< cells when cancelled)
+  int committed;                    // 1 = this replica committed the unit
+  int cancelled;                    // 1 = cut short by WA cancellation (the unit finished elsewhere)
+  int slowed;                       // 1 = ran under the straggler emulation
   float device_ms;                  // CUDA events around the unit's kernels on its stream
+  float dev_t0, dev_t1;             // device ms of its start / end since the worker's start event
 };
 
 static const int kOvfCap = 1 << 20;
@@ -447,8 +516,10 @@ static K2Args k2_args(const Plan &P, const PackedDB &db, DevSearch &S, int strea
   return a;
 }
 
+// sm_cap > 0: the unit's kernels get at most sm_cap SMs' worth of blocks (a slower PE,
+// straggler mode 1)
 static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const Unit &U, int uidx,
-                        int stream_idx, int32_t alpha, int32_t beta, int32_t thresh) {
+                        int stream_idx, int32_t alpha, int32_t beta, int32_t thresh, int sm_cap) {
   Device &D = *S.D;
   cudaStream_t st = D.streams[stream_idx];
   const uint32_t na = ((uint32_t)(-alpha) & 0xffffu) * 0x10001u;
@@ -465,8 +536,10 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     a.border = D.k1_border.p; a.border_slot_cols = D.slot_cols; a.slots_per_sm = D.slots_per_sm;
     a.slot_busy = D.slot_busy.p;
     a.abort_flag = S.abort_d + uidx;
+    a.progress = S.progress.p + uidx;
     a.na = na; a.nb = nbm;
-    launch_k1(a, U.b1 - U.b0, db.groups[U.b1 - 1].ncols, P.pairs[U.pair].rows_padded, st, D.n_sm);
+    launch_k1(a, U.b1 - U.b0, db.groups[U.b1 - 1].ncols, P.pairs[U.pair].rows_padded, st,
+              sm_cap > 0 ? std::min(sm_cap, D.n_sm) : D.n_sm);
   } else {
     K3Args a;
     a.packed = D.packed.p; a.groups = D.groups.p; a.perm = D.perm.p; a.sorted_len = D.sorted_len.p;
@@ -477,11 +550,12 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     a.ovf = S.ovf.p + (size_t)stream_idx * S.ovf_cap; a.ovf_count = S.ovf_count.p + stream_idx;
     a.ovf_cap = S.ovf_cap; a.ovf_bits = S.ovf_bits.p;
     const int64_t stride = (std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16;  // >= tiles * T
-    a.border = S.k3_border.p + (size_t)stream_idx * P.max_k3_seqs * k3_phases() * stride;
+    a.border = S.k3_border.p + (size_t)stream_idx * P.max_k3_seqs * stride;
     a.border_stride = stride;
     a.abort_flag = S.abort_d + uidx;
+    a.progress = S.progress.p + uidx;
     a.na = na; a.nb = nbm;
-    launch_k3(a, P.pairs[U.pair].rows_padded, st);
+    launch_k3(a, P.pairs[U.pair].rows_padded, st, sm_cap);
   }
   S.launches++;
   // saturated pairs listed so far on this stream -> host (4 bytes): the worker launches
@@ -490,6 +564,15 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
   // unit would wait for a K1 block to leave and stall the stream.
   CK(cudaMemcpyAsync(S.ovf_seen_h + stream_idx, S.ovf_count.p + stream_idx, sizeof(int32_t),
                      cudaMemcpyDeviceToHost, st));
+  // and the unit's progress counter (the cells a cancelled replica really computed)
+  CK(cudaMemcpyAsync(S.prog_h + stream_idx, S.progress.p + uidx, sizeof(int32_t),
+                     cudaMemcpyDeviceToHost, st));
+}
+// progress units of a whole unit: K1 groups, K3 (sequence, chunk) pairs
+static int64_t unit_progress_total(const Plan &P, const Unit &U) {
+  if (U.kind == kUnitInter) return U.b1 - U.b0;
+  const int64_t nch = (P.pairs[U.pair].rows + kK3Chunk - 1) / kK3Chunk;
+  return (int64_t)(U.b1 - U.b0) * nch;
 }
 
 }  // namespace sw
@@ -511,6 +594,7 @@ void sw_opts_default(sw_opts *o) {
   o->target_unit_cells = 0;
   o->long_threshold = 0;
   o->straggler_slowdown = 6;
+  o->straggler_mode = SW_STRAGGLER_SM_CAP;
 }
 
 int sw_db_create(const sw_seqset *dbs, const int *devices, int n_devices, sw_db **out) {
@@ -546,6 +630,18 @@ int sw_db_create(const sw_seqset *dbs, const int *devices, int n_devices, sw_db 
       if (!H.sorted_len.empty()) CK(cudaMemcpy(D->sorted_len.p, H.sorted_len.data(), sizeof(int32_t) * H.sorted_len.size(), cudaMemcpyHostToDevice));
       db->devs.push_back(std::move(D));
     }
+    // the merge copies committed units' scores and hits between GPUs: direct over NVLink
+    for (int a : devs)
+      for (int b : devs) {
+        if (a == b) continue;
+        int ok = 0;
+        if (cudaDeviceCanAccessPeer(&ok, a, b) == cudaSuccess && ok) {
+          CK(cudaSetDevice(a));
+          const cudaError_t e = cudaDeviceEnablePeerAccess(b, 0);
+          if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
+          else CK(e);
+        }
+      }
     *out = db.release();
   });
 }
@@ -559,7 +655,7 @@ int sw_topk_device(sw_db *db, const int32_t *scores_dev, int32_t nq, int32_t ndb
                    sw_hit *hits_dev) {
   return guarded([&] {
     if (!db || db->devs.empty()) throw Error(SW_EINVAL, "db is NULL");
-    if (k < 0 || k > 64) throw Error(SW_EINVAL, "top_k must be in [0, 64]");
+    if (k < 0 || k > SW_MAX_TOP_K) throw Error(SW_EINVAL, "top_k must be in [0, 64]");
     if (nq <= 0 || k == 0) return;
     CK(cudaSetDevice(db->devs[0]->id));
     launch_topk(scores_dev, nq, ndb, k, reinterpret_cast<int2 *>(hits_dev), 0);
@@ -581,7 +677,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
     if (gap_open < 0 || gap_extend < 0) throw Error(SW_EINVAL, "gap penalties must be >= 0");
     if ((int64_t)gap_open + 2 * (int64_t)gap_extend > (1 << 20))
       throw Error(SW_EINVAL, "gap_open + 2*gap_extend must be <= 2^20");
-    if (top_k < 0 || top_k > 64) throw Error(SW_EINVAL, "top_k must be in [0, 64]");
+    if (top_k < 0 || top_k > SW_MAX_TOP_K) throw Error(SW_EINVAL, "top_k must be in [0, 64]");
     sw_opts o;
     sw_opts_default(&o);
     if (opts_in) o = *opts_in;
@@ -589,6 +685,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
     if (o.streams_per_device <= 0) o.streams_per_device = 4;
     if (o.streams_per_device > kMaxStreams) throw Error(SW_EINVAL, "streams_per_device must be <= 64");
     if (o.policy != SW_POLICY_SS && o.policy != SW_POLICY_PSS) throw Error(SW_EINVAL, "bad policy");
+    if (o.straggler_mode < 0 || o.straggler_mode > 2) throw Error(SW_EINVAL, "bad straggler_mode");
     const bool dist = o.dist_world > 1;
     if (dist && (o.dist_rank < 0 || o.dist_rank >= o.dist_world || !o.dist_host || o.dist_port <= 0))
       throw Error(SW_EINVAL, "bad multi-process options");
@@ -608,6 +705,9 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
     const int nW = dist ? 1 : (int)db->devs.size();
     Plan P = make_plan(queries, H, o, dist ? o.dist_world : nW, M, thresh);
     const double wall0 = now_s();
+    const int K = (hits && top_k > 0 && nq > 0) ? top_k : 0;   // hits wanted
+    const int64_t nsc = (int64_t)nq * nd;
+    const int32_t nU = (int32_t)P.units.size();
 
     std::vector<DevSearch *> S(nW);
     // ---------------- per device setup (cached, grow-only resources; not device-timed)
@@ -651,7 +751,6 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       X.slices.ensure(D.id, P.slices.size());
       if (!P.slices.empty()) CK(cudaMemcpy(X.slices.p, P.slices.data(), sizeof(SliceInfo) * P.slices.size(), cudaMemcpyHostToDevice));
       CK(cudaMemcpy(X.matrix.p, M, 24 * 24, cudaMemcpyHostToDevice));
-      const size_t nsc = (size_t)nq * nd;
       if (w == 0 && o.outputs_on_device && scores && !dist) X.scores = scores;
       else { X.scores_own.ensure(D.id, nsc); X.scores = X.scores_own.p; }
       // saturated-pair lists: 2^20 per stream, or every pair when the s16x2 path is not
@@ -662,22 +761,37 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       X.ovf_cursor.ensure(D.id, depth);
       X.ovf_bits.ensure(D.id, ((size_t)nq * nd + 31) / 32);
       X.k2_border.ensure(D.id, (size_t)depth * kK2Blocks * std::max<int64_t>(P.max_len, 1) * 2);
-      const size_t k3b = (size_t)depth * std::max(P.max_k3_seqs, 1) * k3_phases() *
+      const size_t k3b = (size_t)depth * std::max(P.max_k3_seqs, 1) *
                          ((std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16);
       if (P.n_long_seqs > 0) X.k3_border.ensure(D.id, k3b);
       const size_t nu = std::max<size_t>(P.units.size(), 1);
       X.abort_dev.ensure(D.id, nu);
       CK(cudaMemset(X.abort_dev.p, 0, sizeof(int32_t) * nu));
+      X.progress.ensure(D.id, nu);
+      CK(cudaMemset(X.progress.p, 0, sizeof(int32_t) * nu));
       X.abort_d = X.abort_dev.p;
       X.cancelled.assign(nu, 0);
+      if (K > 0) {
+        X.pack_q.ensure(D.id, std::max<size_t>(P.pack_q.size(), 1));
+        if (!P.pack_q.empty()) CK(cudaMemcpy(X.pack_q.p, P.pack_q.data(), sizeof(int32_t) * P.pack_q.size(), cudaMemcpyHostToDevice));
+        X.unit_hits.ensure(D.id, nu * P.max_pack_q * K);
+        X.worker_hits.ensure(D.id, (size_t)nq * K);
+      }
       if (!X.one_h) {
         CK(cudaHostAlloc((void **)&X.one_h, sizeof(int32_t), cudaHostAllocDefault));
         *X.one_h = 1;
         CK(cudaHostAlloc((void **)&X.ovf_seen_h, sizeof(int32_t) * kMaxStreams, cudaHostAllocDefault));
+        CK(cudaHostAlloc((void **)&X.prog_h, sizeof(int32_t) * kMaxStreams, cudaHostAllocDefault));
       }
       if (!X.cancel_st) CK(cudaStreamCreateWithFlags(&X.cancel_st, cudaStreamNonBlocking));
+      if (!X.noise_st) {
+        int lo = 0, hi = 0;
+        CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+        CK(cudaStreamCreateWithPriority(&X.noise_st, cudaStreamNonBlocking, hi));
+      }
       if (!X.ev_start) CK(cudaEventCreate(&X.ev_start));
       if (!X.ev_end) CK(cudaEventCreate(&X.ev_end));
+      if (!X.ev_data) CK(cudaEventCreateWithFlags(&X.ev_data, cudaEventDisableTiming));
       while ((int)X.u_start.size() < depth) {
         cudaEvent_t a, b;
         CK(cudaEventCreate(&a));
@@ -698,10 +812,10 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       if (o.dist_rank == 0) {
         server = std::make_unique<MasterServer>();
         server->start(o.dist_port, o.dist_world, (int32_t)ucells.size(), ucells.data(), o.policy,
-                      o.workload_adjust, o.omega);
+                      o.workload_adjust, o.omega, P.hash);
       }
       client = std::make_unique<SchedClient>();
-      client->connect(o.dist_host, o.dist_port, o.dist_rank, 30.0);
+      client->connect(o.dist_host, o.dist_port, o.dist_rank, 30.0, P.hash);
     } else {
       sched = sw_sched_create(nW, (int32_t)ucells.size(), ucells.data(), o.policy, o.workload_adjust, o.omega);
       if (!sched && !ucells.empty()) throw Error(SW_EINVAL, "scheduler creation failed");
@@ -713,6 +827,12 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       if (!sched) return -1;
       return sw_sched_request(sched, w, t, out, cap);
     };
+    // an idle worker's request: one message that waits at the master (long poll)
+    auto sreq_wait = [&](int w, double t, int32_t *out, int cap, double timeout) -> int32_t {
+      if (client) return client->request_wait(t, out, cap, timeout);
+      if (!sched) return -1;
+      return sw_sched_request_wait(sched, w, t, out, cap, timeout);
+    };
     auto srep = [&](int w, double t, double cells, double sec) {
       if (client) client->report(t, cells, sec);
       else if (sched) sw_sched_report(sched, w, t, cells, sec);
@@ -720,6 +840,10 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
     auto scomp = [&](int w, int u, double t) -> int {
       if (client) return client->complete(u, t);
       return sched ? sw_sched_complete(sched, w, u, t) : 1;
+    };
+    auto sabandon = [&](int w, int u, double t) {
+      if (client) client->abandon(u, t);
+      else if (sched) sw_sched_abandon(sched, w, u, t);
     };
     auto sfin = [&](int u) -> int {
       if (client) return client->is_finished(u);
@@ -733,6 +857,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
     // ---------------- workers: one thread per device
     std::vector<UnitLog> ulog;
     std::mutex ulog_mu;
+    std::vector<std::vector<SegInfo>> worker_segs_(nW);   // committed segments of workers > 0
     std::atomic<int> ready{0};
     std::atomic<bool> failed{false};   // a worker failed: the others stop (no hang on its units)
     std::vector<std::string> werr(nW);
@@ -742,6 +867,13 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       DevSearch &X = *S[w];
       Device &D = *X.D;
       const int wid = my_worker_base + w;
+      bool noise_on = false;
+      auto stop_noise = [&] {
+        if (!noise_on) return;
+        noise_on = false;
+        cudaMemcpyAsync(X.noise_flag.p, X.one_h, sizeof(int32_t), cudaMemcpyHostToDevice, X.cancel_st);
+        cudaStreamSynchronize(X.noise_st);
+      };
       try {
         CK(cudaSetDevice(D.id));
         const int depth = o.streams_per_device;
@@ -762,31 +894,49 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         CK(cudaEventCreateWithFlags(&setup_done, cudaEventDisableTiming));
         CK(cudaEventRecord(setup_done, s0));
         for (int k = 1; k < depth; k++) CK(cudaStreamWaitEvent(D.streams[k], setup_done, 0));
+        // slower-PE emulation (SURVEY §8(d) WA experiment; P24 §V.C local load from t_after)
         const bool straggler = (o.straggler_mask >> wid) & 1ull;
-        const double slow = std::max(1, o.straggler_slowdown);
+        const int slow = std::max(1, o.straggler_slowdown);
+        const int sm_cap = (D.n_sm + slow - 1) / slow;     // ceil(n_sm / slowdown)
+        // mode SM cap: the worker's budget of sm_cap SMs is split over its streams (up to
+        // `depth` units run at once), so the whole worker holds ~sm_cap SMs' worth of blocks
+        const int sm_share = std::max(1, (sm_cap + depth - 1) / depth);
+        const double t_after = 1e-3 * std::max(0, o.straggler_after_ms);
         std::deque<int32_t> pending;
         std::vector<int32_t> inflight(depth, -1);
         std::vector<double> t_grant(P.units.size(), 0), t_launch(depth, 0);
         std::vector<double> hold_until(depth, 0);
-        std::vector<int> completed_wait(depth, 0);
+        std::vector<int> completed_wait(depth, 0), slowed(depth, 0);
         std::vector<int32_t> k2_upto(depth, 0);   // saturated pairs handed to K2 per stream
-        bool done = false;
-        double last_report = now_s();
+        bool done = false, changed = true;
+        double last_req = 0;
+        std::vector<double> stream_rate(depth, 0.0);
         int32_t buf[64];
         while (true) {
           if (failed.load()) throw Error(SW_ECUDA, "another worker failed");
           bool progressed = false;
           const double tn = now_s();
+          const bool slow_now = straggler && slow > 1 && tn - t0 >= t_after;
+          if (slow_now && o.straggler_mode == SW_STRAGGLER_NOISE && !noise_on) {
+            // local load: SM-filling blocks on all but ceil(n_sm / slowdown) SMs
+            X.noise_flag.ensure(D.id, 1);
+            X.noise_sink.ensure(D.id, D.n_sm);
+            CK(cudaMemsetAsync(X.noise_flag.p, 0, sizeof(int32_t), X.noise_st));
+            launch_noise(X.noise_flag.p, D.n_sm - sm_cap, 60ull * 1000000000ull, X.noise_sink.p, X.noise_st);
+            CK(cudaGetLastError());
+            noise_on = true;
+          }
           // completions
           for (int k = 0; k < depth; k++) {
             if (inflight[k] < 0) continue;
+            const int u = inflight[k];
             if (!completed_wait[k]) {
               cudaError_t q = cudaEventQuery(X.u_end[k]);
               if (q == cudaErrorNotReady) continue;
               CK(q);
               completed_wait[k] = 1;
-              if (straggler && tn - t0 >= 1e-3 * o.straggler_after_ms) {
-                // emulate a PE `slow` times slower (SURVEY §8(d) WA experiment; P24 §V.C)
+              if (slowed[k] && o.straggler_mode == SW_STRAGGLER_HOLD && !X.cancelled[u]) {
+                // host-side emulation: hold the completion back (slow-1) x the device time
                 float ms = 0;
                 cudaEventElapsedTime(&ms, X.u_start[k], X.u_end[k]);
                 hold_until[k] = tn + (slow - 1.0) * ms * 1e-3;
@@ -794,26 +944,52 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
                 hold_until[k] = tn;
               }
             }
-            // an emulated slow PE stops working on a replica whose task finished elsewhere
+            // an emulated slow PE stops holding a replica whose task finished elsewhere
             // (WA: the first result wins and the other replicas are cancelled)
-            if (tn < hold_until[k] && !sfin(inflight[k])) continue;
-            const int u = inflight[k];
+            const bool cut = tn < hold_until[k] && sfin(u);
+            if (tn < hold_until[k] && !cut) continue;
             const Unit &U = P.units[u];
-            float ms = 0;
+            float ms = 0, d0 = 0, d1 = 0;
             cudaEventElapsedTime(&ms, X.u_start[k], X.u_end[k]);
-            const int committed = scomp(wid, u, tn);
-            srep(wid, tn, (double)U.cells, std::max(1e-6, tn - last_report));
-            last_report = tn;
-            if (U.kind == kUnitInter) { X.k1_sec += ms * 1e-3; X.k1_cells += U.cells; }
-            else { X.k3_sec += ms * 1e-3; X.k3_cells += U.cells; }
-            if (!committed) X.dup_cells += U.cells;
+            cudaEventElapsedTime(&d0, X.ev_start, X.u_start[k]);
+            cudaEventElapsedTime(&d1, X.ev_start, X.u_end[k]);
+            // what the replica really computed: its progress counter (groups / sequence-chunks)
+            const int64_t ptot = std::max<int64_t>(1, unit_progress_total(P, U));
+            const int64_t pdone = std::min<int64_t>(ptot, ((volatile int32_t *)X.prog_h)[k]);
+            const bool was_cancelled = X.cancelled[u] && pdone < ptot;
+            const int64_t cells_done = was_cancelled ? (int64_t)((double)U.cells * pdone / ptot) : U.cells;
+            int committed = 0;
+            if (was_cancelled) {
+              // a losing replica stopped early by its abort flag: give it up; its partial
+              // cells count as duplicated work and as this PE's progress
+              sabandon(wid, u, tn);
+              X.n_cancelled++;
+            } else {
+              committed = scomp(wid, u, tn);
+            }
+            // progress notification (P18 §IV.A.2): the worker's current rate = the sum over
+            // its streams of (cells / duration) of each stream's last unit -- units share the
+            // GPU, so each one's rate is its share; a duration is launch -> observed
+            // completion, which includes a GPU-side slowdown (SM cap, local load) and the
+            // host-side hold
+            if (!cut && cells_done > 0) {
+              stream_rate[k] = (double)cells_done / std::max(1e-6, tn - t_launch[k]);
+              double v = 0;
+              for (double r : stream_rate) v += r;
+              srep(wid, tn, v, 1.0);
+            }
+            if (U.kind == kUnitInter) { X.k1_sec += ms * 1e-3; X.k1_cells += cells_done; }
+            else { X.k3_sec += ms * 1e-3; X.k3_cells += cells_done; }
+            if (!committed) X.dup_cells += cells_done;
+            X.last_dev = std::max(X.last_dev, 1e-3 * d1);
             {
               std::lock_guard<std::mutex> g(ulog_mu);
-              ulog.push_back({u, wid, k, t_grant[u] - t0, t_launch[k] - t0, tn - t0, U.cells, committed, ms});
+              ulog.push_back({u, wid, k, t_grant[u] - t0, t_launch[k] - t0, tn - t0, U.cells, cells_done,
+                              committed, was_cancelled ? 1 : 0, slowed[k], ms, d0, d1});
             }
             inflight[k] = -1;
             completed_wait[k] = 0;
-            progressed = true;
+            progressed = changed = true;
             // int32 re-run of what this unit saturated, on its stream before the next unit
             // (overlaps the units in flight on the other streams)
             const int32_t seen = ((volatile int32_t *)X.ovf_seen_h)[k];
@@ -822,6 +998,19 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
               CK(cudaGetLastError());
               X.launches++;
               k2_upto[k] = seen;
+            }
+            if (committed) {
+              X.committed.push_back(u);
+              // K5u: this unit's top-k per query of its pack (after its int32 re-run)
+              if (K > 0) {
+                int32_t s0u, s1u;
+                unit_seq_range(U, nd, s0u, s1u);
+                const int32_t q0 = P.pack_q_off[U.pair], nqp = P.pack_q_off[U.pair + 1] - q0;
+                launch_unit_topk(X.scores, nd, D.perm.p, s0u, s1u, X.pack_q.p + q0, nqp, K,
+                                 X.unit_hits.p + (size_t)u * P.max_pack_q * K, D.streams[k]);
+                CK(cudaGetLastError());
+                X.launches++;
+              }
             }
           }
           // cancel in-flight replicas whose task finished elsewhere (WA loser)
@@ -837,32 +1026,46 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
             const int u = pending.front();
             pending.pop_front();
             // finished elsewhere, or moved to an idle worker by WA before it started
-            if (!sstart(wid, u, now_s())) { progressed = true; k--; continue; }
+            if (!sstart(wid, u, now_s())) { progressed = changed = true; k--; continue; }
+            const bool sl = straggler && slow > 1 && now_s() - t0 >= t_after;
             CK(cudaEventRecord(X.u_start[k], D.streams[k]));
-            launch_unit(P, H, X, P.units[u], u, k, alpha, beta, thresh);
+            launch_unit(P, H, X, P.units[u], u, k, alpha, beta, thresh,
+                        (sl && o.straggler_mode == SW_STRAGGLER_SM_CAP) ? sm_share : 0);
             CK(cudaGetLastError());
             CK(cudaEventRecord(X.u_end[k], D.streams[k]));
             inflight[k] = u;
+            slowed[k] = sl ? 1 : 0;
             t_launch[k] = now_s();
             progressed = true;
           }
-          // ask the master for more when the local queue is empty and a stream is free
+          // ask the master for more when the local queue is empty and a stream is free:
+          // once per change (a completion) or every 2 ms while units run; an idle worker
+          // sends one request that waits at the master until the task table changes
           int n_inflight = 0;
           for (int k = 0; k < depth; k++) n_inflight += inflight[k] >= 0;
           if (!done && pending.empty() && n_inflight < depth) {
-            const int32_t r = sreq(wid, now_s(), buf, 64);
+            int32_t r = 0;
+            const double tq = now_s();
+            if (n_inflight == 0) {
+              r = sreq_wait(wid, tq, buf, 64, 0.005);
+              last_req = tq;
+              changed = false;
+            } else if (changed || tq - last_req > 2e-3) {
+              r = sreq(wid, tq, buf, 64);
+              last_req = tq;
+              changed = false;
+            }
             if (r < 0) done = true;
             else {
               for (int32_t i = 0; i < r; i++) { pending.push_back(buf[i]); t_grant[buf[i]] = now_s(); }
-              if (r > 0) progressed = true;
+              if (r > 0) progressed = changed = true;
             }
           }
           if (done && pending.empty() && n_inflight == 0) break;
-          // poll completions every 20 us; an idle worker (nothing in flight, nothing granted)
-          // asks the master again every 100 us
-          if (!progressed)
-            std::this_thread::sleep_for(std::chrono::microseconds(n_inflight > 0 ? 20 : 100));
+          // poll completions every 20 us
+          if (!progressed && n_inflight > 0) std::this_thread::sleep_for(std::chrono::microseconds(20));
         }
+        stop_noise();
         // the int32 re-runs ran on each stream after the units that saturated; check the lists
         for (int k = 0; k < depth; k++) CK(cudaStreamSynchronize(D.streams[k]));
         std::vector<int32_t> novf(depth, 0), ncur(depth, 0);
@@ -874,16 +1077,73 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
           X.n_ovf += novf[k];
           if (ncur[k] < novf[k]) throw Error(SW_ECUDA, "int32 re-run left saturated pairs");
         }
+        // ---- data plane, on this device: top-k over the units this worker committed
+        // (K5m), and (in-process, device != first) the committed units' scores packed densely
+        // for the peer copy; multi-process: the committed-only score matrix
+        std::vector<SegInfo> segs;
+        int64_t seg_total = 0;
+        const bool need_segs = (dist && scores) || (!dist && w > 0 && scores);
+        if (need_segs)
+          for (int32_t u : X.committed) {
+            int32_t s0u, s1u;
+            unit_seq_range(P.units[u], nd, s0u, s1u);
+            for (int32_t j = P.pack_q_off[P.units[u].pair]; j < P.pack_q_off[P.units[u].pair + 1]; j++) {
+              segs.push_back({P.pack_q[j], s0u, s1u, 0, seg_total});
+              seg_total += s1u - s0u;
+            }
+          }
+        std::vector<int32_t> tab;   // list_off[nq+1], then list_idx
+        if (K > 0) {
+          std::vector<std::vector<int32_t>> per_q(nq);
+          for (int32_t u : X.committed) {
+            const int32_t p = P.units[u].pair;
+            for (int32_t j = P.pack_q_off[p]; j < P.pack_q_off[p + 1]; j++)
+              per_q[P.pack_q[j]].push_back(u * P.max_pack_q + (j - P.pack_q_off[p]));
+          }
+          tab.assign(nq + 1, 0);
+          for (int32_t q = 0; q < nq; q++) tab[q + 1] = tab[q] + (int32_t)per_q[q].size();
+          for (int32_t q = 0; q < nq; q++) tab.insert(tab.end(), per_q[q].begin(), per_q[q].end());
+        }
+        if (!tab.empty() || !segs.empty()) {
+          X.list_tab.ensure(D.id, std::max<size_t>(tab.size(), 1));
+          if (!tab.empty()) CK(cudaMemcpyAsync(X.list_tab.p, tab.data(), sizeof(int32_t) * tab.size(), cudaMemcpyHostToDevice, s0));
+          X.segs.ensure(D.id, std::max<size_t>(segs.size(), 1));
+          if (!segs.empty()) CK(cudaMemcpyAsync(X.segs.p, segs.data(), sizeof(SegInfo) * segs.size(), cudaMemcpyHostToDevice, s0));
+        }
+        if (K > 0) {
+          launch_merge_topk(X.unit_hits.p, K, X.list_tab.p, X.list_tab.p + nq + 1, nq, K, X.worker_hits.p, s0);
+          X.launches++;
+        }
+        if (dist && scores && nsc > 0) {   // this rank's output: its committed pairs, -1 elsewhere
+          X.out_stage.ensure(D.id, o.outputs_on_device ? 1 : nsc);
+          int32_t *dst = o.outputs_on_device ? scores : X.out_stage.p;
+          launch_fill(dst, nsc, -1, s0);
+          launch_seg_copy(X.scores, dst, nd, D.perm.p, X.segs.p, (int)segs.size(), 2, s0);
+          X.launches += segs.empty() ? 1 : 2;
+        } else if (!segs.empty()) {
+          X.compact.ensure(D.id, std::max<int64_t>(seg_total, 1));
+          launch_seg_copy(X.scores, X.compact.p, nd, D.perm.p, X.segs.p, (int)segs.size(), 0, s0);
+          X.launches++;
+        }
+        CK(cudaGetLastError());
+        CK(cudaEventRecord(X.ev_data, s0));
         CK(cudaEventRecord(X.ev_end, s0));
         CK(cudaEventSynchronize(X.ev_end));
         CK(cudaEventDestroy(setup_done));
         X.finish_wall = now_s();
+        // seg list kept for the merge stage (device 0 needs the offsets)
+        if (!dist && w > 0) {
+          std::lock_guard<std::mutex> g(ulog_mu);
+          worker_segs_[w].swap(segs);
+        }
       } catch (const Error &e) {
+        stop_noise();
         werr[w] = e.what();
         wcode[w] = e.code;
         failed.store(true);
         ready.fetch_add(1 << 20);  // release the barrier
       } catch (const std::exception &e) {
+        stop_noise();
         werr[w] = e.what();
         wcode[w] = SW_ECUDA;
         failed.store(true);
@@ -898,37 +1158,85 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         throw Error(wcode[w], "worker " + std::to_string(w) + ": " + werr[w]);
     for (int w = 0; w < nW; w++)
       if (wcode[w]) throw Error(wcode[w], "worker " + std::to_string(w) + ": " + werr[w]);
-    if (client) client->done();
-    if (server) server->stop();
+    int32_t n_req = 0, n_wa = 0, n_grant = 0;
+    if (sched) {
+      n_wa = (int32_t)sw_sched_counter(sched, 1);
+      n_req = (int32_t)sw_sched_counter(sched, 0);
+      n_grant = (int32_t)sw_sched_counter(sched, 3);
+      db->sched_log = sw_sched_log_json(sched);
+    }
+    if (client) {
+      client->done();
+      n_wa = client->wa_grants();
+      n_req = client->requests();
+      n_grant = client->grant_msgs();
+    }
+    if (server) {
+      server->stop();
+      db->sched_log = server->final_log();
+    } else if (!sched) {
+      db->sched_log = "[]";
+    }
 
-    // ---------------- merge (in-process multi-device: device 0 pulls the others over
-    // NVLink and takes the element-wise max; every pair was written by >= 1 device with
-    // identical values, the rest are -1), then top-k on device 0
+    // ---------------- merge (the paper's "the slaves send their results to the master, that
+    // merges them", P16 §IV).  In-process with several GPUs: every other GPU's committed
+    // units' scores (packed densely on that GPU) and its top-k lists are copied to the first
+    // GPU over NVLink (peer access enabled at sw_db_create) and merged there (scatter + K5m).
+    // Multi-process: each rank keeps its committed pairs and hits; the binding gathers the
+    // hits (NCCL) and merges them with sw_merge_hits.
     DevSearch &X0 = *S[0];
-    CK(cudaSetDevice(X0.D->id));
+    const int dev0 = X0.D->id;
+    CK(cudaSetDevice(dev0));
     cudaStream_t s0 = X0.D->streams[0];
     cudaEvent_t m_start, m_end;
     CK(cudaEventCreate(&m_start));
     CK(cudaEventCreate(&m_end));
     CK(cudaEventRecord(m_start, s0));
-    const int64_t nsc = (int64_t)nq * nd;
-    DBuf<int32_t> tmp;
-    if (nW > 1 && nsc > 0) {
-      tmp.alloc(X0.D->id, nsc);
+    int64_t peer_bytes = 0;
+    DBuf<int32_t> stage;
+    DBuf<SegInfo> segs0;
+    DBuf<int32_t> tab0;
+    DBuf<int2> hits_tmp;
+    const int2 *hits_final = nullptr;
+    if (!dist && nW > 1) {
       for (int w = 1; w < nW; w++) {
-        CK(cudaMemcpyPeerAsync(tmp.p, X0.D->id, S[w]->scores, S[w]->D->id, sizeof(int32_t) * nsc, s0));
-        launch_max_merge(X0.scores, tmp.p, nsc, s0);
+        const std::vector<SegInfo> &sg_ = worker_segs_[w];
+        if (sg_.empty()) continue;
+        const int64_t total = sg_.back().off + (sg_.back().s1 - sg_.back().s0);
+        CK(cudaStreamWaitEvent(s0, S[w]->ev_data, 0));
+        stage.ensure(dev0, std::max<int64_t>(total, 1));
+        CK(cudaMemcpyPeerAsync(stage.p, dev0, S[w]->compact.p, S[w]->D->id, sizeof(int32_t) * total, s0));
+        peer_bytes += sizeof(int32_t) * total;
+        segs0.ensure(dev0, sg_.size());
+        CK(cudaMemcpyAsync(segs0.p, sg_.data(), sizeof(SegInfo) * sg_.size(), cudaMemcpyHostToDevice, s0));
+        launch_seg_copy(stage.p, X0.scores, nd, X0.D->perm.p, segs0.p, (int)sg_.size(), 1, s0);
         X0.launches++;
+        // the staging buffer is reused by the next worker: keep the copies ordered on s0
       }
+      if (K > 0) {
+        X0.all_hits.ensure(dev0, (size_t)nW * nq * K);
+        for (int w = 0; w < nW; w++) {
+          CK(cudaStreamWaitEvent(s0, S[w]->ev_data, 0));
+          CK(cudaMemcpyPeerAsync(X0.all_hits.p + (size_t)w * nq * K, dev0, S[w]->worker_hits.p, S[w]->D->id,
+                                 sizeof(int2) * nq * K, s0));
+          if (w > 0) peer_bytes += sizeof(int2) * nq * K;
+        }
+        std::vector<int32_t> tab(nq + 1 + (size_t)nq * nW);
+        for (int32_t q = 0; q <= nq; q++) tab[q] = q * nW;
+        for (int32_t q = 0; q < nq; q++)
+          for (int w = 0; w < nW; w++) tab[nq + 1 + (size_t)q * nW + w] = w * nq + q;
+        tab0.ensure(dev0, tab.size());
+        CK(cudaMemcpyAsync(tab0.p, tab.data(), sizeof(int32_t) * tab.size(), cudaMemcpyHostToDevice, s0));
+        hits_tmp.ensure(dev0, (size_t)nq * K);
+        launch_merge_topk(X0.all_hits.p, K, tab0.p, tab0.p + nq + 1, nq, K, hits_tmp.p, s0);
+        X0.launches++;
+        hits_final = hits_tmp.p;
+      }
+    } else if (K > 0) {
+      hits_final = X0.worker_hits.p;
     }
-    DBuf<int2> hits_dev;
-    int2 *hits_out = nullptr;
-    if (hits && top_k > 0 && nq > 0) {
-      if (o.outputs_on_device) hits_out = reinterpret_cast<int2 *>(hits);
-      else { hits_dev.alloc(X0.D->id, (size_t)nq * top_k); hits_out = hits_dev.p; }
-      launch_topk(X0.scores, nq, nd, top_k, hits_out, s0);
-      X0.launches++;
-    }
+    if (K > 0 && o.outputs_on_device)
+      CK(cudaMemcpyAsync(hits, hits_final, sizeof(int2) * nq * K, cudaMemcpyDeviceToDevice, s0));
     CK(cudaGetLastError());
     CK(cudaEventRecord(m_end, s0));
     CK(cudaEventSynchronize(m_end));
@@ -946,15 +1254,12 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       dev_sec = std::max(dev_sec, sec);
     }
     // outputs
-    if (scores && nsc > 0) {
-      if (o.outputs_on_device) {
-        if (X0.scores != scores) CK(cudaMemcpy(scores, X0.scores, sizeof(int32_t) * nsc, cudaMemcpyDeviceToDevice));
-      } else {
-        CK(cudaMemcpy(scores, X0.scores, sizeof(int32_t) * nsc, cudaMemcpyDeviceToHost));
-      }
+    if (scores && nsc > 0 && !o.outputs_on_device) {
+      const int32_t *src = dist ? X0.out_stage.p : X0.scores;
+      CK(cudaMemcpy(scores, src, sizeof(int32_t) * nsc, cudaMemcpyDeviceToHost));
     }
-    if (hits && top_k > 0 && nq > 0 && !o.outputs_on_device)
-      CK(cudaMemcpy(hits, hits_dev.p, sizeof(int2) * nq * top_k, cudaMemcpyDeviceToHost));
+    if (K > 0 && !o.outputs_on_device)
+      CK(cudaMemcpy(hits, hits_final, sizeof(int2) * nq * K, cudaMemcpyDeviceToHost));
     const double wall = now_s() - wall0;
 
     if (stats) {
@@ -974,17 +1279,18 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         stats->kernel_seconds_k3 += S[w]->k3_sec;
         stats->cells_k1 += S[w]->k1_cells;
         stats->cells_k3 += S[w]->k3_cells;
-        fin.push_back(S[w]->finish_wall - t0);
+        stats->n_cancelled += S[w]->n_cancelled;
+        fin.push_back(S[w]->last_dev);
       }
+      // tail: makespan of the units minus the (lower) median over workers of
+      // each worker's last device completion (device clocks from each worker's start event)
       std::sort(fin.begin(), fin.end());
-      stats->tail_seconds = fin.empty() ? 0 : fin.back() - fin[fin.size() / 2];
-      if (sched) {
-        stats->n_wa_grants = (int32_t)sw_sched_counter(sched, 1);
-        stats->n_requests = (int32_t)sw_sched_counter(sched, 0);
-      } else if (client) {
-        stats->n_wa_grants = client->wa_grants();
-        stats->n_requests = client->requests();
-      }
+      stats->seconds_last_unit = fin.empty() ? 0 : fin.back();
+      stats->tail_seconds = fin.empty() ? 0 : fin.back() - fin[(fin.size() - 1) / 2];
+      stats->n_wa_grants = n_wa;
+      stats->n_requests = n_req;
+      stats->n_grant_messages = n_grant;
+      stats->peer_bytes = peer_bytes;
       std::ostringstream js;
       js << "[";
       for (size_t k = 0; k < ulog.size(); k++) {
@@ -992,16 +1298,43 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         const Unit &U = P.units[L.unit];
         js << (k ? "," : "") << "{\"unit\":" << L.unit << ",\"kind\":" << U.kind << ",\"pair\":" << U.pair
            << ",\"worker\":" << L.worker << ",\"t_grant\":" << L.t_grant << ",\"t_start\":" << L.t_start
-           << ",\"t_end\":" << L.t_end << ",\"cells\":" << L.cells << ",\"committed\":" << L.committed
-           << ",\"stream\":" << L.stream << ",\"device_ms\":" << L.device_ms << "}";
+           << ",\"t_end\":" << L.t_end << ",\"cells\":" << L.cells << ",\"cells_done\":" << L.cells_done
+           << ",\"committed\":" << L.committed << ",\"cancelled\":" << L.cancelled << ",\"slowed\":" << L.slowed
+           << ",\"stream\":" << L.stream << ",\"device_ms\":" << L.device_ms << ",\"dev_t0\":" << L.dev_t0
+           << ",\"dev_t1\":" << L.dev_t1 << "}";
       }
       js << "]";
       db->unit_log = js.str();
       stats->unit_log_json = db->unit_log.c_str();
+      stats->sched_log_json = db->sched_log.c_str();
     }
   });
   if (db) db->busy.store(0);
   return rc;
+}
+
+int sw_merge_hits(sw_db *db, const sw_hit *lists_dev, int32_t n_sources, int32_t nq, int32_t k_in,
+                  int32_t top_k, sw_hit *hits_dev) {
+  return guarded([&] {
+    if (!db || db->devs.empty()) throw Error(SW_EINVAL, "db is NULL");
+    if (n_sources < 0 || nq < 0 || k_in < 0 || top_k < 0) throw Error(SW_EINVAL, "negative size");
+    if (top_k > SW_MAX_TOP_K) throw Error(SW_EINVAL, "top_k must be in [0, 64]");
+    if (nq == 0 || top_k == 0) return;
+    if (!hits_dev || (n_sources > 0 && k_in > 0 && !lists_dev)) throw Error(SW_EINVAL, "NULL buffer");
+    const int dev = db->devs[0]->id;
+    CK(cudaSetDevice(dev));
+    std::vector<int32_t> tab(nq + 1 + (size_t)nq * n_sources);
+    for (int32_t q = 0; q <= nq; q++) tab[q] = q * n_sources;
+    for (int32_t q = 0; q < nq; q++)
+      for (int32_t r = 0; r < n_sources; r++) tab[nq + 1 + (size_t)q * n_sources + r] = r * nq + q;
+    DBuf<int32_t> t;
+    t.alloc(dev, tab.size());
+    CK(cudaMemcpy(t.p, tab.data(), sizeof(int32_t) * tab.size(), cudaMemcpyHostToDevice));
+    launch_merge_topk(reinterpret_cast<const int2 *>(lists_dev), std::max(k_in, 1), t.p, t.p + nq + 1, nq, top_k,
+                      reinterpret_cast<int2 *>(hits_dev), 0);
+    CK(cudaGetLastError());
+    CK(cudaDeviceSynchronize());
+  });
 }
 
 int sw_align(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t gap_open,

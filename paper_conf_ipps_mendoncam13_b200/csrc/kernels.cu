@@ -53,6 +53,7 @@ __device__ __forceinline__ bool block_aborted(const volatile int32_t *flag) {
   __syncthreads();
   return ab != 0;
 }
+constexpr int kAbortPoll = 32;   // K1 pipeline steps between WA cancellation polls
 __device__ __forceinline__ uint32_t smid() {
   uint32_t r;
   asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
@@ -403,8 +404,19 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
       }
       if (warp == 0) cp_async_commit_wait();
     }
-    __syncthreads();
+    // WA cancellation (P18 §IV.A.3: the first replica to finish wins): every kAbortPoll
+    // steps thread 0 reads the unit's flag and the step's barrier ORs it over the block,
+    // so a losing replica stops within kAbortPoll steps (~0.1 ms), not at the end of its
+    // groups.  Partial maxima already flushed are <= the true scores (atomicMax-safe).
+    if ((s % kAbortPoll) == kAbortPoll - 1 && a.abort_flag) {
+      if (__syncthreads_or(threadIdx.x == 0 && *a.abort_flag != 0)) break;
+    } else {
+      __syncthreads();
+    }
   }
+  // groups this block finished (warp W-1 is the last to leave a group): the host turns
+  // the unit's count into the cells a cancelled replica really computed
+  if (a.progress && warp == W - 1 && lane == 0 && gk > 0) atomicAdd(a.progress, gk);
   if (nb > 1 && threadIdx.x == 0) atomicExch(&a.slot_busy[slot_s], 0);
 }
 
@@ -499,232 +511,254 @@ void launch_k1(const K1Args &a_in, int n_groups, int min_cols, int, cudaStream_t
 // the previous chunk's border row and the packed database (streamed by cp.async through a
 // 3-deep shared-memory ring, two tiles ahead), and lane 31 writes the chunk's bottom row
 // to the border.
-//
-// Chunk phases (PH): the chunks of a pair are dealt round-robin to PH warps, chunk c to
-// phase c % PH, and phase p+1 runs chunk c+1 while phase p is still on chunk c (it reads
-// the border tile by tile, behind a per-warp progress counter in shared memory), so one
-// long pair takes about 1/PH of the single-warp latency: the fine-grained wavefront of
-// Fig. 3a applied once more, across warps ("it sends its border column to P1", P14).
-// Block = kK3Warps sequences x PH phases; the kK3Warps warps of a phase share that
-// phase's chunk profile in shared memory, laid out [code][row-in-lane][lane] (bank =
-// lane: conflict-free although every lane reads a different code).  Every dependency
-// points to a lower chunk (progress: chunk c waits for c-1; the phase barrier before
-// chunk c waits for c-PH), so the warps of a block cannot deadlock.
+// Block = kK3Warps sequences sharing the chunk profile in shared memory, laid out
+// [slot][row pair][lane][2] (8-byte bank pair = lane mod 16: conflict-free although every
+// lane reads a different code).  A block walks sequence blocks blockIdx.x, +gridDim.x, ...
+// (one pass normally; several when the grid is capped to emulate a slower PE).  The unit's
+// WA cancellation flag is polled at every chunk start (__syncthreads_or), and each warp
+// counts the (sequence, chunk) pairs it completed into the unit's progress counter.
 // ------------------------------------------------------------------------------------
-__device__ __forceinline__ void named_barrier(int id, int threads) {
-  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(threads) : "memory");
-}
-
-template <int K, int T, int PH>
-__global__ void __launch_bounds__(kK3Warps * PH * 32) k3_kernel(const K3Args a) {
+template <int K, int T>
+__global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
   static_assert(T == 4 || T == 8, "tile = one or two 32-bit words of packed residues");
   constexpr int NW = T / 4;          // 32-bit residue words per tile
   constexpr int TPU = 4 / NW;        // tiles per 128-bit word
   constexpr int CH = 32 * K;
-  constexpr int NWARP = kK3Warps * PH;
-  constexpr int PROF = kNCodes * K * 32;   // words of one chunk profile
-  extern __shared__ __align__(16) uint32_t smem[];  // [PH][kNCodes][K][32], then the rings
-  uint4 *ring4 = reinterpret_cast<uint4 *>(smem + PH * PROF);      // [warps][3]
-  uint2 *ring2 = reinterpret_cast<uint2 *>(ring4 + NWARP * 3);    // [warps][3][T]
-  __shared__ int prog_s[NWARP];   // tiles of border published by each warp (all its chunks)
+  extern __shared__ __align__(16) uint32_t smem[];  // [kNCodes][K/2][32][2], then the rings
+  uint4 *ring4 = reinterpret_cast<uint4 *>(smem + kNCodes * K * 32);   // [warps][3]
+  uint2 *ring2 = reinterpret_cast<uint2 *>(ring4 + kK3Warps * 3);     // [warps][3][T]
   if (block_aborted(a.abort_flag)) return;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  // sequence slot, phase: the PH warps of a sequence are consecutive, so producer and
-  // consumer sit on different SM sub-partitions (warp % 4) and a waiting consumer does
-  // not take issue slots from its own producer
-  const int sw = warp / PH, ph = warp % PH;
-  if (threadIdx.x < NWARP) prog_s[threadIdx.x] = 0;
   const QueryPair P = a.pairs[a.pair];
   const int rows = P.rows;
   const int nch = (rows + CH - 1) / CH;
   const int nslices = P.rows_padded / 16;
-  const int s = a.l0 + blockIdx.x * kK3Warps + sw;
-  const bool valid = s < a.l1;
-  const int len = valid ? a.sorted_len[s] : 0;
-  const GroupInfo G = a.groups[valid ? s / kGroup : 0];
-  const int gl = s % kGroup;
-  const uint4 *wp = a.packed + G.word_off + gl;
-  // border rows: this warp writes its own (phase ph of sequence slot), reads the previous
-  // phase's (the previous chunk)
-  const size_t bslot = (size_t)(blockIdx.x * kK3Warps + sw) * PH;
-  uint2 *border_out = a.border + (bslot + ph) * a.border_stride;
-  const int pph = ph == 0 ? PH - 1 : ph - 1;
-  const uint2 *border_in = a.border + (bslot + pph) * a.border_stride;
-  const volatile int *prog_in = prog_s + sw * PH + pph;
   const uint32_t koff = pk2(kOff), na = a.na, nbeta = a.nb;
   const uint32_t padw = 0x01010101u * kPadCode;
   const int32_t *gprof = a.prof + P.prof_off;
-  uint32_t *prof_s = smem + ph * PROF;
-  const int ntile = (len + T - 1) / T;   // columns up to ntile*T <= G.ncols carry pad codes
-  const int orig = valid ? a.perm[s] : 0;
-  uint32_t best = koff;
-  int cq_lo = -1, cq_hi = -1;   // queries of this lane's slice (per half)
-  int published = 0;            // border tiles this warp has published (lane 31's count)
-  __syncthreads();              // prog_s initialised
+  uint32_t *prof_s = smem;
+  const int nsb = (a.l1 - a.l0 + kK3Warps - 1) / kK3Warps;
+  int done = 0;          // (sequence, chunk) pairs this warp completed
+  bool aborted = false;
 
-  for (int ch = ph; ch < nch; ch += PH) {
-    // the kK3Warps warps of this phase reload its chunk profile (all done with chunk ch-PH)
-    if (PH == 1) __syncthreads(); else named_barrier(1 + ph, kK3Warps * 32);
-    for (int idx = sw * 32 + lane; idx < kNCodes * CH; idx += kK3Warps * 32) {
-      const int c = idx / CH, r = idx - c * CH;     // r = l*K + i
-      const int l = r / K, i = r - l * K;
-      // [slot][row pair][lane][2]: a lane's rows i, i+1 form one 8-byte word (LDS.64); the
-      // 8-byte bank pair is lane mod 16, so no conflicts although lanes read different slots
-      prof_s[((c * (K / 2) + i / 2) * 32 + l) * 2 + (i & 1)] =
-          (uint32_t)__ldg(gprof + (int64_t)c * P.rows_padded + ch * CH + r);
-    }
-    if (PH == 1) __syncthreads(); else named_barrier(1 + ph, kK3Warps * 32);
-    if (!valid) continue;
-    // lane l's rows of this chunk are slice ch*32 + l: flush a half whose query changed;
-    // the start mask of the slice below applies to what this lane hands down
-    uint32_t omask = 0;
-    {
-      const int sidx = ch * 32 + lane;
-      const SliceInfo si = a.slices[P.slice_off + sidx];
-      if (si.q_lo != cq_lo) {
-        flush_half(cq_lo, lo16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
-        best = (best & 0xffff0000u) | (koff & 0xffffu);
-        cq_lo = si.q_lo;
+  for (int sb = blockIdx.x; sb < nsb && !aborted; sb += gridDim.x) {
+    const int s = a.l0 + sb * kK3Warps + warp;
+    const bool valid = s < a.l1;
+    const int len = valid ? a.sorted_len[s] : 0;
+    const GroupInfo G = a.groups[valid ? s / kGroup : 0];
+    const int gl = s % kGroup;
+    const uint4 *wp = a.packed + G.word_off + gl;
+    uint2 *border = a.border + (size_t)(sb * kK3Warps + warp) * a.border_stride;
+    const int ntile = (len + T - 1) / T;   // columns up to ntile*T <= G.ncols carry pad codes
+    const int orig = valid ? a.perm[s] : 0;
+    uint32_t best = koff;
+    int cq_lo = -1, cq_hi = -1;   // queries of this lane's slice (per half)
+
+    for (int ch = 0; ch < nch; ch++) {
+      // every warp is done with the previous chunk profile; WA cancellation poll
+      if (__syncthreads_or(threadIdx.x == 0 && a.abort_flag && *a.abort_flag != 0)) {
+        aborted = true;
+        break;
       }
-      if (si.q_hi != cq_hi) {
-        flush_half(cq_hi, hi16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
-        best = (best & 0x0000ffffu) | (koff & 0xffff0000u);
-        cq_hi = si.q_hi;
+      for (int idx = threadIdx.x; idx < kNCodes * CH; idx += kK3Warps * 32) {
+        const int c = idx / CH, r = idx - c * CH;     // r = l*K + i
+        const int l = r / K, i = r - l * K;
+        prof_s[((c * (K / 2) + i / 2) * 32 + l) * 2 + (i & 1)] =
+            (uint32_t)__ldg(gprof + (int64_t)c * P.rows_padded + ch * CH + r);
       }
-      if (sidx + 1 < nslices) omask = start_mask(a.slices[P.slice_off + sidx + 1]);
-    }
-    if (len == 0) continue;
-    const bool any_mask = __any_sync(0xffffffffu, omask != 0);   // warp-uniform
-    // border tiles of chunk ch-1 are published by phase pph as tiles
-    // base_in .. base_in + ntile - 1 of its running count
-    const int base_in = (ch - 1 - pph) / PH * ntile;
-    uint32_t H[K], E[K];
+      __syncthreads();
+      if (!valid) continue;
+      // lane l's rows of this chunk are slice ch*32 + l: flush a half whose query changed;
+      // the start mask of the slice below applies to what this lane hands down
+      uint32_t omask = 0;
+      {
+        const int sidx = ch * 32 + lane;
+        const SliceInfo si = a.slices[P.slice_off + sidx];
+        if (si.q_lo != cq_lo) {
+          flush_half(cq_lo, lo16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
+          best = (best & 0xffff0000u) | (koff & 0xffffu);
+          cq_lo = si.q_lo;
+        }
+        if (si.q_hi != cq_hi) {
+          flush_half(cq_hi, hi16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
+          best = (best & 0x0000ffffu) | (koff & 0xffff0000u);
+          cq_hi = si.q_hi;
+        }
+        if (sidx + 1 < nslices) omask = start_mask(a.slices[P.slice_off + sidx + 1]);
+      }
+      done++;
+      if (len == 0) continue;
+      const bool any_mask = __any_sync(0xffffffffu, omask != 0);   // warp-uniform
+      uint32_t H[K], E[K];
 #pragma unroll
-    for (int i = 0; i < K; i++) { H[i] = koff; E[i] = koff; }
-    uint32_t hprev_top = koff;
-    uint32_t out_h[T], out_f[T], out_c[NW];
+      for (int i = 0; i < K; i++) { H[i] = koff; E[i] = koff; }
+      uint32_t hprev_top = koff;
+      uint32_t out_h[T], out_f[T], out_c[NW];
 #pragma unroll
-    for (int jj = 0; jj < T; jj++) { out_h[jj] = koff; out_f[jj] = koff; }
+      for (int jj = 0; jj < T; jj++) { out_h[jj] = koff; out_f[jj] = koff; }
 #pragma unroll
-    for (int q = 0; q < NW; q++) out_c[q] = padw;
-    // lane 0 streams the tile inputs (border row of the previous chunk, residue words)
-    // into a 3-deep per-warp shared-memory ring with cp.async, two tiles ahead
-    uint2 *bring = ring2 + warp * 3 * T;   // [3][T]
-    uint4 *wring = ring4 + warp * 3;       // [3] words of 16 residues
-    auto fetch = [&](int tt) {             // lane 0: inputs of tile tt into slot tt % 3
-      if (tt < ntile) {
-        const int sl = tt % 3;
-        if (ch > 0) {
-          if (PH > 1) {   // wait until the previous chunk's warp has published tile tt
-            while (*prog_in < base_in + tt + 1) {}
-            __threadfence_block();
+      for (int q = 0; q < NW; q++) out_c[q] = padw;
+      // lane 0 streams the tile inputs (border row of the previous chunk, residue words)
+      // into a 3-deep per-warp shared-memory ring with cp.async, two tiles ahead
+      uint2 *bring = ring2 + warp * 3 * T;   // [3][T]
+      uint4 *wring = ring4 + warp * 3;       // [3] words of 16 residues
+      auto fetch = [&](int tt) {             // lane 0: inputs of tile tt into slot tt % 3
+        if (tt < ntile) {
+          const int sl = tt % 3;
+          if (ch > 0) {
+#pragma unroll
+            for (int jj = 0; jj < T; jj += 2) cp_async16(&bring[sl * T + jj], &border[tt * T + jj]);
           }
-#pragma unroll
-          for (int jj = 0; jj < T; jj += 2) cp_async16(&bring[sl * T + jj], &border_in[tt * T + jj]);
+          if (tt % TPU == 0) cp_async16(&wring[(tt / TPU) % 3], &wp[(size_t)(tt / TPU) * kGroup]);
         }
-        if (tt % TPU == 0) cp_async16(&wring[(tt / TPU) % 3], &wp[(size_t)(tt / TPU) * kGroup]);
+      };
+      if (lane == 0) {
+        fetch(0);
+        asm volatile("cp.async.commit_group;" ::: "memory");
+        fetch(1);
+        cp_async_commit_wait1();   // tile 0 has landed
       }
-    };
-    if (lane == 0) {
-      fetch(0);
-      asm volatile("cp.async.commit_group;" ::: "memory");
-      fetch(1);
-      cp_async_commit_wait1();   // tile 0 has landed
-    }
-    __syncwarp();
-    const int steps = ntile + 31;
-    for (int t = 0; t < steps; t++) {
-      uint32_t in_h[T], in_f[T], in_c[NW];
-#pragma unroll
-      for (int jj = 0; jj < T; jj++) {
-        in_h[jj] = __shfl_up_sync(0xffffffffu, out_h[jj], 1);
-        in_f[jj] = __shfl_up_sync(0xffffffffu, out_f[jj], 1);
-      }
-#pragma unroll
-      for (int q = 0; q < NW; q++) in_c[q] = __shfl_up_sync(0xffffffffu, out_c[q], 1);
-      if (lane == 0 && t < ntile) {
-        const uint4 wv = wring[(t / TPU) % 3];
-        const int q0 = (t % TPU) * NW;
-#pragma unroll
-        for (int q = 0; q < NW; q++) {
-          const int k = q0 + q;
-          in_c[q] = k == 0 ? wv.x : k == 1 ? wv.y : k == 2 ? wv.z : wv.w;
-        }
-        const int sl = t % 3;
+      __syncwarp();
+      const int steps = ntile + 31;
+      for (int t = 0; t < steps; t++) {
+        uint32_t in_h[T], in_f[T], in_c[NW];
 #pragma unroll
         for (int jj = 0; jj < T; jj++) {
-          const uint2 v = ch > 0 ? bring[sl * T + jj] : make_uint2(koff, koff);
-          in_h[jj] = v.x;
-          in_f[jj] = v.y;
+          in_h[jj] = __shfl_up_sync(0xffffffffu, out_h[jj], 1);
+          in_f[jj] = __shfl_up_sync(0xffffffffu, out_f[jj], 1);
         }
-        fetch(t + 2);              // slot (t+2)%3 == (t-1)%3, consumed last step
-        cp_async_commit_wait1();   // tile t+1 has landed
-      }
-      const int tile = t - lane;
-      if (tile >= 0 && tile < ntile) {
-        const uint32_t *prc[T];
-        uint32_t hdc[T];
 #pragma unroll
-        for (int jj = 0; jj < T; jj++) {
-          const uint32_t c = (in_c[jj / 4] >> (8 * (jj % 4))) & 0xffu;
-          prc[jj] = prof_s + (c * (K / 2) * 32 + lane) * 2;
-          hdc[jj] = hprev_top;
-          out_f[jj] = in_f[jj];
-          hprev_top = in_h[jj];
-        }
-        dp_tile<K, T, 32, true, 64>(prc, H, E, hdc, out_f, out_h, best, na, nbeta, koff);
-        if (any_mask) {   // bit-select: omask is 0 except in a lane above a query start
+        for (int q = 0; q < NW; q++) in_c[q] = __shfl_up_sync(0xffffffffu, out_c[q], 1);
+        if (lane == 0 && t < ntile) {
+          const uint4 wv = wring[(t / TPU) % 3];
+          const int q0 = (t % TPU) * NW;
+#pragma unroll
+          for (int q = 0; q < NW; q++) {
+            const int k = q0 + q;
+            in_c[q] = k == 0 ? wv.x : k == 1 ? wv.y : k == 2 ? wv.z : wv.w;
+          }
+          const int sl = t % 3;
 #pragma unroll
           for (int jj = 0; jj < T; jj++) {
-            out_h[jj] = (out_h[jj] & ~omask) | (koff & omask);
-            out_f[jj] = (out_f[jj] & ~omask) | (koff & omask);
+            const uint2 v = ch > 0 ? bring[sl * T + jj] : make_uint2(koff, koff);
+            in_h[jj] = v.x;
+            in_f[jj] = v.y;
           }
+          fetch(t + 2);              // slot (t+2)%3 == (t-1)%3, consumed last step
+          cp_async_commit_wait1();   // tile t+1 has landed
         }
+        const int tile = t - lane;
+        if (tile >= 0 && tile < ntile) {
+          const uint32_t *prc[T];
+          uint32_t hdc[T];
 #pragma unroll
-        for (int q = 0; q < NW; q++) out_c[q] = in_c[q];
-        if (lane == 31 && ch < nch - 1) {
+          for (int jj = 0; jj < T; jj++) {
+            const uint32_t c = (in_c[jj / 4] >> (8 * (jj % 4))) & 0xffu;
+            prc[jj] = prof_s + (c * (K / 2) * 32 + lane) * 2;
+            hdc[jj] = hprev_top;
+            out_f[jj] = in_f[jj];
+            hprev_top = in_h[jj];
+          }
+          dp_tile<K, T, 32, true, 64>(prc, H, E, hdc, out_f, out_h, best, na, nbeta, koff);
+          if (any_mask) {   // bit-select: omask is 0 except in a lane above a query start
 #pragma unroll
-          for (int jj = 0; jj < T; jj++) border_out[tile * T + jj] = make_uint2(out_h[jj], out_f[jj]);
-          if (PH > 1) {   // publish: the border stores are ordered before the counter
-            __threadfence_block();
-            *(volatile int *)&prog_s[warp] = ++published;
+            for (int jj = 0; jj < T; jj++) {
+              out_h[jj] = (out_h[jj] & ~omask) | (koff & omask);
+              out_f[jj] = (out_f[jj] & ~omask) | (koff & omask);
+            }
+          }
+#pragma unroll
+          for (int q = 0; q < NW; q++) out_c[q] = in_c[q];
+          if (lane == 31 && ch < nch - 1) {
+#pragma unroll
+            for (int jj = 0; jj < T; jj++) border[tile * T + jj] = make_uint2(out_h[jj], out_f[jj]);
           }
         }
       }
+      if (lane == 0) asm volatile("cp.async.wait_all;" ::: "memory");
+    }
+    if (valid && !aborted) {   // every lane flushes what it holds
+      flush_half(cq_lo, lo16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
+      flush_half(cq_hi, hi16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
     }
   }
-  if (valid) {   // every lane flushes what it holds
-    flush_half(cq_lo, lo16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
-    flush_half(cq_hi, hi16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
-  }
+  if (a.progress && lane == 0 && done > 0) atomicAdd(a.progress, done);
 }
 
-// K3 tile width (tuning; SW_K3_T): 8 columns per lane step (default) or 4.  Chunk phases
-// (SW_K3_PHASES): 1 (default) or 2 -- measured slower on C4 (-2.7 %) and C5 (-11 %, also at
-// 1/8 of its database): with 16 warps per SM the SM is already busy, and the phase
-// barriers and the consumer's wait at each chunk start only add idle time.
+// K3 tile width (tuning; SW_K3_T): 8 columns per lane step (default) or 4.
 static int k3_tile() {
   static const int v = [] { const char *e = getenv("SW_K3_T"); return (e && atoi(e) == 4) ? 4 : 8; }();
   return v;
 }
-int k3_phases() {
-  static const int v = [] { const char *e = getenv("SW_K3_PHASES"); return (e && atoi(e) == 2) ? 2 : 1; }();
+template <int T>
+static size_t k3_smem() {
+  return sizeof(uint32_t) * kNCodes * kK3Rows * 32 + sizeof(uint4) * kK3Warps * 3 +
+         sizeof(uint2) * kK3Warps * 3 * T;
+}
+template <int T>
+static void k3_go(const K3Args &a, int n, int max_blocks, cudaStream_t st) {
+  const size_t smem = k3_smem<T>();
+  const int blocks = std::min((n + kK3Warps - 1) / kK3Warps, std::max(1, max_blocks));
+  cudaFuncSetAttribute(k3_kernel<kK3Rows, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  k3_kernel<kK3Rows, T><<<blocks, kK3Warps * 32, smem, st>>>(a);
+}
+int k3_blocks_per_sm() {
+  static std::once_flag once;
+  static int v = 4;
+  std::call_once(once, [] {
+    int n = 0;
+    const size_t smem = k3_tile() == 4 ? k3_smem<4>() : k3_smem<8>();
+    auto fn = k3_tile() == 4 ? k3_kernel<kK3Rows, 4> : k3_kernel<kK3Rows, 8>;
+    cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, kK3Warps * 32, smem) == cudaSuccess && n > 0) v = n;
+  });
   return v;
 }
-template <int T, int PH>
-static void k3_go(const K3Args &a, int n, cudaStream_t st) {
-  const size_t smem = sizeof(uint32_t) * PH * kNCodes * kK3Rows * 32 + sizeof(uint4) * kK3Warps * PH * 3 +
-                      sizeof(uint2) * kK3Warps * PH * 3 * T;
-  const int blocks = (n + kK3Warps - 1) / kK3Warps;
-  cudaFuncSetAttribute(k3_kernel<kK3Rows, T, PH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  k3_kernel<kK3Rows, T, PH><<<blocks, kK3Warps * PH * 32, smem, st>>>(a);
-}
-void launch_k3(const K3Args &a, int, cudaStream_t st) {
+// n_sm_cap > 0 caps the grid to that many SMs' worth of resident blocks (slower-PE
+// emulation); otherwise one block per kK3Warps sequences
+void launch_k3(const K3Args &a, int, cudaStream_t st, int n_sm_cap) {
   const int n = a.l1 - a.l0;
   if (n <= 0) return;
-  const bool two = k3_phases() == 2;
-  if (k3_tile() == 4) { if (two) k3_go<4, 2>(a, n, st); else k3_go<4, 1>(a, n, st); }
-  else { if (two) k3_go<8, 2>(a, n, st); else k3_go<8, 1>(a, n, st); }
+  const int maxb = n_sm_cap > 0 ? n_sm_cap * k3_blocks_per_sm() : INT32_MAX;
+  if (k3_tile() == 4) k3_go<4>(a, n, maxb, st);
+  else k3_go<8>(a, n, maxb, st);
+}
+
+// ------------------------------------------------------------------------------------
+// Local load (P24 §V.C "introduced local load ... after 60 seconds", the superpi analogue
+// on a GPU): one block per SM holding all of its shared memory, so no DP block can share
+// the SM, spinning on integer work until the host raises *stop (or max_ns elapses: the
+// kernel can never outlive a lost host).  Launched on its own high-priority stream.
+// ------------------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t globaltimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__global__ void __launch_bounds__(256) noise_kernel(const volatile int32_t *stop, uint64_t max_ns,
+                                                    uint32_t *sink) {
+  extern __shared__ uint32_t noise_s[];
+  const uint64_t t0 = globaltimer();
+  uint32_t x = threadIdx.x * 2654435761u + blockIdx.x;
+  while (true) {
+#pragma unroll 8
+    for (int k = 0; k < 4096; k++) x = __vimax3_s16x2(x * 1664525u + 1013904223u, x, k);
+    if (*stop != 0 || globaltimer() - t0 > max_ns) break;
+  }
+  noise_s[threadIdx.x] = x;
+  if (x == 0x9e3779b9u) sink[blockIdx.x] = noise_s[(threadIdx.x + 1) & 255];
+}
+size_t noise_smem() {
+  int dev = 0, v = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+  return v > 0 ? (size_t)v : 227 * 1024;
+}
+void launch_noise(const int32_t *stop, int n_blocks, uint64_t max_ns, uint32_t *sink, cudaStream_t st) {
+  if (n_blocks <= 0) return;
+  const size_t smem = noise_smem();
+  cudaFuncSetAttribute(noise_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  noise_kernel<<<n_blocks, 256, smem, st>>>(stop, max_ns, sink);
 }
 
 // ------------------------------------------------------------------------------------
@@ -1024,33 +1058,54 @@ __global__ void fill_kernel(int32_t *p, int64_t n, int32_t v) {
 void launch_fill(int32_t *p, int64_t n, int32_t v, cudaStream_t st) {
   if (n > 0) fill_kernel<<<592, 256, 0, st>>>(p, n, v);
 }
-__global__ void max_merge_kernel(int32_t *dst, const int32_t *src, int64_t n) {
-  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x)
-    dst[k] = max(dst[k], src[k]);
+// ------------------------------------------------------------------------------------
+// Segments of committed units (the cross-GPU data plane): a segment is query
+// q x sorted sequences [s0, s1) of one committed unit; its pairs sit at scores[q][perm[s]]
+// (original order) and at compact[off + s - s0] in a dense per-worker buffer.
+//   mode 0: gather  matrix -> compact      (committing GPU, before the peer copy)
+//   mode 1: scatter compact -> matrix      (device 0, after the peer copy)
+//   mode 2: copy    matrix -> matrix       (multi-process: this rank's committed pairs only)
+// ------------------------------------------------------------------------------------
+__global__ void seg_copy_kernel(const int32_t *__restrict__ src, int32_t *__restrict__ dst, int64_t ndb,
+                                const int32_t *__restrict__ perm, const SegInfo *__restrict__ segs, int mode) {
+  const SegInfo g = segs[blockIdx.x];
+  const int64_t row = (int64_t)g.q * ndb;
+  for (int s = g.s0 + threadIdx.x; s < g.s1; s += blockDim.x) {
+    const int64_t m = row + perm[s];
+    const int64_t c = g.off + (s - g.s0);
+    if (mode == 0) dst[c] = src[m];
+    else if (mode == 1) dst[m] = src[c];
+    else dst[m] = src[m];
+  }
 }
-void launch_max_merge(int32_t *dst, const int32_t *src, int64_t n, cudaStream_t st) {
-  if (n > 0) max_merge_kernel<<<592, 256, 0, st>>>(dst, src, n);
+void launch_seg_copy(const int32_t *src, int32_t *dst, int64_t ndb, const int32_t *perm, const SegInfo *segs,
+                     int nseg, int mode, cudaStream_t st) {
+  if (nseg > 0) seg_copy_kernel<<<nseg, 256, 0, st>>>(src, dst, ndb, perm, segs, mode);
 }
 
 // ------------------------------------------------------------------------------------
-// K5: per-query top-k under (score desc, db_index asc); entries < 0 are ignored.
-// One block per query: each thread keeps its own sorted top-k of 64-bit keys
-// (score << 32 | ~index) over a strided slice, then warps and finally warp 0 merge the
-// lists k rounds at a time with shuffles.
+// K5: top-k under (score desc, db_index asc) -- R13.  Keys are score << 32 | ~index (0 =
+// empty), so one unsigned comparison orders both fields.  A block keeps one descending
+// list per thread over a strided slice of its candidates (an insertion per candidate
+// above the thread's k-th key, equal keys kept once), then warps merge their lanes' lists
+// with shuffles and warp 0 merges the warps' lists.
+//   K5u  unit_topk_kernel:  one block per query of a committed unit's pack, candidates =
+//        that query's pairs in the unit (scores[q][perm[s]], s in [s0, s1)), on the unit's
+//        stream right after it (and after the int32 re-run of what it saturated);
+//   K5m  merge_topk_kernel: one block per query, candidates = the hits of several lists
+//        (a worker's committed units, then the workers / ranks): the paper's "merges" (P16).
 // ------------------------------------------------------------------------------------
 constexpr int kTopkMax = 64;
-__device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
-  uint32_t lo = __shfl_sync(0xffffffffu, (uint32_t)v, src);
-  uint32_t hi = __shfl_sync(0xffffffffu, (uint32_t)(v >> 32), src);
-  return ((uint64_t)hi << 32) | lo;
-}
 __device__ __forceinline__ uint64_t xor64(uint64_t v, int o) {
   uint32_t lo = __shfl_xor_sync(0xffffffffu, (uint32_t)v, o);
   uint32_t hi = __shfl_xor_sync(0xffffffffu, (uint32_t)(v >> 32), o);
   return ((uint64_t)hi << 32) | lo;
 }
-// warp merge: each lane holds a descending list (len k, 0 = empty); returns in lane 0..
-// the merged top-k written to out[0..k)
+__device__ __forceinline__ uint64_t hit_key(int score, int idx) {
+  return (idx < 0 || score < 0) ? 0ull : (((uint64_t)(uint32_t)score << 32) | (uint32_t)(~(uint32_t)idx));
+}
+// warp merge: each lane holds a descending list (len k, 0 = empty); lane 0 gets the merged
+// top-k in out[0..k).  A key held by several lanes is emitted once.
 __device__ void warp_merge(const uint64_t *list, int k, uint64_t *out) {
   const int lane = threadIdx.x & 31;
   int head = 0;
@@ -1059,29 +1114,24 @@ __device__ void warp_merge(const uint64_t *list, int k, uint64_t *out) {
     uint64_t m = mine;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) { uint64_t v = xor64(m, o); m = v > m ? v : m; }
-    // keys are unique (index in the low bits) except 0 = empty
     if (m != 0ull && mine == m) head++;
     if (lane == 0) out[r] = m;
   }
 }
-
-__global__ void __launch_bounds__(1024) topk_kernel(const int32_t *__restrict__ scores, int64_t ndb,
-                                                    int k, int2 *__restrict__ hits) {
-  __shared__ uint64_t wl[32][kTopkMax];
-  const int q = blockIdx.x, lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int32_t *row = scores + (int64_t)q * ndb;
+template <int NT, class KeyOf>
+__device__ void block_topk(KeyOf key_of, int64_t n, int k, int2 *out) {
+  __shared__ uint64_t wl[NT / 32][kTopkMax];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   uint64_t list[kTopkMax];
-#pragma unroll
-  for (int i = 0; i < kTopkMax; i++) list[i] = 0ull;
+  for (int i = 0; i < k; i++) list[i] = 0ull;
   uint64_t kth = 0ull;
-  for (int64_t d = threadIdx.x; d < ndb; d += blockDim.x) {
-    const int32_t sc = row[d];
-    if (sc < 0) continue;
-    const uint64_t key = ((uint64_t)(uint32_t)sc << 32) | (uint32_t)(~(uint32_t)d);
+  for (int64_t d = threadIdx.x; d < n; d += NT) {
+    const uint64_t key = key_of(d);
     if (key <= kth) continue;
-    // insert into the descending list
     int pos = k - 1;
-    while (pos > 0 && list[pos - 1] < key) { list[pos] = list[pos - 1]; pos--; }
+    while (pos > 0 && list[pos - 1] < key) pos--;
+    if (pos > 0 && list[pos - 1] == key) continue;   // already held
+    for (int i = k - 1; i > pos; i--) list[i] = list[i - 1];
     list[pos] = key;
     kth = list[k - 1];
   }
@@ -1092,20 +1142,60 @@ __global__ void __launch_bounds__(1024) topk_kernel(const int32_t *__restrict__ 
   __syncthreads();
   if (warp == 0) {
     uint64_t l2[kTopkMax];
-    for (int i = 0; i < k; i++) l2[i] = wl[lane][i];
+    for (int i = 0; i < k; i++) l2[i] = lane < NT / 32 ? wl[lane][i] : 0ull;
     uint64_t fin[kTopkMax];
     warp_merge(l2, k, fin);
     if (lane == 0)
       for (int i = 0; i < k; i++) {
         const uint64_t v = fin[i];
-        hits[(int64_t)q * k + i] = v ? make_int2((int)(v >> 32), (int)(~(uint32_t)v)) : make_int2(0, -1);
+        out[i] = v ? make_int2((int)(v >> 32), (int)(~(uint32_t)v)) : make_int2(0, -1);
       }
   }
 }
 
+__global__ void __launch_bounds__(1024) topk_kernel(const int32_t *__restrict__ scores, int64_t ndb,
+                                                    int k, int2 *__restrict__ hits) {
+  const int32_t *row = scores + (int64_t)blockIdx.x * ndb;
+  block_topk<1024>([&](int64_t d) { return hit_key(row[d], (int)d); }, ndb, k, hits + (int64_t)blockIdx.x * k);
+}
 void launch_topk(const int32_t *scores, int32_t nq, int64_t ndb, int32_t k, int2 *hits, cudaStream_t st) {
   if (nq <= 0 || k <= 0) return;
   topk_kernel<<<nq, 1024, 0, st>>>(scores, ndb, k, hits);
+}
+
+__global__ void __launch_bounds__(256) unit_topk_kernel(const int32_t *__restrict__ scores, int64_t ndb,
+                                                        const int32_t *__restrict__ perm, int32_t s0, int32_t s1,
+                                                        const int32_t *__restrict__ queries, int k,
+                                                        int2 *__restrict__ out) {
+  const int q = queries[blockIdx.x];
+  const int32_t *row = scores + (int64_t)q * ndb;
+  block_topk<256>([&](int64_t d) {
+        const int o = perm[s0 + (int)d];
+        return hit_key(row[o], o);
+      }, (int64_t)(s1 - s0), k, out + (int64_t)blockIdx.x * k);
+}
+void launch_unit_topk(const int32_t *scores, int64_t ndb, const int32_t *perm, int32_t s0, int32_t s1,
+                      const int32_t *queries, int nqp, int k, int2 *out, cudaStream_t st) {
+  if (nqp <= 0 || k <= 0) return;
+  unit_topk_kernel<<<nqp, 256, 0, st>>>(scores, ndb, perm, s0, s1, queries, k, out);
+}
+
+__global__ void __launch_bounds__(256) merge_topk_kernel(const int2 *__restrict__ lists, int k_in,
+                                                         const int32_t *__restrict__ list_off,
+                                                         const int32_t *__restrict__ list_idx, int k,
+                                                         int2 *__restrict__ out) {
+  const int q = blockIdx.x;
+  const int32_t j0 = list_off[q], nl = list_off[q + 1] - j0;
+  block_topk<256>([&](int64_t d) {
+        const int l = (int)(d / k_in), r = (int)(d - (int64_t)l * k_in);
+        const int2 h = lists[(int64_t)list_idx[j0 + l] * k_in + r];
+        return hit_key(h.x, h.y);
+      }, (int64_t)nl * k_in, k, out + (int64_t)q * k);
+}
+void launch_merge_topk(const int2 *lists, int k_in, const int32_t *list_off, const int32_t *list_idx, int nq,
+                       int k, int2 *out, cudaStream_t st) {
+  if (nq <= 0 || k <= 0) return;
+  merge_topk_kernel<<<nq, 256, 0, st>>>(lists, k_in, list_off, list_idx, k, out);
 }
 
 }  // namespace sw

@@ -18,10 +18,11 @@ namespace sw {
 
 namespace {
 enum Op : int32_t { kHello = 0, kRequest = 1, kReport = 2, kComplete = 3, kAbandon = 4,
-                    kFinishedMap = 5, kDone = 6, kCounters = 7, kStart = 8 };
+                    kFinishedMap = 5, kDone = 6, kCounters = 7, kStart = 8, kRequestWait = 9 };
 struct Msg {
   int32_t op, worker, unit, cap;
-  double t, cells, sec;
+  double t, cells, sec;   // kRequestWait: sec = timeout
+  uint64_t hash;          // kHello: the slave's plan hash
 };
 struct RepHdr {
   int32_t rc, nextra;
@@ -58,8 +59,9 @@ void nodelay(int fd) {
 MasterServer::~MasterServer() { stop(); }
 
 void MasterServer::start(int port, int world, int32_t n_units, const int64_t *unit_cells,
-                         int32_t policy, int32_t wa, int32_t omega) {
+                         int32_t policy, int32_t wa, int32_t omega, uint64_t plan_hash) {
   world_ = world;
+  plan_hash_ = plan_hash;
   sched_ = sw_sched_create(world, n_units, unit_cells, policy, wa, omega);
   if (!sched_ && n_units > 0) throw Error(SW_EINVAL, "master: scheduler creation failed");
   listen_fd_ = ::socket(AF_INET, SOCK_STREAM, 0);
@@ -91,18 +93,32 @@ void MasterServer::serve(int fd) {
   Msg m;
   std::vector<int32_t> buf;
   int32_t worker = -1;
+  bool left = false;
   while (recv_all(fd, &m, sizeof(m))) {
     RepHdr h{0, 0};
     buf.clear();
     const double t = now_s();  // the master's clock
     switch (m.op) {
-      case kHello: worker = m.worker; registered_.fetch_add(1); break;
-      case kRequest: {
+      case kHello:
+        // a slave whose unit table differs from rank 0's would execute other (pack, group)
+        // ranges under the same unit ids: refuse it
+        if (m.hash != plan_hash_) { h.rc = -1; break; }
+        worker = m.worker;
+        registered_.fetch_add(1);
+        break;
+      case kRequest:
+      case kRequestWait: {
         // "the master process starts the execution and waits for the slaves to register"
         // (P16 §IV): no task is handed out before every slave has registered
-        if (registered_.load() < world_) { h.rc = 0; break; }
+        if (registered_.load() < world_) {
+          if (m.op == kRequestWait) std::this_thread::sleep_for(std::chrono::milliseconds(1));
+          h.rc = 0;
+          break;
+        }
         buf.resize(std::max(1, m.cap));
-        h.rc = sched_ ? sw_sched_request(sched_, worker, t, buf.data(), m.cap) : -1;
+        if (!sched_) h.rc = -1;
+        else if (m.op == kRequest) h.rc = sw_sched_request(sched_, worker, t, buf.data(), m.cap);
+        else h.rc = sw_sched_request_wait(sched_, worker, t, buf.data(), m.cap, m.sec);
         buf.resize(h.rc > 0 ? h.rc : 0);
         break;
       }
@@ -118,16 +134,23 @@ void MasterServer::serve(int fd) {
         break;
       }
       case kCounters:
-        buf.assign(2, 0);
-        if (sched_) { buf[0] = (int32_t)sw_sched_counter(sched_, 0); buf[1] = (int32_t)sw_sched_counter(sched_, 1); }
+        buf.assign(3, 0);
+        if (sched_)
+          for (int k = 0; k < 3; k++) buf[k] = (int32_t)sw_sched_counter(sched_, k == 2 ? 3 : k);
         break;
-      case kDone: done_.fetch_add(1); break;
+      case kDone: done_.fetch_add(1); left = true; break;
       default: break;
     }
     h.nextra = (int32_t)buf.size();
     if (!send_all(fd, &h, sizeof(h)) || (h.nextra && !send_all(fd, buf.data(), sizeof(int32_t) * buf.size())))
       break;
-    if (m.op == kDone) break;
+    if (m.op == kDone || (m.op == kHello && h.rc < 0)) break;
+  }
+  if (!left) {
+    // the connection closed without DONE: the slave is gone; its unfinished tasks go back
+    // to READY so the others can still finish the search (and stop() does not wait for it)
+    if (sched_ && worker >= 0) sw_sched_fail_worker(sched_, worker, now_s());
+    done_.fetch_add(1);
   }
   ::close(fd);
 }
@@ -142,14 +165,18 @@ void MasterServer::stop() {
   std::lock_guard<std::mutex> g(mu_);
   for (auto &t : conns_) if (t.joinable()) t.join();
   conns_.clear();
-  if (sched_) { sw_sched_destroy(sched_); sched_ = nullptr; }
+  if (sched_) {
+    final_log_ = sw_sched_log_json(sched_);
+    sw_sched_destroy(sched_);
+    sched_ = nullptr;
+  }
 }
 
 SchedClient::~SchedClient() {
   if (fd_ >= 0) ::close(fd_);
 }
 
-void SchedClient::connect(const char *host, int port, int rank, double timeout_s) {
+void SchedClient::connect(const char *host, int port, int rank, double timeout_s, uint64_t plan_hash) {
   rank_ = rank;
   const double t0 = now_s();
   addrinfo hints{}, *res = nullptr;
@@ -172,12 +199,17 @@ void SchedClient::connect(const char *host, int port, int rank, double timeout_s
   freeaddrinfo(res);
   nodelay(fd_);
   // "the slaves can register themselves in the master" (P16 §IV)
-  call(kHello, 0, 0, 0, 0, 0, nullptr);
+  if (call(kHello, 0, 0, 0, 0, 0, nullptr, plan_hash) < 0) {
+    ::close(fd_);
+    fd_ = -1;
+    throw Error(SW_ENET, "slave: the master refused rank " + std::to_string(rank) +
+                             ": its unit table differs from rank 0's (different inputs or options)");
+  }
 }
 
 int32_t SchedClient::call(int32_t op, int32_t unit, int32_t cap, double t, double cells, double sec,
-                          std::vector<int32_t> *extra) {
-  Msg m{op, rank_, unit, cap, t, cells, sec};
+                          std::vector<int32_t> *extra, uint64_t hash) {
+  Msg m{op, rank_, unit, cap, t, cells, sec, hash};
   RepHdr h;
   if (!send_all(fd_, &m, sizeof(m)) || !recv_all(fd_, &h, sizeof(h)))
     throw Error(SW_ENET, "slave: lost the connection to the master");
@@ -194,6 +226,18 @@ int32_t SchedClient::request(double t, int32_t *out, int32_t cap) {
   const int32_t rc = call(kRequest, 0, cap, t, 0, 0, &e);
   for (int32_t k = 0; k < rc && k < (int32_t)e.size(); k++) out[k] = e[k];
   return rc;
+}
+int32_t SchedClient::request_wait(double t, int32_t *out, int32_t cap, double timeout_s) {
+  std::vector<int32_t> e;
+  const int32_t rc = call(kRequestWait, 0, cap, t, 0, timeout_s, &e);
+  for (int32_t k = 0; k < rc && k < (int32_t)e.size(); k++) out[k] = e[k];
+  return rc;
+}
+int64_t SchedClient::counter(int32_t which) {
+  std::vector<int32_t> e;
+  call(kCounters, 0, 0, 0, 0, 0, &e);
+  if (e.size() < 3) return 0;
+  return which == 0 ? e[0] : which == 1 ? e[1] : which == 3 ? e[2] : 0;
 }
 void SchedClient::report(double t, double cells, double sec) { call(kReport, 0, 0, t, cells, sec, nullptr); }
 int32_t SchedClient::complete(int32_t unit, double t) { return call(kComplete, unit, 0, t, 0, 0, nullptr); }
@@ -212,7 +256,7 @@ int32_t SchedClient::is_finished(int32_t unit) {
 void SchedClient::done() {
   std::vector<int32_t> e;
   call(kCounters, 0, 0, 0, 0, 0, &e);
-  if (e.size() >= 2) { req_ = e[0]; wa_ = e[1]; }
+  if (e.size() >= 3) { req_ = e[0]; wa_ = e[1]; grants_ = e[2]; }
   call(kDone, 0, 0, 0, 0, 0, nullptr);
   ::close(fd_);
   fd_ = -1;
@@ -229,10 +273,10 @@ namespace sw { void set_last_error(const std::string &m); }
 extern "C" {
 
 sw_master *sw_master_start(int32_t port, int32_t world, int32_t n_units, const int64_t *unit_cells,
-                           int32_t policy, int32_t wa, int32_t omega) {
+                           int32_t policy, int32_t wa, int32_t omega, uint64_t plan_hash) {
   auto *m = new sw_master();
   try {
-    m->s.start(port, world, n_units, unit_cells, policy, wa, omega);
+    m->s.start(port, world, n_units, unit_cells, policy, wa, omega, plan_hash);
     return m;
   } catch (const std::exception &e) {
     sw::set_last_error(e.what());
@@ -245,10 +289,11 @@ void sw_master_stop(sw_master *m) {
   m->s.stop();
   delete m;
 }
-sw_slave *sw_slave_connect(const char *host, int32_t port, int32_t rank, double timeout_s) {
+sw_slave *sw_slave_connect(const char *host, int32_t port, int32_t rank, double timeout_s,
+                           uint64_t plan_hash) {
   auto *c = new sw_slave();
   try {
-    c->c.connect(host, port, rank, timeout_s);
+    c->c.connect(host, port, rank, timeout_s, plan_hash);
     return c;
   } catch (const std::exception &e) {
     sw::set_last_error(e.what());
@@ -262,6 +307,12 @@ static double clk() {
 }
 int32_t sw_slave_request(sw_slave *c, int32_t *out, int32_t cap) {
   try { return c->c.request(clk(), out, cap); } catch (const std::exception &e) { sw::set_last_error(e.what()); return -2; }
+}
+int32_t sw_slave_request_wait(sw_slave *c, int32_t *out, int32_t cap, double timeout_s) {
+  try { return c->c.request_wait(clk(), out, cap, timeout_s); } catch (const std::exception &e) { sw::set_last_error(e.what()); return -2; }
+}
+int64_t sw_slave_counter(sw_slave *c, int32_t which) {
+  try { return c->c.counter(which); } catch (const std::exception &e) { sw::set_last_error(e.what()); return -2; }
 }
 void sw_slave_report(sw_slave *c, double cells, double seconds) {
   try { c->c.report(clk(), cells, seconds); } catch (const std::exception &e) { sw::set_last_error(e.what()); }

@@ -97,7 +97,8 @@ struct K1Args {
   int32_t thresh;                    // overflow threshold on best~ (offset repr)
   int2 *ovf; int32_t *ovf_count; int32_t ovf_cap; uint32_t *ovf_bits;
   uint2 *border; int32_t border_slot_cols; int32_t slots_per_sm; int32_t *slot_busy;
-  const volatile int32_t *abort_flag;
+  const volatile int32_t *abort_flag; // WA cancellation flag of the unit (polled in the loop)
+  int32_t *progress;                 // unit's counter: groups completed (atomicAdd per block)
   uint32_t na, nb;                   // packed -alpha, -beta
 };
 struct K3Args {   // sequences [l0,l1) in sorted order (the long groups)
@@ -107,8 +108,9 @@ struct K3Args {   // sequences [l0,l1) in sorted order (the long groups)
   int32_t *scores; int64_t ndb;
   int32_t thresh;
   int2 *ovf; int32_t *ovf_count; int32_t ovf_cap; uint32_t *ovf_bits;
-  uint2 *border; int64_t border_stride;   // per (sequence, phase) border (>= max long len)
-  const volatile int32_t *abort_flag;
+  uint2 *border; int64_t border_stride;   // per sequence border row (>= max long len)
+  const volatile int32_t *abort_flag;     // WA cancellation flag (polled at chunk starts)
+  int32_t *progress;                      // unit's counter: (sequence, chunk) pairs completed
   uint32_t na, nb;
 };
 constexpr int kMaxStreams = 64;    // sw_opts.streams_per_device limit
@@ -147,14 +149,25 @@ void launch_profile(const uint8_t *qcodes, const int64_t *qoff, const QueryPair 
                     cudaStream_t st);
 void launch_k1(const K1Args &a, int n_groups, int min_cols, int rows_padded, cudaStream_t st,
                int n_sm);
-void launch_k3(const K3Args &a, int rows_padded, cudaStream_t st);
+void launch_k3(const K3Args &a, int rows_padded, cudaStream_t st, int n_sm_cap);
 void launch_k2(const K2Args &a, int blocks, cudaStream_t st);
 void launch_fill(int32_t *p, int64_t n, int32_t v, cudaStream_t st);
-void launch_max_merge(int32_t *dst, const int32_t *src, int64_t n, cudaStream_t st);
+// committed-unit segments (cross-GPU data plane): query q x sorted sequences [s0, s1)
+struct SegInfo { int32_t q, s0, s1, pad_; int64_t off; };
+void launch_seg_copy(const int32_t *src, int32_t *dst, int64_t ndb, const int32_t *perm, const SegInfo *segs,
+                     int nseg, int mode, cudaStream_t st);   // 0 gather, 1 scatter, 2 copy
 void launch_topk(const int32_t *scores, int32_t nq, int64_t ndb, int32_t k, int2 *hits,
                  cudaStream_t st);
+// K5u: top-k of one committed unit, per query of its pack -> out[nqp][k]
+void launch_unit_topk(const int32_t *scores, int64_t ndb, const int32_t *perm, int32_t s0, int32_t s1,
+                      const int32_t *queries, int nqp, int k, int2 *out, cudaStream_t st);
+// K5m: per query q, merge lists list_idx[list_off[q] .. list_off[q+1]) (k_in hits each)
+void launch_merge_topk(const int2 *lists, int k_in, const int32_t *list_off, const int32_t *list_idx, int nq,
+                       int k, int2 *out, cudaStream_t st);
 int k1_blocks_per_sm();
-int k3_phases();   // warps per long pair (chunk phases of K3)
+int k3_blocks_per_sm();
+// local-load kernel: n_blocks SM-filling blocks spinning until *stop != 0 (or max_ns)
+void launch_noise(const int32_t *stop, int n_blocks, uint64_t max_ns, uint32_t *sink, cudaStream_t st);
 int k1_band_rows();   // rows per K1 band (W*K of the selected variant)
 
 // ---- host packing (pack.cpp) ----------------------------------------------------------------

@@ -128,46 +128,104 @@ def test_tcp_master_slaves_commit_each_task_once(wa):
     assert sorted(committed) == list(range(len(cells)))
 
 
-def _gloo_merge(rank, world, port, q):
+def _gloo_gather(rank, world, port, q):
+    """The multi-process data plane on CPU (gloo, world 2): each rank contributes its top-k
+    lists over its committed units; gather_hits stacks every rank's [nq, k, 2] block."""
     import torch
     import torch.distributed as dist
     from paper_conf_ipps_mendoncam13_b200 import dist as swdist
     dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
-    full = torch.arange(3 * 10, dtype=torch.int32).reshape(3, 10) % 7
-    part = torch.full_like(full, -1)
-    cols = [c for c in range(10) if c % world == rank] + [4]   # column 4 computed by both (WA)
-    part[:, cols] = full[:, cols]
-    swdist.merge_scores(part)
-    ok_scores = bool((part == full).all()) if rank == 0 else True
-    # hits: each rank's local top-3 (score desc, index asc) over its columns
-    def local_topk(t, k):
-        out_s = torch.zeros((t.shape[0], k), dtype=torch.int32)
-        out_i = torch.full((t.shape[0], k), -1, dtype=torch.int32)
-        for qi in range(t.shape[0]):
-            c = sorted([(int(v), i) for i, v in enumerate(t[qi].tolist()) if v >= 0], key=lambda x: (-x[0], x[1]))[:k]
-            for r, (v, i) in enumerate(c):
-                out_s[qi, r], out_i[qi, r] = v, i
-        return out_s, out_i
-    p2 = torch.full_like(full, -1)
-    p2[:, cols] = full[:, cols]
-    ls, li = local_topk(p2, 3)
-    gs, gi = swdist.merge_hits(ls, li, 3)
-    es, ei = local_topk(full, 3)
-    q.put((rank, ok_scores, bool((gs == es).all() and (gi == ei).all())))
+    nq, k = 3, 4
+    local = torch.full((nq, k, 2), -1, dtype=torch.int32)
+    local[..., 0] = 10 * rank + torch.arange(k, dtype=torch.int32).flip(0)
+    local[..., 1] = 100 * rank + torch.arange(k, dtype=torch.int32)
+    allh = swdist.gather_hits(local)
+    ok = allh.shape == (world, nq, k, 2) and all(
+        bool((allh[r][..., 1] == 100 * r + torch.arange(k, dtype=torch.int32)).all()) for r in range(world))
+    q.put((rank, ok))
     dist.destroy_process_group()
 
 
-def test_gloo_world2_merge():
+def test_gloo_world2_gather_hits():
     port = _free_port()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_gloo_merge, args=(r, 2, port, q)) for r in range(2)]
+    procs = [ctx.Process(target=_gloo_gather, args=(r, 2, port, q)) for r in range(2)]
     for p in procs:
         p.start()
-    out = [q.get(timeout=120) for _ in procs]
+    out = [q.get(timeout=60) for _ in procs]
     for p in procs:
-        p.join(timeout=60)
-    assert all(o[1] and o[2] for o in out), out
+        p.join(timeout=30)
+    assert all(o[1] for o in out), out
+
+
+def test_master_refuses_a_rank_with_another_unit_table():
+    """ranks must agree on the unit table (its hash travels in the hello)."""
+    port = _free_port()
+    m = Master(port, 2, [5, 5, 5], plan_hash=1234)
+    ok = Slave("127.0.0.1", port, 0, timeout=10, plan_hash=1234)
+    with pytest.raises(pkg.SwError):
+        Slave("127.0.0.1", port, 1, timeout=10, plan_hash=999)
+    ok.done()
+    m.stop()
+
+
+def _quitter(port, q):
+    """A slave that takes one task and disappears without completing it."""
+    sl = Slave("127.0.0.1", port, 1)
+    got = []
+    while not got:
+        got = sl.request()
+    q.put(got)
+    os._exit(0)   # connection closes without DONE
+
+
+def test_lost_slave_tasks_go_back_to_ready_wa_off():
+    """A slave whose connection closes without DONE is failed: its unfinished tasks return to
+    READY, so the other slave completes the search even with workload adjustment off."""
+    port = _free_port()
+    cells = [10] * 6
+    m = Master(port, 2, cells, policy="ss", wa=False)
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    p = ctx.Process(target=_quitter, args=(port, q))
+    p.start()
+    sl = Slave("127.0.0.1", port, 0)
+    done = []
+    t_end = time.time() + 60
+    taken = None
+    while time.time() < t_end:
+        got = sl.request_wait(0.05)
+        if got is None:
+            break
+        for u in got:
+            sl.report(10, 0.01)
+            done.append((u, sl.complete(u)))
+        if taken is None and not q.empty():
+            taken = q.get()
+    p.join(timeout=30)
+    sl.done()
+    m.stop()
+    assert sorted(u for u, c in done if c) == list(range(6))
+
+
+def test_request_wait_is_one_message():
+    """An idle worker's request waits at the master: many idle periods cost few messages
+    (SS/PSS 'master interactions' count messages, not polls)."""
+    S = pkg.Scheduler(2, [100, 100], policy="ss", wa=False)
+    assert S.request(0, 0.0) == [0] and S.request(1, 0.0) == [1]
+    t = time.perf_counter()
+    assert S.request_wait(1, 0.0, 0.05) == []      # nothing grantable: waits the timeout
+    assert time.perf_counter() - t >= 0.04
+    import threading
+    th = threading.Thread(target=lambda: (time.sleep(0.05), S.report(0, 0.1, 100, 0.1), S.complete(0, 0, 0.1),
+                                          S.report(1, 0.1, 100, 0.1), S.complete(1, 1, 0.1)))
+    th.start()
+    t = time.perf_counter()
+    assert S.request_wait(1, 0.0, 5.0) is None      # woken by the last completion: all finished
+    assert time.perf_counter() - t < 2.0
+    th.join()
+    assert S.counter(0) == 4 and S.counter(3) == 2  # 4 request messages, 2 of them granted
 
 
 def test_chrome_trace_of_a_unit_log():
@@ -178,11 +236,15 @@ def test_chrome_trace_of_a_unit_log():
                 cells=10**9, committed=1, device_ms=9.5),
            dict(unit=1, kind=1, pair=2, worker=1, stream=0, t_grant=0.002, t_start=0.003, t_end=0.04,
                 cells=3 * 10**9, committed=0, device_ms=36.0)]
-    tr = chrome_trace(log)
+    sched = [dict(ev="G", worker=0, unit=0, t=5.0, phi=1, rate=1e12),
+             dict(ev="W", worker=1, unit=0, t=5.5, phi=6, rate=6e12), dict(ev="C", worker=0, unit=0, t=6.0)]
+    tr = chrome_trace(log, sched_log=sched)
     ev = tr["traceEvents"]
     units = [e for e in ev if e["ph"] == "X"]
     assert len(units) == 2 and len([e for e in ev if e["ph"] == "i"]) == 2
+    cnt = [e for e in ev if e["ph"] == "C"]
+    assert len(cnt) == 4 and cnt[2]["args"]["phi"] == 6 and abs(cnt[2]["ts"] - 5e5) < 1e-6
     assert units[0]["pid"] == 0 and units[0]["tid"] == 1 and abs(units[0]["dur"] - 1e4) < 1e-6
-    assert units[1]["args"]["committed"] == 0 and "K3" in units[1]["name"]
+    assert units[1]["args"]["committed"] == 0 and "K3" in units[1]["name"] and "lost" in units[1]["name"]
     assert {e["pid"] for e in ev if e["ph"] == "M"} == {0, 1}
     json.dumps(tr)

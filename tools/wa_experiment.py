@@ -1,14 +1,25 @@
 """The paper's workload-adjustment experiment (Fig. 6, P22 §V.B) and non-dedicated run
 (Figs. 7/8, P24 §V.C) on one B200: P slave workers share the GPU (separate streams and
-replicas of the database); one of them can emulate a slower PE (6x, Fig. 5's ratio),
-from the start or from a point mid-run (local load).  For each policy (SS, PSS) and WA
-on/off it reports makespan (device), GCUPS, tail (makespan - median worker finish),
-duplicated cells, WA grants and master interactions; scores are checked identical across
-all runs.
+replicas of the database); one of them is a slower PE -- GPU-side by default (its DP kernels
+get ceil(148/s) SMs: straggler mode "sm_cap"), or a local-load kernel ("noise"), or the
+host-side hold of round 1 ("hold") -- from the start or from a point mid-run (local load).
 
-  python tools/wa_experiment.py [--config C2] [--workers 4] [--reps 2] [--out FILE]
+For each scenario x policy (SS, PSS) x WA on/off it reports (best of --reps by makespan):
+  makespan  device time of the whole search (libsw's CUDA events);
+  last      device time of the last unit completion, and the tail = last - median over the
+            workers of their last unit completion (device clocks);
+  dup       cells of replicas that lost the race (cancelled replicas count what they computed);
+  messages  request messages to the master and how many of them granted tasks (an idle
+            worker's request waits at the master: one message, not a poll loop);
+  grants    the master's per-grant Φ and v̄ of the requesting worker (Figs. 7/8 marks).
+Scores are checked identical across all runs (and against the oracle's digest when the
+config has one).
+
+  python tools/wa_experiment.py [--config C2] [--workers 4] [--reps 2] [--mode sm_cap]
+                                [--unit-cells N] [--out FILE]
 """
 import argparse
+import hashlib
 import json
 import os
 import sys
@@ -18,72 +29,96 @@ import numpy as np
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 import seqgen  # noqa: E402
-from paper_conf_ipps_mendoncam13_b200 import Database  # noqa: E402
+from paper_conf_ipps_mendoncam13_b200 import Database, grant_timeline  # noqa: E402
+
+
+def digest(scores):
+    return hashlib.sha256(np.ascontiguousarray(scores, dtype="<i4").tobytes()).hexdigest()
 
 
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--config", default="C2")
     ap.add_argument("--workers", type=int, default=4)
+    ap.add_argument("--streams", type=int, default=2)
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--slowdown", type=int, default=6)
+    ap.add_argument("--mode", default="sm_cap", choices=["sm_cap", "noise", "hold"])
+    ap.add_argument("--policies", default="pss,ss")
+    ap.add_argument("--scenarios", default="homogeneous,straggler,local_load_midrun")
     ap.add_argument("--out", default=None)
     ap.add_argument("--unit-cells", type=int, default=0,
                     help="target_unit_cells (0 = auto; 2**62 = the paper's very coarse tasks, one per pack)")
     args = ap.parse_args()
     w = seqgen.make_workload(args.config)
+    gold = json.load(open(os.path.join(ROOT, "tests", "golden", "oracle_digests.json"))).get(args.config)
     D = Database(w.db, devices=[0] * args.workers)
     straggler = 1 << (args.workers - 1)
-    base = D.search(w.queries, top_k=10, streams=2)   # warm-up + reference scores
-    ref = base.scores.copy()
+    base = D.search(w.queries, top_k=10, streams=args.streams)   # warm-up + reference scores
+    ref = digest(base.scores)
+    if gold:
+        assert ref == gold["sha256_scores"], "scores differ from the oracle's digest"
     t_ref = base.stats["seconds_device"]
-    scenarios = [("homogeneous", 0, 0), ("straggler", straggler, 0),
-                 ("local_load_midrun", straggler, int(1000 * 0.3 * t_ref))]
+    scen = {"homogeneous": (0, 0), "straggler": (straggler, 0),
+            "local_load_midrun": (straggler, int(1000 * 0.3 * t_ref))}
     rows = []
-    for name, mask, after in scenarios:
-        for policy in ("pss", "ss"):
+    for name in args.scenarios.split(","):
+        mask, after = scen[name]
+        for policy in args.policies.split(","):
             for wa in (True, False):
                 best = None
                 for _ in range(args.reps):
-                    r = D.search(w.queries, top_k=10, streams=2, policy=policy, workload_adjust=wa,
+                    r = D.search(w.queries, top_k=10, streams=args.streams, policy=policy, workload_adjust=wa,
                                  straggler_mask=mask, straggler_slowdown=args.slowdown,
-                                 straggler_after_ms=after, target_unit_cells=args.unit_cells)
-                    assert (r.scores == ref).all(), "scores differ across schedules"
+                                 straggler_after_ms=after, straggler_mode=args.mode,
+                                 target_unit_cells=args.unit_cells)
+                    assert digest(r.scores) == ref, "scores differ across schedules"
                     st = r.stats
                     if best is None or st["seconds_device"] < best["seconds_device"]:
                         best = st
                 log = best["unit_log"]
                 per_worker = {}
                 for e in log:
-                    d = per_worker.setdefault(e["worker"], {"units": 0, "committed": 0, "cells": 0,
-                                                            "last_end": 0.0})
-                    d["units"] += 1
+                    d = per_worker.setdefault(e["worker"], {"replicas": 0, "committed": 0, "cancelled": 0,
+                                                            "cells_done": 0, "last_dev_ms": 0.0})
+                    d["replicas"] += 1
                     d["committed"] += e["committed"]
-                    d["cells"] += e["cells"]
-                    d["last_end"] = max(d["last_end"], e["t_end"])
+                    d["cancelled"] += e["cancelled"]
+                    d["cells_done"] += e["cells_done"]
+                    d["last_dev_ms"] = max(d["last_dev_ms"], e["dev_t1"])
+                grants = grant_timeline(best["sched_log"])
                 row = dict(scenario=name, policy=policy, wa=wa, makespan_s=best["seconds_device"],
-                           gcups=best["gcups"], tail_s=best["tail_seconds"],
-                           duplicated_cells=best["duplicated_cells"], wa_grants=best["n_wa_grants"],
-                           requests=best["n_requests"], units=best["n_units"], per_worker=per_worker,
-                           timeline=[(e["worker"], round(e["t_start"], 4), round(e["t_end"], 4),
-                                      e["cells"], e["committed"]) for e in log])
+                           last_unit_s=best["seconds_last_unit"], tail_s=best["tail_seconds"],
+                           gcups=best["gcups"], duplicated_cells=best["duplicated_cells"],
+                           wa_grants=best["n_wa_grants"], cancelled=best["n_cancelled"],
+                           request_messages=best["n_requests"], grant_messages=best["n_grant_messages"],
+                           units=best["n_units"], per_worker=per_worker,
+                           grants=[(round(g["t_rel"], 4), g["worker"], g["unit"], g["phi"],
+                                    round(g["rate"] / 1e9, 1), g["wa"]) for g in grants],
+                           timeline=[(e["worker"], e["unit"], round(e["dev_t0"], 2), round(e["dev_t1"], 2),
+                                      e["cells"], e["cells_done"], e["committed"], e["cancelled"], e["slowed"])
+                                     for e in log])
                 rows.append(row)
                 print(f"{name:18s} {policy:3s} WA={'on ' if wa else 'off'} makespan {row['makespan_s']:.3f}s "
-                      f"{row['gcups']:8.1f} GCUPS tail {row['tail_s']:.3f}s dup {row['duplicated_cells']:.2e} "
-                      f"wa {row['wa_grants']} req {row['requests']}", flush=True)
-    # WA gain per scenario/policy (the paper's Fig. 6 quantity)
+                      f"last {row['last_unit_s']:.3f}s tail {row['tail_s']:.3f}s {row['gcups']:8.1f} GCUPS "
+                      f"dup {row['duplicated_cells']:.2e} wa {row['wa_grants']} cancelled {row['cancelled']} "
+                      f"msgs {row['request_messages']} (granting {row['grant_messages']})", flush=True)
     summary = {}
-    for name, _, _ in scenarios:
-        for policy in ("pss", "ss"):
+    for name in args.scenarios.split(","):
+        for policy in args.policies.split(","):
             on = next(r for r in rows if r["scenario"] == name and r["policy"] == policy and r["wa"])
             off = next(r for r in rows if r["scenario"] == name and r["policy"] == policy and not r["wa"])
-            summary[f"{name}/{policy}"] = dict(gcups_gain_pct=100.0 * (on["gcups"] / off["gcups"] - 1.0),
-                                               makespan_on=on["makespan_s"], makespan_off=off["makespan_s"],
-                                               tail_on=on["tail_s"], tail_off=off["tail_s"])
-            print(f"WA gain {name}/{policy}: {summary[f'{name}/{policy}']['gcups_gain_pct']:+.1f} % GCUPS")
-    out = dict(config=args.config, workers=args.workers, slowdown=args.slowdown, unit_cells=args.unit_cells,
-               note="P workers share one B200 (separate streams/replicas); the straggler holds each "
-                    "completion back by (slowdown-1) x the unit's device time",
+            summary[f"{name}/{policy}"] = dict(
+                gcups_gain_pct=100.0 * (on["gcups"] / off["gcups"] - 1.0),
+                makespan_on=on["makespan_s"], makespan_off=off["makespan_s"],
+                tail_on=on["tail_s"], tail_off=off["tail_s"],
+                tail_reduction_pct=(100.0 * (1 - on["tail_s"] / off["tail_s"]) if off["tail_s"] > 0 else None))
+            s = summary[f"{name}/{policy}"]
+            print(f"WA {name}/{policy}: {s['gcups_gain_pct']:+.1f} % GCUPS, makespan {s['makespan_off']:.3f} -> "
+                  f"{s['makespan_on']:.3f} s, tail {s['tail_off']:.3f} -> {s['tail_on']:.3f} s")
+    out = dict(config=args.config, workers=args.workers, streams=args.streams, slowdown=args.slowdown,
+               mode=args.mode, unit_cells=args.unit_cells, oracle_digest_checked=bool(gold),
+               note="P workers share one B200 (separate streams/replicas); the straggler is the last worker",
                summary=summary, runs=rows)
     if args.out:
         with open(args.out, "w") as f:
