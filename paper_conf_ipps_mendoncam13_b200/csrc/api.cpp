@@ -243,7 +243,7 @@ static void validate_seqset(const sw_seqset *s, const char *what) {
 }
 
 static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, int n_workers,
-                      const int8_t *M, int32_t thresh) {
+                      const int8_t *M, int32_t thresh, int32_t k1_wave) {
   Plan P;
   const int32_t nq = q->n;
   P.qoff.resize(nq + 1);
@@ -411,18 +411,39 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
     // K1 units over the short groups
     const int64_t band = k1_band_rows();
     const int64_t rows_k1 = (int64_t)(qp.rows + band - 1) / band * band;
+    // Auto sizing cuts a unit at whole waves of groups (k1_wave = resident K1 blocks of the
+    // GPU, each block streams through its groups): 1.5 waves would leave half the SMs idle
+    // for the last third of the launch.  The groups of a unit have nearly equal widths (length
+    // sort), so k waves take ~k group times on every block.  The remainder of a segment
+    // (< k waves) is its own, short unit, scheduled late by the LPT order below.
     for (int32_t g = gl; g < ng;) {
-      int32_t e = g;
-      int64_t cells = 0, work = 0;
       // (units do not straddle the kWideCols boundary: each launch uses one K1 instance)
       const bool wide = db.groups[g].ncols >= kWideCols;
-      while (e < ng && (cells < target || e == g) && (db.groups[e].ncols >= kWideCols) == wide) {
-        cells += rows_eff * grp_res[e];
-        work += rows_k1 * db.groups[e].ncols * kGroup;
-        e++;
+      int32_t seg_end = g;
+      int64_t seg_cells = 0;
+      while (seg_end < ng && (db.groups[seg_end].ncols >= kWideCols) == wide) seg_cells += rows_eff * grp_res[seg_end++];
+      int32_t per_unit = 0;   // groups per unit, 0 = cut by cells
+      if (o.target_unit_cells <= 0 && k1_wave > 0) {
+        const double n_u = std::max(1.0, std::floor((double)seg_cells / (double)target + 0.5));
+        const int32_t gpu = (int32_t)std::ceil((seg_end - g) / n_u);
+        // k = ceil(groups / wave) waves; a unit under half a wave keeps its cell-based cut
+        // (several streams' small units fill the GPU together; rounding them up to a wave
+        // would coarsen small databases for no gain).  SW_K1_WAVES forces k (tuning).
+        static const int forced = [] { const char *e = getenv("SW_K1_WAVES"); return e ? atoi(e) : 0; }();
+        if (forced > 0) per_unit = forced * k1_wave;
+        else if (2 * gpu >= k1_wave) per_unit = (gpu + k1_wave - 1) / k1_wave * k1_wave;
       }
-      P.units.push_back({kUnitInter, p, g, e, cells, work});
-      g = e;
+      while (g < seg_end) {
+        int32_t e = g;
+        int64_t cells = 0, work = 0;
+        while (e < seg_end && (per_unit > 0 ? e - g < per_unit : (cells < target || e == g))) {
+          cells += rows_eff * grp_res[e];
+          work += rows_k1 * db.groups[e].ncols * kGroup;
+          e++;
+        }
+        P.units.push_back({kUnitInter, p, g, e, cells, work});
+        g = e;
+      }
     }
   }
   // drop empty units (e.g. all-empty queries still produce valid zero scores: keep them
@@ -703,7 +724,13 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
     const PackedDB &H = db->host;
     const int32_t nq = queries->n, nd = H.n;
     const int nW = dist ? 1 : (int)db->devs.size();
-    Plan P = make_plan(queries, H, o, dist ? o.dist_world : nW, M, thresh);
+    // one wave of K1 blocks on the (first) GPU: SMs x resident K1 blocks per SM
+    int32_t k1_wave = 0;
+    if (!db->devs.empty()) {
+      CK(cudaSetDevice(db->devs[0]->id));
+      k1_wave = db->devs[0]->n_sm * k1_blocks_per_sm();
+    }
+    Plan P = make_plan(queries, H, o, dist ? o.dist_world : nW, M, thresh, k1_wave);
     const double wall0 = now_s();
     const int K = (hits && top_k > 0 && nq > 0) ? top_k : 0;   // hits wanted
     const int64_t nsc = (int64_t)nq * nd;

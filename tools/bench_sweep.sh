@@ -1,19 +1,12 @@
 #!/bin/bash
-# bench_sweep.sh "<label>|<VAR=val ...>|<bench args>" ... : short C4 bench lines for tuning experiments
-# (3 timed steps, no e2e / cpu baseline), one summary line per setting into gpurun_out/sweep.txt
-mkdir -p gpurun_out
+# Parameter sweep on the bench workload: each line is "label ENV=..." ; prints value and the
+# K1-alone roofline fraction.  Usage: tools/bench_sweep.sh "base" "w2 SW_K1_WAVES=2" ...
 for spec in "$@"; do
-  IFS='|' read -r label envs args <<< "$spec"
-  env $envs python bench.py $args --steps 3 --warmup 2 --e2e-steps 0 --no-cpu-baseline > gpurun_out/sweep_$label.log 2>&1
-  python - "$label" <<'PY' >> gpurun_out/sweep.txt
+  label=${spec%% *}; envs=${spec#* }; [ "$envs" = "$spec" ] && envs=""
+  line=$(env $envs python bench.py --steps ${STEPS:-3} --warmup 2 --e2e-steps 0 --no-cpu-baseline 2>/dev/null | tail -1)
+  python - "$label" "$line" <<'PY'
 import json, sys
-lab = sys.argv[1]
-try:
-    d = json.loads(open(f"gpurun_out/sweep_{lab}.log").read().strip().splitlines()[-1])
-    r = d["roofline"]
-    print(f"{lab:24s} {d['value']:8.1f} GCUPS  frac {r['frac']:.3f}  k1_alone {r['k1_alone_gcups'] or 0:7.1f}  "
-          f"k3_alone {r['k3_alone_gcups'] or 0:7.1f}  units {d['config']['units_per_step']}  clk {d['clocks']['sm_mhz']}")
-except Exception as e:
-    print(f"{lab:24s} FAILED {e}")
+d = json.loads(sys.argv[2]); r = d["roofline"]
+print(f'{sys.argv[1]:12s} step {d["value"]:8.1f} GCUPS  k1_alone {r["achieved"]:8.1f} (frac {r["frac"]:.3f})  units {d["config"]["units_per_step"]}  k3_alone {r["k3_alone_gcups"]:.0f}', flush=True)
 PY
 done
