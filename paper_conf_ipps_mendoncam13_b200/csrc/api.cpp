@@ -121,7 +121,9 @@ struct DevSearch {
   DBuf<int32_t> ovf_cursor;    // [streams] entries taken by the int32 re-run
   DBuf<uint32_t> ovf_bits;     // [nq*ndb] bits: pair already listed
   int32_t ovf_cap = 0;         // entries per stream list
-  DBuf<uint2> k3_border;   // [streams][max_k3_seqs][max_len]
+  DBuf<uint2> k3_border;   // [streams][k3_rows][max_len]
+  int64_t k3_rows = 0;
+  DBuf<int32_t> k3_prog;   // [streams][k3 slots x warps]: clustered K3 progress counters
   DBuf<int32_t> k2_border;
   DBuf<int32_t> abort_dev;      // per-unit WA cancellation flags (device memory)
   DBuf<int32_t> progress;       // per-unit progress counters (K1 groups / K3 sequence-chunks)
@@ -243,7 +245,7 @@ static void validate_seqset(const sw_seqset *s, const char *what) {
 }
 
 static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, int n_workers,
-                      const int8_t *M, int32_t thresh, int32_t k1_wave) {
+                      const int8_t *M, int32_t thresh, int32_t k1_wave, int32_t k3_slots) {
   Plan P;
   const int32_t nq = q->n;
   P.qoff.resize(nq + 1);
@@ -369,6 +371,26 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
   int64_t total_cells = 0;
   for (int64_t r : P.real_rows) total_cells += r * db.residues;
   P.cells = total_cells;
+  // K3 cluster size (auto sizing): when long sequences carry most of the work and one
+  // worker's share of (pack, long-sequence block) tasks fills too few of the GPU's resident
+  // K3 CTAs -- C5 at 8 GPUs: 256 blocks for 592 slots -- each pair's chunks are split over a
+  // cluster of 4 (fill < 1/2) or 2 CTAs.  SW_K3_CLUSTER forces a size (tuning, tests).
+  int32_t k3_cluster = 1;
+  {
+    int64_t long_res = 0;
+    for (int32_t s = 0; s < P.n_long_seqs; s++) long_res += db.sorted_len[s];
+    int64_t rows_all = 0;
+    for (int64_t r : P.real_rows) rows_all += r;
+    const int64_t c3 = rows_all * long_res, c1 = total_cells - c3;
+    const double sb_per_worker = (double)P.pairs.size() * ((P.n_long_seqs + kK3Warps - 1) / kK3Warps) /
+                                 std::max(1, n_workers);
+    static const int forced = [] { const char *e = getenv("SW_K3_CLUSTER"); return e ? atoi(e) : 0; }();
+    if (forced == 1 || forced == 2 || forced == 4 || forced == 8) k3_cluster = forced;
+    else if (o.target_unit_cells <= 0 && P.n_long_seqs > 0 && c3 >= c1 && k3_slots > 0) {
+      const double fill = sb_per_worker / k3_slots;
+      k3_cluster = fill < 0.5 ? 4 : fill < 1.0 ? 2 : 1;
+    }
+  }
   int64_t target = o.target_unit_cells;
   const int depth = std::max(1, o.streams_per_device);
   if (target <= 0) {
@@ -396,15 +418,24 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
       const int64_t per_pack = ((int64_t)n_workers * depth + n_packs - 1) / n_packs;
       if (per_pack > 1) k3_target = std::max<int64_t>(1, std::min<int64_t>(k3_target, (long_cells + per_pack - 1) / per_pack));
     }
+    // clustered K3 (k3_cluster > 1): each pack's long sequences in just enough units for
+    // every stream of every worker to get one (a launch holds one stream's share of the GPU)
+    int32_t k3_unit_seqs = 0;
+    if (k3_cluster > 1) {
+      const int64_t per_pack = std::max<int64_t>(1, ((int64_t)n_workers * depth + n_packs - 1) / n_packs);
+      k3_unit_seqs = (int32_t)std::max<int64_t>(kK3Warps, (P.n_long_seqs + per_pack - 1) / per_pack);
+      k3_unit_seqs = (k3_unit_seqs + kK3Warps - 1) / kK3Warps * kK3Warps;
+    }
     for (int32_t s = 0; s < P.n_long_seqs;) {
       int32_t e = s;
       int64_t cells = 0, work = 0;
-      while (e < P.n_long_seqs && (cells < k3_target || e == s || (e - s) % kK3Warps)) {
+      while (e < P.n_long_seqs && (k3_unit_seqs > 0 ? e - s < k3_unit_seqs
+                                                     : (cells < k3_target || e == s || (e - s) % kK3Warps))) {
         cells += rows_eff * db.sorted_len[e];
         work += (int64_t)qp.rows_padded * db.sorted_len[e];
         e++;
       }
-      P.units.push_back({kUnitIntra, p, s, e, cells, work});
+      P.units.push_back({kUnitIntra, p, s, e, cells, work, k3_cluster, 0});
       P.max_k3_seqs = std::max(P.max_k3_seqs, e - s);
       s = e;
     }
@@ -441,7 +472,7 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
           work += rows_k1 * db.groups[e].ncols * kGroup;
           e++;
         }
-        P.units.push_back({kUnitInter, p, g, e, cells, work});
+        P.units.push_back({kUnitInter, p, g, e, cells, work, 1, 0});
         g = e;
       }
     }
@@ -455,7 +486,9 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
   // K1 units instead (K3, K1, K3, K1, ...): small K3 units alone on every stream would
   // leave SMs idle at the start of the step (C4 at 1/8 of its database: 140 ms of 447)
   static const bool interleave = [] { const char *e = getenv("SW_UNIT_INTERLEAVE"); return !(e && atoi(e) == 0); }();
-  auto small3 = [](const Unit &u) { return interleave && u.kind == kUnitIntra && u.b1 - u.b0 < kK3UnitSeqs; };
+  auto small3 = [](const Unit &u) {
+    return interleave && u.kind == kUnitIntra && u.cluster == 1 && u.b1 - u.b0 < kK3UnitSeqs;
+  };
   std::stable_sort(P.units.begin(), P.units.end(), [&](const Unit &a, const Unit &b) {
     const int ra = a.kind == kUnitIntra ? (small3(a) ? 1 : 0) : 2;
     const int rb = b.kind == kUnitIntra ? (small3(b) ? 1 : 0) : 2;
@@ -498,7 +531,7 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
     for (int b = 0; b < 8; b++) { h ^= (uint64_t)((v >> (8 * b)) & 0xff); h *= 1099511628211ull; }
   };
   mix(nq); mix(db.n); mix(db.residues); mix((int64_t)P.units.size());
-  for (const Unit &u : P.units) { mix(u.kind); mix(u.pair); mix(u.b0); mix(u.b1); mix(u.cells); }
+  for (const Unit &u : P.units) { mix(u.kind); mix(u.pair); mix(u.b0); mix(u.b1); mix(u.cells); mix(u.cluster); }
   for (int32_t q : P.pack_q) mix(q);
   P.hash = h;
   return P;
@@ -537,6 +570,12 @@ static K2Args k2_args(const Plan &P, const PackedDB &db, DevSearch &S, int strea
   return a;
 }
 
+// resident K3 CTAs a clustered launch may use: its stream's share (SW_K3_SHARE: percent of
+// that share, tuning)
+static int k3_share(int slots, int streams) {
+  static const int pct = [] { const char *e = getenv("SW_K3_SHARE"); return e && atoi(e) > 0 ? atoi(e) : 100; }();
+  return (int)((int64_t)slots * pct / 100 / std::max(1, streams));
+}
 // sm_cap > 0: the unit's kernels get at most sm_cap SMs' worth of blocks (a slower PE,
 // straggler mode 1)
 static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const Unit &U, int uidx,
@@ -571,12 +610,28 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     a.ovf = S.ovf.p + (size_t)stream_idx * S.ovf_cap; a.ovf_count = S.ovf_count.p + stream_idx;
     a.ovf_cap = S.ovf_cap; a.ovf_bits = S.ovf_bits.p;
     const int64_t stride = (std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16;  // >= tiles * T
-    a.border = S.k3_border.p + (size_t)stream_idx * P.max_k3_seqs * stride;
+    a.border = S.k3_border.p + (size_t)stream_idx * S.k3_rows * stride;
     a.border_stride = stride;
+    a.kprog = nullptr;
+    a.claim = nullptr;
+    // tiles between a clustered chunk's progress publications (SW_K3_PUB: tuning)
+    static const int pub = [] { const char *e = getenv("SW_K3_PUB"); return e && atoi(e) > 0 ? atoi(e) : 8; }();
+    a.pub_every = pub;
+    const int slots = D.n_sm * k3_blocks_per_sm();
+    if (U.cluster > 1) {   // counters + the launch's claim counter, zeroed on its stream
+      a.kprog = S.k3_prog.p + (size_t)stream_idx * (slots * kK3Warps + 1);
+      a.claim = a.kprog + slots * kK3Warps;
+      CK(cudaMemsetAsync(a.kprog, 0, sizeof(int32_t) * (slots * kK3Warps + 1), st));
+    }
     a.abort_flag = S.abort_d + uidx;
     a.progress = S.progress.p + uidx;
     a.na = na; a.nb = nbm;
-    launch_k3(a, P.pairs[U.pair].rows_padded, st, sm_cap);
+    // grid: cluster 1 -> a block per kK3Warps sequences; clustered -> an equal share of the
+    // resident CTAs per stream (the streams' units run side by side, each claiming its
+    // sequence blocks longest first); a slower PE -> its SM budget
+    const int maxb = sm_cap > 0 ? std::min(D.n_sm, sm_cap) * k3_blocks_per_sm()
+                   : U.cluster > 1 ? std::max(U.cluster, k3_share(slots, (int)D.streams.size())) : INT32_MAX;
+    launch_k3(a, U.cluster, maxb, st);
   }
   S.launches++;
   // saturated pairs listed so far on this stream -> host (4 bytes): the worker launches
@@ -725,12 +780,18 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
     const int32_t nq = queries->n, nd = H.n;
     const int nW = dist ? 1 : (int)db->devs.size();
     // one wave of K1 blocks on the (first) GPU: SMs x resident K1 blocks per SM
-    int32_t k1_wave = 0;
+    int32_t k1_wave = 0, k3_slots = 0;
     if (!db->devs.empty()) {
       CK(cudaSetDevice(db->devs[0]->id));
       k1_wave = db->devs[0]->n_sm * k1_blocks_per_sm();
+      k3_slots = db->devs[0]->n_sm * k3_blocks_per_sm();
     }
-    Plan P = make_plan(queries, H, o, dist ? o.dist_world : nW, M, thresh, k1_wave);
+    Plan P = make_plan(queries, H, o, dist ? o.dist_world : nW, M, thresh, k1_wave, k3_slots);
+    bool any_cluster = false;
+    for (const Unit &u : P.units) any_cluster |= u.cluster > 1;
+    // K3 border rows per stream: one per sequence of the largest unit (cluster 1), and
+    // (resident clusters x warps x C buffers) = k3_slots x kK3Warps when a unit is clustered
+    const int64_t k3_rows = std::max<int64_t>(std::max(P.max_k3_seqs, 1), any_cluster ? (int64_t)k3_slots * kK3Warps : 0);
     const double wall0 = now_s();
     const int K = (hits && top_k > 0 && nq > 0) ? top_k : 0;   // hits wanted
     const int64_t nsc = (int64_t)nq * nd;
@@ -788,9 +849,10 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       X.ovf_cursor.ensure(D.id, depth);
       X.ovf_bits.ensure(D.id, ((size_t)nq * nd + 31) / 32);
       X.k2_border.ensure(D.id, (size_t)depth * kK2Blocks * std::max<int64_t>(P.max_len, 1) * 2);
-      const size_t k3b = (size_t)depth * std::max(P.max_k3_seqs, 1) *
-                         ((std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16);
+      const size_t k3b = (size_t)depth * k3_rows * ((std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16);
       if (P.n_long_seqs > 0) X.k3_border.ensure(D.id, k3b);
+      if (any_cluster) X.k3_prog.ensure(D.id, (size_t)depth * (k3_slots * kK3Warps + 1));
+      X.k3_rows = k3_rows;
       const size_t nu = std::max<size_t>(P.units.size(), 1);
       X.abort_dev.ensure(D.id, nu);
       CK(cudaMemset(X.abort_dev.p, 0, sizeof(int32_t) * nu));
@@ -1324,6 +1386,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         const UnitLog &L = ulog[k];
         const Unit &U = P.units[L.unit];
         js << (k ? "," : "") << "{\"unit\":" << L.unit << ",\"kind\":" << U.kind << ",\"pair\":" << U.pair
+           << ",\"b0\":" << U.b0 << ",\"b1\":" << U.b1 << ",\"cluster\":" << U.cluster
            << ",\"worker\":" << L.worker << ",\"t_grant\":" << L.t_grant << ",\"t_start\":" << L.t_start
            << ",\"t_end\":" << L.t_end << ",\"cells\":" << L.cells << ",\"cells_done\":" << L.cells_done
            << ",\"committed\":" << L.committed << ",\"cancelled\":" << L.cancelled << ",\"slowed\":" << L.slowed

@@ -19,6 +19,7 @@
 // Saturation: no half can wrap while best~ + max(S) <= 32767;
 // a lane half whose best~ reaches 32768 - max(S) is flagged and re-scored in int32 (K2).
 #include <cuda_runtime.h>
+#include <cooperative_groups.h>
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
@@ -54,6 +55,12 @@ __device__ __forceinline__ bool block_aborted(const volatile int32_t *flag) {
   return ab != 0;
 }
 constexpr int kAbortPoll = 32;   // K1 pipeline steps between WA cancellation polls
+__device__ __forceinline__ uint64_t globaltimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
 __device__ __forceinline__ uint32_t smid() {
   uint32_t r;
   asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
@@ -443,6 +450,7 @@ template <int W, int T, int MINB, int UQ>
 static int k1_occ() {
   auto fn = k1_kernel<kK1Rows, W, T, MINB, UQ>;
   cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem<W, T>());
+  cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared);
   int n = 0;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, W * 32, k1_smem<W, T>()) != cudaSuccess) n = 8;
   return n > 0 ? n : 1;
@@ -477,6 +485,7 @@ template <int W, int T, int MINB, int UQ>
 static void k1_go(const K1Args &a, dim3 g, cudaStream_t st) {
   auto fn = k1_kernel<kK1Rows, W, T, MINB, UQ>;
   cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)k1_smem<W, T>());
+  cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared);
   fn<<<g, W * 32, k1_smem<W, T>(), st>>>(a);
 }
 
@@ -513,13 +522,40 @@ void launch_k1(const K1Args &a_in, int n_groups, int min_cols, int, cudaStream_t
 // to the border.
 // Block = kK3Warps sequences sharing the chunk profile in shared memory, laid out
 // [slot][row pair][lane][2] (8-byte bank pair = lane mod 16: conflict-free although every
-// lane reads a different code).  A block walks sequence blocks blockIdx.x, +gridDim.x, ...
-// (one pass normally; several when the grid is capped to emulate a slower PE).  The unit's
-// WA cancellation flag is polled at every chunk start (__syncthreads_or), and each warp
-// counts the (sequence, chunk) pairs it completed into the unit's progress counter.
+// lane reads a different code).  The unit's WA cancellation flag is polled at every chunk
+// start (__syncthreads_or), and each warp counts the (sequence, chunk) pairs it completed
+// into the unit's progress counter.
+//
+// Chunk split over a thread-block cluster (C = 2 or 4, for units with too few long pairs to
+// fill the GPU -- one GPU's share of C5 at 8 GPUs): the C CTAs of a cluster take the same
+// kK3Warps sequences, CTA r the chunks r, r+C, r+2C, ... (the wavefront of Fig. 3a once more,
+// across CTAs: "it sends its border column to P1", P14).  Chunk ch writes its bottom row to
+// border buffer ch % C and publishes its progress every kK3Pub tiles (st.release, a
+// per-(warp slot, buffer) counter counting tiles since the launch); the CTA running chunk
+// ch+1 acquires that counter before prefetching a tile (cp.async.cg: L2, never a stale L1
+// line).  A buffer is rewritten by chunk ch+C only after chunk ch+1 consumed it: chunk ch+C
+// tile t needs chunk ch+C-1 tile t, ..., which needs chunk ch+1 past tile t.  The cluster
+// guarantees producer and consumer are co-resident, so the waits cannot deadlock.  Border
+// rows go through L2 rather than DSMEM: a DSMEM ring must hold the producer's 32-tile lane
+// skew (>= 40 tiles x 64 B x 4 warps), which would drop K3 from 4 to 3 CTAs per SM.
+// A persistent loop walks sequence blocks (grid capped to the resident clusters for C > 1,
+// or to an SM budget when emulating a slower PE).
 // ------------------------------------------------------------------------------------
-template <int K, int T>
-__global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
+__device__ __forceinline__ void cp_async16_cg(void *smem_dst, const void *gsrc) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(smem_dst);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d), "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ int ld_acquire(const int *p) {
+  int v;
+  asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(int *p, int v) {
+  asm volatile("st.release.gpu.global.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+template <int K, int T, int C>
+__global__ void __launch_bounds__(kK3Warps * 32, 4) k3_kernel(const K3Args a) {
   static_assert(T == 4 || T == 8, "tile = one or two 32-bit words of packed residues");
   constexpr int NW = T / 4;          // 32-bit residue words per tile
   constexpr int TPU = 4 / NW;        // tiles per 128-bit word
@@ -538,23 +574,46 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
   const int32_t *gprof = a.prof + P.prof_off;
   uint32_t *prof_s = smem;
   const int nsb = (a.l1 - a.l0 + kK3Warps - 1) / kK3Warps;
+  const int crank = C > 1 ? (int)(blockIdx.x % C) : 0;     // CTA rank in the cluster
+  const int cid = blockIdx.x / C, ncl = gridDim.x / C;
+  // C > 1: this warp's (slot, buffer) border rows and progress counters are per grid slot
+  // (reused across the sequence blocks of the persistent loop); cum[b] = tiles of buffer b
+  // published in earlier sequence blocks, identical in the producer and consumer CTAs
+  const int gslot = cid * kK3Warps + warp;
+  int cum[C];
+#pragma unroll
+  for (int b = 0; b < C; b++) cum[b] = 0;
   int done = 0;          // (sequence, chunk) pairs this warp completed
   bool aborted = false;
+  // C > 1: the clusters of a launch claim sequence blocks dynamically (longest first, the
+  // sorted order) from a per-launch counter; rank 0 claims and broadcasts over DSMEM
+  __shared__ int sb_claim;
+  auto next_sb = [&](int prev) -> int {
+    if (C == 1) return prev < 0 ? cid : prev + ncl;
+    namespace cg = cooperative_groups;
+    cg::cluster_group cl = cg::this_cluster();
+    if (crank == 0 && threadIdx.x == 0)
+      sb_claim = (aborted || (a.abort_flag && *a.abort_flag != 0)) ? nsb : atomicAdd(a.claim, 1);
+    cl.sync();
+    const int v = *cl.map_shared_rank(&sb_claim, 0);
+    cl.sync();   // rank 0 may overwrite sb_claim only after every CTA read it
+    return v;
+  };
 
-  for (int sb = blockIdx.x; sb < nsb && !aborted; sb += gridDim.x) {
+  for (int sb = next_sb(-1); sb < nsb; sb = next_sb(sb)) {
+    if (aborted) continue;   // C > 1: go straight to the next claim (it returns the end)
     const int s = a.l0 + sb * kK3Warps + warp;
     const bool valid = s < a.l1;
     const int len = valid ? a.sorted_len[s] : 0;
     const GroupInfo G = a.groups[valid ? s / kGroup : 0];
     const int gl = s % kGroup;
     const uint4 *wp = a.packed + G.word_off + gl;
-    uint2 *border = a.border + (size_t)(sb * kK3Warps + warp) * a.border_stride;
     const int ntile = (len + T - 1) / T;   // columns up to ntile*T <= G.ncols carry pad codes
     const int orig = valid ? a.perm[s] : 0;
     uint32_t best = koff;
     int cq_lo = -1, cq_hi = -1;   // queries of this lane's slice (per half)
 
-    for (int ch = 0; ch < nch; ch++) {
+    for (int ch = crank; ch < nch; ch += C) {
       // every warp is done with the previous chunk profile; WA cancellation poll
       if (__syncthreads_or(threadIdx.x == 0 && a.abort_flag && *a.abort_flag != 0)) {
         aborted = true;
@@ -588,6 +647,20 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
       }
       done++;
       if (len == 0) continue;
+      // border rows: C == 1: one row per sequence (slot sb*kK3Warps + warp of the unit);
+      // C > 1: buffer ch % C of this grid slot
+      const int bin = (ch + C - 1) % C, bout = ch % C;
+      const uint2 *border_in = C == 1 ? a.border + (size_t)(sb * kK3Warps + warp) * a.border_stride
+                                      : a.border + (size_t)(gslot * C + bin) * a.border_stride;
+      uint2 *border_out = C == 1 ? a.border + (size_t)(sb * kK3Warps + warp) * a.border_stride
+                                 : a.border + (size_t)(gslot * C + bout) * a.border_stride;
+      const int *prog_in = a.kprog + gslot * C + bin;
+      int *prog_out = a.kprog + gslot * C + bout;
+      // counters count tiles written into a buffer since the launch: earlier sequence blocks
+      // (cum[]) plus this sequence's earlier chunks of the same residue class mod C
+      const int need0 = C > 1 && ch > 0 ? cum[bin] + ((ch - 1) / C) * ntile : 0;
+      const int pub0 = C > 1 ? cum[bout] + (ch / C) * ntile : 0;
+      int seen = 0;                 // (lane 0) last acquired value of prog_in
       const bool any_mask = __any_sync(0xffffffffu, omask != 0);   // warp-uniform
       uint32_t H[K], E[K];
 #pragma unroll
@@ -606,8 +679,26 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
         if (tt < ntile) {
           const int sl = tt % 3;
           if (ch > 0) {
+            if (C > 1) {   // wait until the chunk above has published tile tt
+              const int want = need0 + tt + 1;
+              if (seen < want) {
+                seen = ld_acquire(prog_in);
+                if (seen < want) {
+                  // really waiting.  (%globaltimer is slow to read: an earlier version that
+                  // read it on every entry here ran the first consumer chunks ~3x slower.)
+                  const long long t_wait = clock64();
+                  while ((seen = ld_acquire(prog_in)) < want) {
+                    if (a.abort_flag && *a.abort_flag != 0) break;   // the producer stops too
+                    if (clock64() - t_wait > (1ll << 36)) __trap();   // ~35 s: never hang the GPU
+                  }
+                }
+              }
 #pragma unroll
-            for (int jj = 0; jj < T; jj += 2) cp_async16(&bring[sl * T + jj], &border[tt * T + jj]);
+              for (int jj = 0; jj < T; jj += 2) cp_async16_cg(&bring[sl * T + jj], &border_in[tt * T + jj]);
+            } else {
+#pragma unroll
+              for (int jj = 0; jj < T; jj += 2) cp_async16(&bring[sl * T + jj], &border_in[tt * T + jj]);
+            }
           }
           if (tt % TPU == 0) cp_async16(&wring[(tt / TPU) % 3], &wp[(size_t)(tt / TPU) * kGroup]);
         }
@@ -671,20 +762,27 @@ __global__ void __launch_bounds__(kK3Warps * 32) k3_kernel(const K3Args a) {
           for (int q = 0; q < NW; q++) out_c[q] = in_c[q];
           if (lane == 31 && ch < nch - 1) {
 #pragma unroll
-            for (int jj = 0; jj < T; jj++) border[tile * T + jj] = make_uint2(out_h[jj], out_f[jj]);
+            for (int jj = 0; jj < T; jj++) border_out[tile * T + jj] = make_uint2(out_h[jj], out_f[jj]);
+            if (C > 1 && ((tile + 1) % a.pub_every == 0 || tile + 1 == ntile))
+              st_release(prog_out, pub0 + tile + 1);   // orders this lane's border stores
           }
         }
       }
       if (lane == 0) asm volatile("cp.async.wait_all;" ::: "memory");
     }
+    // every CTA of the cluster advances the same cum[]: buffer b received ntile tiles from
+    // each chunk ch < nch - 1 with ch % C == b
+#pragma unroll
+    for (int b = 0; b < C; b++)
+      if (C > 1 && nch - 1 > b) cum[b] += ((nch - 1 - b + C - 1) / C) * ntile;
     if (valid && !aborted) {   // every lane flushes what it holds
       flush_half(cq_lo, lo16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
       flush_half(cq_hi, hi16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
     }
+    if (C == 1 && aborted) break;   // (C > 1: every CTA of the cluster reaches the claim, which ends)
   }
   if (a.progress && lane == 0 && done > 0) atomicAdd(a.progress, done);
 }
-
 // K3 tile width (tuning; SW_K3_T): 8 columns per lane step (default) or 4.
 static int k3_tile() {
   static const int v = [] { const char *e = getenv("SW_K3_T"); return (e && atoi(e) == 4) ? 4 : 8; }();
@@ -695,12 +793,31 @@ static size_t k3_smem() {
   return sizeof(uint32_t) * kNCodes * kK3Rows * 32 + sizeof(uint4) * kK3Warps * 3 +
          sizeof(uint2) * kK3Warps * 3 * T;
 }
-template <int T>
+template <int T, int C>
 static void k3_go(const K3Args &a, int n, int max_blocks, cudaStream_t st) {
   const size_t smem = k3_smem<T>();
-  const int blocks = std::min((n + kK3Warps - 1) / kK3Warps, std::max(1, max_blocks));
-  cudaFuncSetAttribute(k3_kernel<kK3Rows, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  k3_kernel<kK3Rows, T><<<blocks, kK3Warps * 32, smem, st>>>(a);
+  const int nsb = (n + kK3Warps - 1) / kK3Warps;
+  auto fn = k3_kernel<kK3Rows, T, C>;
+  cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared);
+  const int clusters = std::max(1, std::min(nsb, std::max(1, max_blocks / C)));
+  if (C == 1) {
+    fn<<<clusters, kK3Warps * 32, smem, st>>>(a);
+    return;
+  }
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(clusters * C);
+  cfg.blockDim = dim3(kK3Warps * 32);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = C;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  cudaLaunchKernelEx(&cfg, fn, a);
 }
 int k3_blocks_per_sm() {
   static std::once_flag once;
@@ -708,20 +825,27 @@ int k3_blocks_per_sm() {
   std::call_once(once, [] {
     int n = 0;
     const size_t smem = k3_tile() == 4 ? k3_smem<4>() : k3_smem<8>();
-    auto fn = k3_tile() == 4 ? k3_kernel<kK3Rows, 4> : k3_kernel<kK3Rows, 8>;
+    auto fn = k3_tile() == 4 ? k3_kernel<kK3Rows, 4, 1> : k3_kernel<kK3Rows, 8, 1>;
     cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared);
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, kK3Warps * 32, smem) == cudaSuccess && n > 0) v = n;
   });
   return v;
 }
-// n_sm_cap > 0 caps the grid to that many SMs' worth of resident blocks (slower-PE
-// emulation); otherwise one block per kK3Warps sequences
-void launch_k3(const K3Args &a, int, cudaStream_t st, int n_sm_cap) {
+// cluster size 1, 2 or 4 (a.kprog: [grid slots][C] zeroed progress counters when C > 1).
+// max_blocks caps the grid (resident CTAs; an SM budget when emulating a slower PE);
+// C > 1 needs at most the resident clusters (persistent loop, sequence blocks claimed
+// through a.claim, zeroed), C == 1 one block per kK3Warps sequences
+void launch_k3(const K3Args &a, int cluster, int max_blocks, cudaStream_t st) {
   const int n = a.l1 - a.l0;
   if (n <= 0) return;
-  const int maxb = n_sm_cap > 0 ? n_sm_cap * k3_blocks_per_sm() : INT32_MAX;
-  if (k3_tile() == 4) k3_go<4>(a, n, maxb, st);
-  else k3_go<8>(a, n, maxb, st);
+  const bool t4 = k3_tile() == 4;
+  switch (cluster) {
+    case 2: if (t4) k3_go<4, 2>(a, n, max_blocks, st); else k3_go<8, 2>(a, n, max_blocks, st); break;
+    case 4: if (t4) k3_go<4, 4>(a, n, max_blocks, st); else k3_go<8, 4>(a, n, max_blocks, st); break;
+    case 8: k3_go<8, 8>(a, n, max_blocks, st); break;
+    default: if (t4) k3_go<4, 1>(a, n, max_blocks, st); else k3_go<8, 1>(a, n, max_blocks, st); break;
+  }
 }
 
 // ------------------------------------------------------------------------------------
@@ -730,11 +854,6 @@ void launch_k3(const K3Args &a, int, cudaStream_t st, int n_sm_cap) {
 // the SM, spinning on integer work until the host raises *stop (or max_ns elapses: the
 // kernel can never outlive a lost host).  Launched on its own high-priority stream.
 // ------------------------------------------------------------------------------------
-__device__ __forceinline__ uint64_t globaltimer() {
-  uint64_t t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  return t;
-}
 __global__ void __launch_bounds__(256) noise_kernel(const volatile int32_t *stop, uint64_t max_ns,
                                                     uint32_t *sink) {
   extern __shared__ uint32_t noise_s[];

@@ -66,6 +66,8 @@ struct Unit {
   int32_t b0, b1;        // group range [b0,b1) (inter) or long-seq range (intra)
   int64_t cells;         // real cells (sum |q|*|d|), for GCUPS and PSS rates
   int64_t work;          // padded lane-cells (balancing)
+  int32_t cluster = 1;   // K3: CTAs per thread-block cluster splitting each pair's chunks
+  int32_t pad_ = 0;
 };
 
 // ---- query packs ------------------------------------------------------------------------
@@ -108,7 +110,11 @@ struct K3Args {   // sequences [l0,l1) in sorted order (the long groups)
   int32_t *scores; int64_t ndb;
   int32_t thresh;
   int2 *ovf; int32_t *ovf_count; int32_t ovf_cap; uint32_t *ovf_bits;
-  uint2 *border; int64_t border_stride;   // per sequence border row (>= max long len)
+  uint2 *border; int64_t border_stride;   // border rows (>= max long len): per sequence (C = 1)
+                                          // or per (grid slot, buffer) (cluster C > 1)
+  int32_t *kprog;                         // C > 1: per (grid slot, buffer) progress counters (zeroed)
+  int32_t *claim;                         // C > 1: sequence blocks claimed so far (zeroed)
+  int32_t pub_every;                      // C > 1: tiles between progress publications
   const volatile int32_t *abort_flag;     // WA cancellation flag (polled at chunk starts)
   int32_t *progress;                      // unit's counter: (sequence, chunk) pairs completed
   uint32_t na, nb;
@@ -149,7 +155,7 @@ void launch_profile(const uint8_t *qcodes, const int64_t *qoff, const QueryPair 
                     cudaStream_t st);
 void launch_k1(const K1Args &a, int n_groups, int min_cols, int rows_padded, cudaStream_t st,
                int n_sm);
-void launch_k3(const K3Args &a, int rows_padded, cudaStream_t st, int n_sm_cap);
+void launch_k3(const K3Args &a, int cluster, int max_blocks, cudaStream_t st);
 void launch_k2(const K2Args &a, int blocks, cudaStream_t st);
 void launch_fill(int32_t *p, int64_t n, int32_t v, cudaStream_t st);
 // committed-unit segments (cross-GPU data plane): query q x sorted sequences [s0, s1)

@@ -24,13 +24,16 @@ def _golden():
         return json.load(f)
 
 
-@pytest.mark.parametrize("cfg", ["C1", "C2", "C3", "C4", "C5", "RAT", "MOUSE"])
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3", "C4", "C5", "RAT", "MOUSE", "C5@256"])
 def test_full_matrix_digest(cfg):
+    """(C5@256: C5's database cut to 256 sequences, one GPU's share at 8 GPUs -- the K3
+    cluster-split path.)"""
     g = _golden()
     if cfg not in g:
         pytest.skip(f"no oracle digest for {cfg} yet")
     e = g[cfg]
-    w = seqgen.make_workload(cfg)
+    name, _, n_db = cfg.partition("@")
+    w = seqgen.make_workload(name, n_db=int(n_db) if n_db else None)
     assert (w.queries.n, w.db.n) == (e["n_queries"], e["n_db"])
     D = Database(w.db, devices=[0])
     try:

@@ -237,16 +237,17 @@ def _digest(cfg, scores):
 
 def test_wa_beats_a_gpu_side_straggler():
     """workload adjustment against a genuinely slow GPU.  Two workers share the
-    B200; after 30 % of the run worker 1's DP kernels get ceil(148/6) SMs (local load, P24 §V.C).
-    C2 with the paper's coarse tasks (one per pack and kernel kind) so a slow unit decides the end.  With WA on, the fast worker re-executes the
+    B200; worker 1's DP kernels get ceil(148/24) SMs.  C2 with the paper's coarse tasks (one per
+    pack), one stream per worker: the slow worker takes its first task before the master knows
+    its rate, so without WA that task decides the end.  With WA on, the fast worker re-executes the
     straggler's last unit, the straggler's replica is cancelled IN its kernel (abort flag polled
     in the group/chunk loops) and abandoned with the cells it really computed; makespan and tail
     drop.  Both runs are bit-exact against the oracle's C2 digest."""
     w = seqgen.make_workload("C2")
     D = Database(w.db, devices=[0, 0])
-    base = D.search(w.queries, top_k=10, target_unit_cells=2**62)
-    kw = dict(top_k=10, target_unit_cells=2**62, straggler_mask=0b10, straggler_slowdown=6,
-              straggler_mode="sm_cap", straggler_after_ms=int(300 * base.stats["seconds_device"]))
+    kw = dict(top_k=10, target_unit_cells=2**62, straggler_mask=0b10, straggler_slowdown=24,
+              straggler_mode="sm_cap", streams=1, long_threshold=-1)
+    D.search(w.queries, **kw)   # warm-up (lazy module loading, buffers)
     on = D.search(w.queries, workload_adjust=True, **kw)
     ok_on, e = _digest("C2", on.scores)
     off = D.search(w.queries, workload_adjust=False, **kw)
@@ -512,3 +513,50 @@ def test_extreme_lengths():
         r = _search(dbs, qs, top_k=4, long_threshold=thr)
         assert (r.scores == ref).all(), (thr, np.argwhere(r.scores != ref)[:5])
         _check_topk(r, ref, 4)
+
+
+_CLUSTER_SCRIPT = r"""
+import sys; sys.path.insert(0, %r)
+import numpy as np, oracle, seqgen
+from paper_conf_ipps_mendoncam13_b200 import Database
+w = seqgen.make_workload("C5", n_db=24)
+ref = oracle.search(w.queries, w.db)
+qs = seqgen.SeqSet.from_list([seqgen.residues(41, 0, L).tobytes() for L in (1300, 600, 17, 3000)])
+db = seqgen.random_seqset(42, 300, 0, 4000)
+db = seqgen.SeqSet.from_list([db.seq(i) for i in range(db.n)] + [b"W" * 3000])
+ref2 = oracle.search(qs, db)
+D = Database(w.db, devices=[0])
+r = D.search(w.queries, top_k=5)
+assert (r.scores == ref).all(), np.argwhere(r.scores != ref)[:5]
+assert r.stats["n_overflow_pairs"] >= 1
+# slower-PE grid cap: fewer resident clusters than sequence blocks (persistent loop)
+r = D.search(w.queries, top_k=5, straggler_mask=1, straggler_slowdown=40)
+assert (r.scores == ref).all()
+D.close()
+D = Database(db, devices=[0])
+for thr in (0, 500):
+    r = D.search(qs, top_k=3, long_threshold=thr)
+    assert (r.scores == ref2).all(), np.argwhere(r.scores != ref2)[:5]
+D.close()
+# WA replicas of clustered units cancelled mid-run (spinning consumers must see the abort)
+D = Database(w.db, devices=[0, 0])
+r = D.search(w.queries, top_k=5, target_unit_cells=10**9, straggler_mask=2, straggler_slowdown=8)
+assert (r.scores == ref).all()
+D.close()
+print("ok", r.stats["n_cancelled"], r.stats["n_wa_grants"])
+"""
+
+
+@pytest.mark.parametrize("cluster", ["2", "4"])
+def test_k3_cluster_split(cluster):
+    """K3 with each pair's chunks split over a thread-block cluster (SW_K3_CLUSTER forces the
+    size; auto picks it for small long-sequence shares): bit-exact on C5-shaped pairs with an
+    overflow, with a capped (persistent) grid, on mixed lengths, and with WA cancellations."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, SW_K3_CLUSTER=cluster)
+    out = subprocess.run([sys.executable, "-c", _CLUSTER_SCRIPT % root], env=env, capture_output=True,
+                         text=True, timeout=900)
+    assert out.returncode == 0 and "ok" in out.stdout, (out.stdout[-2000:], out.stderr[-3000:])

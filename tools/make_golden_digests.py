@@ -7,6 +7,8 @@ checked bit-exactly (BASELINE.json north_star: "bit-exact scores versus the orac
 five configs").
 
   python tools/make_golden_digests.py [C1 C2 C3 C5 C4 ...]   (C4 takes ~1 h on 8 cores)
+  A name "CFG@N" is config CFG with its database cut to N sequences (e.g. C5@256: one GPU's
+  share of C5 at 8 GPUs).
 """
 import hashlib
 import json
@@ -34,7 +36,8 @@ def main(cfgs):
         with open(OUT) as f:
             data = json.load(f)
     for cfg in cfgs:
-        w = seqgen.make_workload(cfg)
+        name, _, n_db = cfg.partition("@")
+        w = seqgen.make_workload(name, n_db=int(n_db) if n_db else None)
         t = time.perf_counter()
         sc = oracle.search(w.queries, w.db)
         dt = time.perf_counter() - t
@@ -47,7 +50,7 @@ def main(cfgs):
             "top10_scores": s.tolist(), "top10_index": i.tolist(),
             "oracle_seconds": round(dt, 1), "oracle_threads": os.cpu_count(),
             "matrix": "BLOSUM62", "gap_open": 10, "gap_extend": 2,
-            "writer": "tools/make_golden_digests.py (oracle.search on seqgen.make_workload(cfg))",
+            "writer": "tools/make_golden_digests.py (oracle.search on seqgen.make_workload(cfg[, n_db]))",
         }
         with open(OUT + ".tmp", "w") as f:
             json.dump(data, f, indent=1)
