@@ -118,7 +118,12 @@ typedef struct {
   int32_t straggler_after_ms;/* the straggler slows down only after this many ms (local
                                 load introduced mid-run, P24 §V.C); 0 = from the start */
   int32_t straggler_mode;    /* SW_STRAGGLER_* (default SW_STRAGGLER_SM_CAP) */
-  int32_t reserved[6];
+  int32_t worker_sms;        /* experiments: > 0 caps EVERY worker's DP kernels to this many SMs'
+                                worth of resident blocks (split over its streams), so several
+                                workers sharing one GPU behave like separate smaller GPUs; a
+                                straggler (SW_STRAGGLER_SM_CAP) then gets ceil(worker_sms / s).
+                                0 = no partition (default) */
+  int32_t reserved[5];
 } sw_opts;
 
 typedef struct {

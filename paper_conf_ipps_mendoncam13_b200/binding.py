@@ -48,7 +48,8 @@ class sw_opts(ctypes.Structure):
                 ("straggler_slowdown", ctypes.c_int32), ("dist_rank", ctypes.c_int32),
                 ("dist_world", ctypes.c_int32), ("dist_port", ctypes.c_int32),
                 ("dist_host", ctypes.c_char_p), ("straggler_after_ms", ctypes.c_int32),
-                ("straggler_mode", ctypes.c_int32), ("reserved", ctypes.c_int32 * 6)]
+                ("straggler_mode", ctypes.c_int32), ("worker_sms", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 5)]
 
 
 class sw_alignment(ctypes.Structure):
@@ -291,7 +292,7 @@ class Database:
     def search(self, queries, matrix=None, gap_open=10, gap_extend=2, top_k=10, want_scores=True,
                policy="pss", workload_adjust=True, omega=4, streams=4, target_unit_cells=0,
                long_threshold=0, outputs_on_device=False, straggler_mask=0, straggler_slowdown=6,
-               straggler_after_ms=0, straggler_mode="sm_cap", dist=None, out_scores=None,
+               straggler_after_ms=0, straggler_mode="sm_cap", worker_sms=0, dist=None, out_scores=None,
                out_hits=None) -> SearchResult:
         """sw_search.  Host outputs are numpy arrays (pinned buffers may be passed via
         out_scores / out_hits); with outputs_on_device the outputs are torch CUDA tensors.
@@ -313,6 +314,7 @@ class Database:
         o.straggler_slowdown = straggler_slowdown
         o.straggler_after_ms = straggler_after_ms
         o.straggler_mode = _STRAGGLER_MODES[straggler_mode]
+        o.worker_sms = worker_sms
         if dist is not None:
             o.dist_rank, o.dist_world, o.dist_port = dist["rank"], dist["world"], dist["port"]
             host = dist.get("host", "127.0.0.1").encode()

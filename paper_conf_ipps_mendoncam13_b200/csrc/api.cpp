@@ -133,6 +133,7 @@ struct DevSearch {
   int32_t *prog_h = nullptr;     // pinned [kMaxStreams]: the unit's progress after it ran
   cudaStream_t cancel_st = nullptr;
   cudaStream_t noise_st = nullptr;   // high priority: the local-load kernel (straggler mode 2)
+  std::vector<cudaStream_t> epi;     // [1] high priority: the units' K2 + K5u epilogues
   DBuf<int32_t> noise_flag;
   DBuf<uint32_t> noise_sink;
   std::vector<char> cancelled;
@@ -186,6 +187,7 @@ inline DevSearch::~DevSearch() {
   if (prog_h) cudaFreeHost(prog_h);
   if (cancel_st) cudaStreamDestroy(cancel_st);
   if (noise_st) cudaStreamDestroy(noise_st);
+  for (auto e : epi) cudaStreamDestroy(e);
   if (ev_start) cudaEventDestroy(ev_start);
   if (ev_end) cudaEventDestroy(ev_end);
   if (ev_data) cudaEventDestroy(ev_data);
@@ -873,10 +875,15 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         CK(cudaHostAlloc((void **)&X.prog_h, sizeof(int32_t) * kMaxStreams, cudaHostAllocDefault));
       }
       if (!X.cancel_st) CK(cudaStreamCreateWithFlags(&X.cancel_st, cudaStreamNonBlocking));
-      if (!X.noise_st) {
+      {
         int lo = 0, hi = 0;
         CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
-        CK(cudaStreamCreateWithPriority(&X.noise_st, cudaStreamNonBlocking, hi));
+        if (!X.noise_st) CK(cudaStreamCreateWithPriority(&X.noise_st, cudaStreamNonBlocking, hi));
+        while (X.epi.empty()) {   // one per worker (the hardware work queues are limited)
+          cudaStream_t e;
+          CK(cudaStreamCreateWithPriority(&e, cudaStreamNonBlocking, hi));
+          X.epi.push_back(e);
+        }
       }
       if (!X.ev_start) CK(cudaEventCreate(&X.ev_start));
       if (!X.ev_end) CK(cudaEventCreate(&X.ev_end));
@@ -986,10 +993,13 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         // slower-PE emulation (SURVEY §8(d) WA experiment; P24 §V.C local load from t_after)
         const bool straggler = (o.straggler_mask >> wid) & 1ull;
         const int slow = std::max(1, o.straggler_slowdown);
-        const int sm_cap = (D.n_sm + slow - 1) / slow;     // ceil(n_sm / slowdown)
-        // mode SM cap: the worker's budget of sm_cap SMs is split over its streams (up to
-        // `depth` units run at once), so the whole worker holds ~sm_cap SMs' worth of blocks
+        // the worker's SM budget: the whole GPU, or its partition (worker_sms, experiments)
+        const int budget = o.worker_sms > 0 ? std::min(o.worker_sms, D.n_sm) : D.n_sm;
+        const int sm_cap = (budget + slow - 1) / slow;     // ceil(budget / slowdown)
+        // a budget is split over the worker's streams (up to `depth` units run at once), so
+        // the whole worker holds ~budget SMs' worth of blocks
         const int sm_share = std::max(1, (sm_cap + depth - 1) / depth);
+        const int part_share = o.worker_sms > 0 ? std::max(1, (budget + depth - 1) / depth) : 0;
         const double t_after = 1e-3 * std::max(0, o.straggler_after_ms);
         std::deque<int32_t> pending;
         std::vector<int32_t> inflight(depth, -1);
@@ -1079,11 +1089,16 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
             inflight[k] = -1;
             completed_wait[k] = 0;
             progressed = changed = true;
-            // int32 re-run of what this unit saturated, on its stream before the next unit
-            // (overlaps the units in flight on the other streams)
+            // epilogue of a completed unit on the worker's high-priority epilogue stream, so
+            // the stream goes straight on to its next unit: the int32 re-run of what the
+            // stream's units saturated (K2), then (committed) the unit's top-k (K5u).  Both
+            // small kernels wait for free SM slots behind persistent K1 blocks; on the unit's
+            // own stream they delayed its next unit (C4 at 1/8 of its database: 16 % idle).
+            // K2 may see entries a later unit on the stream is appending: it recomputes such
+            // a pair exactly, and the later partial maxima of its other slices are smaller.
             const int32_t seen = ((volatile int32_t *)X.ovf_seen_h)[k];
             if (seen > k2_upto[k]) {
-              launch_k2(k2_args(P, H, X, k, alpha, beta), kK2Blocks, D.streams[k]);
+              launch_k2(k2_args(P, H, X, k, alpha, beta), kK2Blocks, X.epi[0]);
               CK(cudaGetLastError());
               X.launches++;
               k2_upto[k] = seen;
@@ -1096,7 +1111,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
                 unit_seq_range(U, nd, s0u, s1u);
                 const int32_t q0 = P.pack_q_off[U.pair], nqp = P.pack_q_off[U.pair + 1] - q0;
                 launch_unit_topk(X.scores, nd, D.perm.p, s0u, s1u, X.pack_q.p + q0, nqp, K,
-                                 X.unit_hits.p + (size_t)u * P.max_pack_q * K, D.streams[k]);
+                                 X.unit_hits.p + (size_t)u * P.max_pack_q * K, X.epi[0]);
                 CK(cudaGetLastError());
                 X.launches++;
               }
@@ -1119,7 +1134,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
             const bool sl = straggler && slow > 1 && now_s() - t0 >= t_after;
             CK(cudaEventRecord(X.u_start[k], D.streams[k]));
             launch_unit(P, H, X, P.units[u], u, k, alpha, beta, thresh,
-                        (sl && o.straggler_mode == SW_STRAGGLER_SM_CAP) ? sm_share : 0);
+                        (sl && o.straggler_mode == SW_STRAGGLER_SM_CAP) ? sm_share : part_share);
             CK(cudaGetLastError());
             CK(cudaEventRecord(X.u_end[k], D.streams[k]));
             inflight[k] = u;
@@ -1157,6 +1172,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         stop_noise();
         // the int32 re-runs ran on each stream after the units that saturated; check the lists
         for (int k = 0; k < depth; k++) CK(cudaStreamSynchronize(D.streams[k]));
+        CK(cudaStreamSynchronize(X.epi[0]));
         std::vector<int32_t> novf(depth, 0), ncur(depth, 0);
         CK(cudaMemcpy(novf.data(), X.ovf_count.p, sizeof(int32_t) * depth, cudaMemcpyDeviceToHost));
         CK(cudaMemcpy(ncur.data(), X.ovf_cursor.p, sizeof(int32_t) * depth, cudaMemcpyDeviceToHost));
@@ -1473,27 +1489,30 @@ int sw_align(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t 
     CK(cudaMemcpy(dq.p, qc.data(), qc.size(), cudaMemcpyHostToDevice));
     DBuf<int8_t> dm; dm.alloc(D.id, 24 * 24);
     CK(cudaMemcpy(dm.p, M, 24 * 24, cudaMemcpyHostToDevice));
-    const int64_t kBudget = int64_t(2) << 30;   // direction bytes per batch
+    // K6 works in linear space: per pair one chunk of direction bytes (256 x n) plus the
+    // chunk checkpoints ((nch - 1) x n x 8 B); pairs are batched under 1 GiB of both
+    const int64_t kBudget = int64_t(1) << 30;
     int64_t ops_pos = 0;
     for (int32_t p0 = 0; p0 < n_pairs;) {
       std::vector<TbPair> batch;
-      int64_t dir_total = 0, ops_total = 0;
-      int32_t max_n = 1;
+      int64_t dir_total = 0, ckpt_total = 0, ops_total = 0;
       int32_t p1 = p0;
       while (p1 < n_pairs) {
         TbPair T;
         T.m = (int32_t)(qoff[query_index[p1] + 1] - qoff[query_index[p1]]);
         T.sorted = inv[db_index[p1]];
         T.n = Hd.sorted_len[T.sorted];
-        const int64_t cells = (int64_t)T.m * T.n;
-        if (!batch.empty() && dir_total + cells > kBudget) break;
+        const int64_t nch = (T.m + kTbChunk - 1) / kTbChunk;
+        const int64_t dbytes = (int64_t)kTbChunk * T.n, cbytes = std::max<int64_t>(0, nch - 1) * T.n * 8;
+        if (!batch.empty() && dir_total + ckpt_total * 8 + dbytes + cbytes > kBudget) break;
         T.q_off = qoff[query_index[p1]];
         T.pad_ = 0;
         T.dir_off = dir_total;
         T.ops_off = ops_total;
-        dir_total += cells;
+        T.ckpt_off = ckpt_total;
+        dir_total += dbytes;
+        ckpt_total += cbytes / 8;
         ops_total += T.m + T.n;
-        max_n = std::max(max_n, T.n);
         batch.push_back(T);
         p1++;
       }
@@ -1506,11 +1525,11 @@ int sw_align(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t 
       // copied back, so clear it (compute-sanitizer initcheck clean)
       CK(cudaMemset(dops.p, 0, std::max<int64_t>(ops_total, 1)));
       DBuf<TbResult> dres; dres.alloc(D.id, nb);
-      DBuf<int32_t> dborder; dborder.alloc(D.id, (size_t)nb * max_n * 2);
+      DBuf<int2> dckpt; dckpt.alloc(D.id, std::max<int64_t>(ckpt_total, 1));
       TbArgs a;
       a.qcodes = dq.p; a.packed = D.packed.p; a.groups = D.groups.p; a.matrix = dm.p;
       a.pairs = dp.p; a.dir = ddir.p; a.ops = dops.p; a.results = dres.p;
-      a.border = dborder.p; a.border_stride = max_n;
+      a.border = reinterpret_cast<int32_t *>(dckpt.p);
       a.alpha = gap_open + gap_extend; a.beta = gap_extend;
       launch_traceback(a, nb, 0);
       CK(cudaGetLastError());

@@ -1049,14 +1049,85 @@ void launch_k2(const K2Args &a, int blocks, cudaStream_t st) {
 }
 
 // ------------------------------------------------------------------------------------
-// K6: Phase 2 (P12 §II.A.2, NEXT-3): direction bytes + traceback of selected pairs.
-// One warp per pair, int32, the same wavefront as K2 (lane l owns rows [l*R, (l+1)*R) of
-// each 32*R-row chunk).  Byte per cell: bits 0-1 = H source (0 zero, 1 diagonal, 2 E,
-// 3 F), bit 2 = E extends E(i,j-1), bit 3 = F extends F(i-1,j).  The highest cell (ties:
-// smallest row, then smallest column) is found by a warp reduction; lane 0 then follows
-// the arrows back to a zero, writing ops ('M', 'I', 'D') backwards.
+// K6: Phase 2 (P12 §II.A.2, NEXT-3): the optimal local alignment of selected pairs, in
+// linear space.  One warp per pair, int32 DPX, the wavefront of K2/K3 (lane l owns rows
+// [l*R, (l+1)*R) of each chunk of 32*R = 256 rows).
+//   forward:   every chunk in order, score only; the bottom row (H, F) of each chunk is kept
+//              as a checkpoint (nch * n * 8 bytes) and the highest cell is found (ties:
+//              smallest row, then smallest column);
+//   backtrack: the chunk holding the current cell is recomputed from the checkpoint above
+//              it, for columns [0, j) only, storing one direction byte per cell (256 * n
+//              bytes, reused): bits 0-1 = H source (0 zero, 1 diagonal, 2 E, 3 F), bit 2 = E
+//              extends E(i,j-1), bit 3 = F extends F(i-1,j); lane 0 follows the arrows until
+//              they leave the chunk (upwards: the chunk above is recomputed, the H/E/F state
+//              carries over) or reach a zero, writing ops ('M', 'I', 'D') backwards.
+// Work: <= 2x the cells (each chunk is recomputed at most once, and only left of j);
+// memory: (nch * 8 + 256) bytes per database column instead of m bytes per column.
 // ------------------------------------------------------------------------------------
 constexpr int K6R = 8;
+constexpr int K6CH = 32 * K6R;   // rows per chunk
+static_assert(K6CH == kTbChunk, "host and kernel chunk heights");
+__device__ __forceinline__ void tb_chunk(const TbArgs &a, const TbPair &T, const int32_t *Ms, const uint8_t *qc,
+                                         const uint8_t *bytes, const GroupInfo &G, int gl, int ch, int ncols,
+                                         bool fwd, int &bv, int &bi, int &bj) {
+  constexpr int NEG = -(1 << 29);
+  const int lane = threadIdx.x & 31;
+  const int m = T.m, n = T.n;
+  const int nch = (m + K6CH - 1) / K6CH;
+  int2 *ckpt = reinterpret_cast<int2 *>(a.border) + T.ckpt_off;   // [nch - 1][n]
+  const int2 *top = ch > 0 ? ckpt + (size_t)(ch - 1) * n : nullptr;
+  int2 *bottom = (fwd && ch < nch - 1) ? ckpt + (size_t)ch * n : nullptr;
+  uint8_t *dir = a.dir + T.dir_off;   // [K6CH][n] (backtrack only)
+  int qr[K6R];
+#pragma unroll
+  for (int i = 0; i < K6R; i++) {
+    const int row = ch * K6CH + lane * K6R + i;
+    qr[i] = row < m ? qc[row] : kPadCode;
+  }
+  int H[K6R], E[K6R];
+#pragma unroll
+  for (int i = 0; i < K6R; i++) { H[i] = 0; E[i] = NEG; }
+  int hprev_top = 0, out_h = 0, out_f = NEG, out_c = kPadCode;
+  for (int t = 0; t < ncols + 31; t++) {
+    int in_h = __shfl_up_sync(0xffffffffu, out_h, 1);
+    int in_f = __shfl_up_sync(0xffffffffu, out_f, 1);
+    int in_c = __shfl_up_sync(0xffffffffu, out_c, 1);
+    if (lane == 0 && t < ncols) {
+      in_c = bytes[(G.word_off + (int64_t)(t >> 4) * kGroup + gl) * 16 + (t & 15)];
+      if (top) { const int2 v = top[t]; in_h = v.x; in_f = v.y; }
+      else { in_h = 0; in_f = NEG; }
+    }
+    const int col = t - lane;
+    if (col >= 0 && col < ncols) {
+      int hd = hprev_top, hup = in_h, f = in_f;
+      hprev_top = in_h;
+#pragma unroll
+      for (int i = 0; i < K6R; i++) {
+        const int row = ch * K6CH + lane * K6R + i;   // 0-based query row
+        const int eo = H[i] - a.alpha, ee = E[i] - a.beta;
+        const int e = max(ee, eo);                        // E(i,j)
+        const int fo = hup - a.alpha, fe = f - a.beta;
+        f = max(fe, fo);                                  // F(i,j)
+        const int dg = hd + Ms[qr[i] * 32 + in_c];        // diagonal
+        const int h = __vimax3_s32(max(dg, 0), e, f);     // H(i,j)
+        if (row < m) {
+          if (fwd) {
+            if (h > bv || (h == bv && h > 0 && (row + 1 < bi || (row + 1 == bi && col + 1 < bj)))) {
+              bv = h; bi = row + 1; bj = col + 1;
+            }
+          } else {
+            const int src = h == 0 ? 0 : h == dg ? 1 : h == e ? 2 : 3;
+            dir[(size_t)(lane * K6R + i) * n + col] = (uint8_t)(src | ((ee > eo) << 2) | ((fe > fo) << 3));
+          }
+        }
+        hd = H[i]; H[i] = h; E[i] = e; hup = h;
+      }
+      out_h = H[K6R - 1]; out_f = f; out_c = in_c;
+      if (lane == 31 && bottom) bottom[col] = make_int2(out_h, out_f);
+    }
+  }
+}
+
 __global__ void __launch_bounds__(32) traceback_kernel(const TbArgs a) {
   __shared__ int32_t Ms[kNCodes * 32];
   for (int k = threadIdx.x; k < kNCodes * 32; k += 32) {
@@ -1071,90 +1142,58 @@ __global__ void __launch_bounds__(32) traceback_kernel(const TbArgs a) {
   const GroupInfo G = a.groups[T.sorted / kGroup];
   const int gl = T.sorted % kGroup;
   const uint8_t *bytes = reinterpret_cast<const uint8_t *>(a.packed);
-  uint8_t *dir = a.dir + T.dir_off;
-  int32_t *border = a.border + (size_t)blockIdx.x * a.border_stride * 2;
-  constexpr int NEG = -(1 << 29);
+  const int nch = (m + K6CH - 1) / K6CH;
+  // forward pass: checkpoints + the highest cell
   int bv = 0, bi = 0, bj = 0;   // best value and its 1-based cell (0,0 = empty alignment)
-  const int nch = (m + 32 * K6R - 1) / (32 * K6R);
-  for (int ch = 0; ch < nch; ch++) {
-    int qr[K6R];
+  for (int ch = 0; ch < nch; ch++) tb_chunk(a, T, Ms, qc, bytes, G, gl, ch, n, true, bv, bi, bj);
 #pragma unroll
-    for (int i = 0; i < K6R; i++) {
-      const int row = ch * 32 * K6R + lane * K6R + i;
-      qr[i] = row < m ? qc[row] : kPadCode;
-    }
-    int H[K6R], E[K6R];
-#pragma unroll
-    for (int i = 0; i < K6R; i++) { H[i] = 0; E[i] = NEG; }
-    int hprev_top = 0, out_h = 0, out_f = NEG, out_c = kPadCode;
-    for (int t = 0; t < n + 31; t++) {
-      int in_h = __shfl_up_sync(0xffffffffu, out_h, 1);
-      int in_f = __shfl_up_sync(0xffffffffu, out_f, 1);
-      int in_c = __shfl_up_sync(0xffffffffu, out_c, 1);
-      if (lane == 0 && t < n) {
-        in_c = bytes[(G.word_off + (int64_t)(t >> 4) * kGroup + gl) * 16 + (t & 15)];
-        if (ch == 0) { in_h = 0; in_f = NEG; }
-        else { in_h = border[2 * t]; in_f = border[2 * t + 1]; }
-      }
-      const int col = t - lane;
-      if (col >= 0 && col < n) {
-        int hd = hprev_top, hup = in_h, f = in_f;
-        hprev_top = in_h;
-#pragma unroll
-        for (int i = 0; i < K6R; i++) {
-          const int row = ch * 32 * K6R + lane * K6R + i;   // 0-based query row
-          const int eo = H[i] - a.alpha, ee = E[i] - a.beta;
-          const int e = max(ee, eo);                        // E(i,j)
-          const int fo = hup - a.alpha, fe = f - a.beta;
-          f = max(fe, fo);                                  // F(i,j)
-          const int dg = hd + Ms[qr[i] * 32 + in_c];        // diagonal
-          int h = max(max(dg, e), max(f, 0));               // H(i,j)
-          if (row < m) {
-            const int src = h == 0 ? 0 : h == dg ? 1 : h == e ? 2 : 3;
-            dir[(size_t)row * n + col] = (uint8_t)(src | ((ee > eo) << 2) | ((fe > fo) << 3));
-            if (h > bv || (h == bv && h > 0 && (row + 1 < bi || (row + 1 == bi && col + 1 < bj)))) {
-              bv = h; bi = row + 1; bj = col + 1;
-            }
-          }
-          hd = H[i]; H[i] = h; E[i] = e; hup = h;
-        }
-        out_h = H[K6R - 1]; out_f = f; out_c = in_c;
-        if (lane == 31 && ch < nch - 1) { border[2 * col] = out_h; border[2 * col + 1] = out_f; }
-      }
-    }
-  }
-  // warp reduction of (value desc, row asc, column asc)
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) {
+  for (int o = 16; o > 0; o >>= 1) {   // warp reduction of (value desc, row asc, column asc)
     const int v2 = __shfl_xor_sync(0xffffffffu, bv, o), i2 = __shfl_xor_sync(0xffffffffu, bi, o),
               j2 = __shfl_xor_sync(0xffffffffu, bj, o);
     if (v2 > bv || (v2 == bv && (i2 < bi || (i2 == bi && j2 < bj)))) { bv = v2; bi = i2; bj = j2; }
   }
-  __syncwarp();
-  if (lane != 0) return;
   TbResult R;
   R.score = bv;
   int k = 0;
   char *ops_end = a.ops + T.ops_off + (m + n);   // ops written backwards from here
   int i = bi, j = bj, state = 0;                 // 0 = H, 1 = E, 2 = F
-  if (bv > 0) {
-    while (i > 0 && j > 0) {
-      const uint8_t b = dir[(size_t)(i - 1) * n + (j - 1)];
-      if (state == 0) {
-        const int src = b & 3;
-        if (src == 0) break;
-        if (src == 1) { *(--ops_end) = 'M'; k++; i--; j--; }
-        else state = src == 2 ? 1 : 2;
-      } else if (state == 1) {
-        *(--ops_end) = 'D'; k++;
-        state = (b >> 2) & 1 ? 1 : 0;
-        j--;
-      } else {
-        *(--ops_end) = 'I'; k++;
-        state = (b >> 3) & 1 ? 2 : 0;
-        i--;
+  bool stop = bv <= 0;
+  const uint8_t *dir = a.dir + T.dir_off;
+  int dummy_v = 0, dummy_i = 0, dummy_j = 0;
+  while (!stop) {
+    // recompute the chunk holding row i-1 (0-based), columns [0, j)
+    const int ch = (i - 1) / K6CH, row0 = ch * K6CH;
+    __syncwarp();
+    tb_chunk(a, T, Ms, qc, bytes, G, gl, ch, j, false, dummy_v, dummy_i, dummy_j);
+    __syncwarp();
+    __threadfence_block();
+    if (lane == 0) {
+      while (i > 0 && j > 0 && i - 1 >= row0) {
+        const uint8_t b = dir[(size_t)(i - 1 - row0) * n + (j - 1)];
+        if (state == 0) {
+          const int src = b & 3;
+          if (src == 0) { stop = true; break; }
+          if (src == 1) { *(--ops_end) = 'M'; k++; i--; j--; }
+          else state = src == 2 ? 1 : 2;
+        } else if (state == 1) {
+          *(--ops_end) = 'D'; k++;
+          state = (b >> 2) & 1 ? 1 : 0;
+          j--;
+        } else {
+          *(--ops_end) = 'I'; k++;
+          state = (b >> 3) & 1 ? 2 : 0;
+          i--;
+        }
       }
+      if (i == 0 || j == 0) stop = true;
     }
+    stop = __shfl_sync(0xffffffffu, (int)stop, 0);
+    i = __shfl_sync(0xffffffffu, i, 0);
+    j = __shfl_sync(0xffffffffu, j, 0);
+    state = __shfl_sync(0xffffffffu, state, 0);
+  }
+  if (lane != 0) return;
+  if (bv > 0) {
     R.q_begin = i; R.q_end = bi; R.d_begin = j; R.d_end = bj;
   } else {
     R.q_begin = R.q_end = R.d_begin = R.d_end = 0;

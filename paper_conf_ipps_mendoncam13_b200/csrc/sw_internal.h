@@ -138,16 +138,18 @@ struct TbPair {     // one pair of a traceback batch
   int64_t q_off;     // query codes offset
   int32_t sorted;    // database sequence (sorted order)
   int32_t pad_;
-  int64_t dir_off;   // direction bytes (m*n) offset in the batch buffer
+  int64_t dir_off;   // direction bytes of one chunk (256 * n) offset in the batch buffer
   int64_t ops_off;   // ops area (m+n bytes) offset in the batch buffer
+  int64_t ckpt_off;  // chunk checkpoints ((nch - 1) * n int2) offset in the batch buffer
 };
 struct TbResult { int32_t score, q_begin, q_end, d_begin, d_end, n_ops; };
 struct TbArgs {
   const uint8_t *qcodes; const uint4 *packed; const GroupInfo *groups; const int8_t *matrix;
   const TbPair *pairs; uint8_t *dir; char *ops; TbResult *results;
-  int32_t *border; int64_t border_stride;
+  int32_t *border;   // checkpoint rows (int2 (H, F) per column), per pair at TbPair::ckpt_off
   int32_t alpha, beta;
 };
+constexpr int kTbChunk = 256;   // K6 rows per chunk (32 lanes x 8)
 void launch_traceback(const TbArgs &a, int n_pairs, cudaStream_t st);
 
 void launch_profile(const uint8_t *qcodes, const int64_t *qoff, const QueryPair *pairs, int npairs,

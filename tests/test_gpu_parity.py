@@ -560,3 +560,23 @@ def test_k3_cluster_split(cluster):
     out = subprocess.run([sys.executable, "-c", _CLUSTER_SCRIPT % root], env=env, capture_output=True,
                          text=True, timeout=900)
     assert out.returncode == 0 and "ok" in out.stdout, (out.stdout[-2000:], out.stderr[-3000:])
+
+
+def test_traceback_gaps_across_chunks():
+    """K6 linear space: the alignment's insertion / deletion runs cross the 256-row chunk
+    boundaries where the backtrack recomputes the chunk above (the H/E/F state carries over)."""
+    r = seqgen.residues(91, 0, 900).tobytes()
+    q = r[:240] + b"W" * 40 + r[240:600] + r[620:900]   # insertion spanning row 256, deletion near 600
+    d = r[:900]
+    qs = seqgen.SeqSet.from_list([q, r[:520], b"W" * 300 + r[:300]])
+    db = seqgen.SeqSet.from_list([d, r[100:700], r[:260] + b"K" * 30 + r[260:900]])
+    D = Database(db)
+    qi = np.repeat(np.arange(3), 3).astype(np.int32)
+    di = np.tile(np.arange(3), 3).astype(np.int32)
+    al = D.align(qs, qi, di)
+    ref = oracle.pairs(qs, db, qi, di)
+    for k, a in enumerate(al):
+        assert a["score"] == ref[k]
+        _check_alignment(qs.seq(int(qi[k])).decode(), db.seq(int(di[k])).decode(), a)
+    assert "I" * 40 in al[0]["ops"]
+    D.close()

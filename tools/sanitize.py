@@ -5,8 +5,10 @@ memcheck / racecheck / synccheck / initcheck also proves the results unchanged.
   compute-sanitizer --tool racecheck python tools/sanitize.py
 
 Covers: K4 profiles, K1 (8- and 16-column-step instances: groups below and above 144
-columns), K3 (sequences above the long threshold, several chunks), K2 (planted int32
-overflow; precision routing), K5 top-k, K6 traceback, several streams with WA off/on."""
+columns), K3 (sequences above the long threshold, several chunks; SW_K3_CLUSTER=2/4 in the
+environment runs the cluster-split instance), K2 (planted int32 overflow; precision
+routing), K5u/K5m top-k and merges, the committed-segment gather/scatter of two workers,
+WA cancellation of a GPU-side straggler's replicas, K6 linear-space traceback."""
 import os
 import sys
 
@@ -48,12 +50,20 @@ def main():
         check("matrix with many overflows", D.search(qs, matrix=M, top_k=3, long_threshold=1000), ref2, 3)
         ref3 = oracle.search(qs, db, gap_open=20000, gap_extend=1)
         check("precision routing (all int32)", D.search(qs, gap_open=20000, gap_extend=1, top_k=3), ref3, 3)
-        al = D.align(qs, [1, 2, 3], [7, 100, 141])
-        for a, (qi, di) in zip(al, [(1, 7), (2, 100), (3, 141)]):
+        al = D.align(qs, [1, 2, 3, 0, 4], [7, 100, 141, 5, 143])
+        for a, (qi, di) in zip(al, [(1, 7), (2, 100), (3, 141), (0, 5), (4, 143)]):
             assert a["score"] == ref[qi, di], "traceback score"
-        print("traceback (K6): ok", flush=True)
+        print("traceback (K6, linear space): ok", flush=True)
     finally:
         D.close()
+    # two workers on the device: committed segments gathered/scattered, hit lists merged;
+    # worker 1 a GPU-side straggler with WA on (cancelled replicas)
+    D2 = Database(db, devices=[0, 0])
+    try:
+        check("two workers, straggler, WA", D2.search(qs, top_k=5, long_threshold=1000, target_unit_cells=2_000_000,
+                                                      straggler_mask=2, straggler_slowdown=8), ref, 5)
+    finally:
+        D2.close()
 
 
 if __name__ == "__main__":

@@ -15,6 +15,7 @@ ap.add_argument("--n-db", type=int, default=None)
 ap.add_argument("--streams", type=int, default=4)
 ap.add_argument("--reps", type=int, default=2)
 ap.add_argument("--unit-cells", type=int, default=0)
+ap.add_argument("--summary", action="store_true", help="print only the summary line")
 args = ap.parse_args()
 w = seqgen.make_workload(args.config, n_db=args.n_db)
 D = Database(w.db, devices=[0])
@@ -26,7 +27,7 @@ for _ in range(args.reps + 1):
         best = st
 print(f"{args.config} n_db={w.db.n}: {best['gcups']:.1f} GCUPS, device {1e3 * best['seconds_device']:.2f} ms, "
       f"units {best['n_units']}, overflow pairs {best['n_overflow_pairs']}, launches {best['kernel_launches']}")
-for e in sorted(best["unit_log"], key=lambda e: (e["stream"], e["dev_t0"])):
+for e in ([] if args.summary else sorted(best["unit_log"], key=lambda e: (e["stream"], e["dev_t0"]))):
     print(f"  stream {e['stream']} unit {e['unit']:4d} kind {'K1' if e['kind'] == 0 else 'K3'} pack {e['pair']:3d} "
           f"[{e.get('b0')},{e.get('b1')}) C={e.get('cluster')} "
           f"dev {e['dev_t0']:8.2f} -> {e['dev_t1']:8.2f} ms ({e['device_ms']:7.2f}) cells {e['cells']:.3e} "

@@ -47,14 +47,19 @@ def main():
     ap.add_argument("--policies", default="pss,ss")
     ap.add_argument("--scenarios", default="homogeneous,straggler,local_load_midrun")
     ap.add_argument("--out", default=None)
+    ap.add_argument("--partition", action="store_true",
+                    help="each worker gets n_SM / workers SMs (worker_sms): the workers behave like separate GPUs")
     ap.add_argument("--unit-cells", type=int, default=0,
                     help="target_unit_cells (0 = auto; 2**62 = the paper's very coarse tasks, one per pack)")
     args = ap.parse_args()
     w = seqgen.make_workload(args.config)
     gold = json.load(open(os.path.join(ROOT, "tests", "golden", "oracle_digests.json"))).get(args.config)
     D = Database(w.db, devices=[0] * args.workers)
+    import torch
+    n_sm = torch.cuda.get_device_properties(0).multi_processor_count
+    wsms = n_sm // args.workers if args.partition else 0
     straggler = 1 << (args.workers - 1)
-    base = D.search(w.queries, top_k=10, streams=args.streams)   # warm-up + reference scores
+    base = D.search(w.queries, top_k=10, streams=args.streams, worker_sms=wsms)   # warm-up + reference
     ref = digest(base.scores)
     if gold:
         assert ref == gold["sha256_scores"], "scores differ from the oracle's digest"
@@ -71,7 +76,7 @@ def main():
                     r = D.search(w.queries, top_k=10, streams=args.streams, policy=policy, workload_adjust=wa,
                                  straggler_mask=mask, straggler_slowdown=args.slowdown,
                                  straggler_after_ms=after, straggler_mode=args.mode,
-                                 target_unit_cells=args.unit_cells)
+                                 target_unit_cells=args.unit_cells, worker_sms=wsms)
                     assert digest(r.scores) == ref, "scores differ across schedules"
                     st = r.stats
                     if best is None or st["seconds_device"] < best["seconds_device"]:
@@ -117,8 +122,9 @@ def main():
             print(f"WA {name}/{policy}: {s['gcups_gain_pct']:+.1f} % GCUPS, makespan {s['makespan_off']:.3f} -> "
                   f"{s['makespan_on']:.3f} s, tail {s['tail_off']:.3f} -> {s['tail_on']:.3f} s")
     out = dict(config=args.config, workers=args.workers, streams=args.streams, slowdown=args.slowdown,
-               mode=args.mode, unit_cells=args.unit_cells, oracle_digest_checked=bool(gold),
-               note="P workers share one B200 (separate streams/replicas); the straggler is the last worker",
+               mode=args.mode, unit_cells=args.unit_cells, oracle_digest_checked=bool(gold), worker_sms=wsms,
+               note="P workers share one B200 (separate streams/replicas); the straggler is the last worker"
+                    + (f"; each worker is capped to {wsms} SMs (worker_sms), i.e. P emulated GPUs" if wsms else ""),
                summary=summary, runs=rows)
     if args.out:
         with open(args.out, "w") as f:
