@@ -1,5 +1,6 @@
 """The seeded input generator: determinism, shapes and the recipe of DESIGN.md §4."""
 import numpy as np
+import pytest
 
 import seqgen
 
@@ -60,3 +61,24 @@ def test_seqset_indexed_format():
     s = seqgen.SeqSet.from_list(["AC", "", "WWW"])
     assert s.n == 3 and s.offsets.tolist() == [0, 2, 2, 5] and s.max_len == 3
     assert s.seq(2) == b"WWW" and s.seq(1) == b""
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3", "C5", "RAT", "MOUSE", "C5@256", "C4"])
+def test_generated_inputs_match_committed_digests(cfg):
+    """The seeded inputs behind tests/golden/oracle_digests.json are byte-identical on this
+    host (the generator's length draws use libm; a different rounding fails here, loudly)."""
+    import hashlib
+    import json
+    import os
+    import numpy as np
+    g = json.load(open(os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden", "input_digests.json")))[cfg]
+
+    def dig(s):
+        h = hashlib.sha256()
+        h.update(np.ascontiguousarray(s.offsets, dtype="<i8").tobytes())
+        h.update(np.ascontiguousarray(s.residues, dtype=np.uint8).tobytes())
+        return h.hexdigest()
+    name, _, n_db = cfg.partition("@")
+    w = seqgen.make_workload(name, n_db=int(n_db) if n_db else None)
+    assert (w.queries.n, w.db.n) == (g["n_queries"], g["n_db"])
+    assert dig(w.queries) == g["queries"] and dig(w.db) == g["db"]
