@@ -482,6 +482,20 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
   // drop empty units (e.g. all-empty queries still produce valid zero scores: keep them
   // so that every pair gets written, but they must have cells > 0 for the scheduler)
   for (auto &u : P.units) u.cells = std::max<int64_t>(u.cells, 1);
+  // mixed regime (K1 carries most cells; K3 units overlap K1 units): a K3 unit too small for
+  // its stream's share of the resident K3 CTAs holds a stream for its longest pair's whole
+  // critical path; split its chunks over clusters of 4 (C4 at 1/8 of its database, 64
+  // sequence blocks per unit: 5.82 -> 6.17 TCUPS; at full size, 148 blocks per unit, C = 4
+  // costs 2 %)
+  {
+    static const int forced = [] { const char *e = getenv("SW_K3_CLUSTER"); return e ? atoi(e) : 0; }();
+    if (forced == 0 && k3_cluster == 1 && o.target_unit_cells <= 0 && k3_slots > 0)
+      for (Unit &u : P.units)
+        if (u.kind == kUnitIntra) {
+          const double ratio = (double)((u.b1 - u.b0 + kK3Warps - 1) / kK3Warps) * depth / k3_slots;
+          if (ratio < 0.75) u.cluster = 4;
+        }
+  }
   // LPT by expected duration: intra-task (long-sequence) units first -- each warp walks a
   // whole long pair, so they have the longest latency -- then inter-task units by work.
   // A small K3 unit (fewer sequences than one block per SM) is interleaved with the largest
