@@ -335,10 +335,17 @@ def main():
         bytes_per_cell, ncu = load_traffic()
         cells_per_launch = alone["cells_k1"] / k1_launches if k1_launches else None
         traffic = (bytes_per_cell * cells_per_launch) if (bytes_per_cell and cells_per_launch) else None
-        roofline = {"bound": "alu", "achieved": k1_alone, "peak": peak, "unit": "GCUPS",
-                    "frac": (k1_alone / peak) if k1_alone else None, "traffic": traffic,
-                    "kernel": "k1_kernel (inter-task DP, the dominant kernel): cells per launch / average "
-                              "launch duration, each launch alone on the GPU (1 stream)",
+        # the dominant kernel: K1 unless long sequences carry most cells (C5: K3)
+        k3_dominant = alone["cells_k3"] > alone["cells_k1"]
+        dom = k3_alone if k3_dominant else k1_alone
+        if k3_dominant:
+            traffic = None   # the committed ncu capture is of K1
+        roofline = {"bound": "alu", "achieved": dom, "peak": peak, "unit": "GCUPS",
+                    "frac": (dom / peak) if dom else None, "traffic": traffic,
+                    "kernel": ("k3_kernel (intra-task DP, the dominant kernel for this workload)" if k3_dominant else
+                               "k1_kernel (inter-task DP, the dominant kernel)") +
+                              ": cells per launch / average launch duration, each launch alone on the GPU (1 stream)",
+                    "k1_alone_gcups": k1_alone,
                     "k1_launches": k1_launches, "k1_cells_per_launch": cells_per_launch,
                     "k1_avg_launch_ms": (1e3 * alone["kernel_seconds_k1"] / k1_launches) if k1_launches else None,
                     "k3_alone_gcups": k3_alone,
