@@ -127,6 +127,7 @@ struct DevSearch {
   DBuf<int32_t> k2_border;
   DBuf<int32_t> abort_dev;      // per-unit WA cancellation flags (device memory)
   DBuf<int32_t> progress;       // per-unit progress counters (K1 groups / K3 sequence-chunks)
+  DBuf<int32_t> gclaim;         // per-unit K1 group claim counters
   int32_t *abort_d = nullptr;
   int32_t *one_h = nullptr;      // pinned constant 1, source of the cancellation copies
   int32_t *ovf_seen_h = nullptr; // pinned [kMaxStreams]: ovf_count copied after each unit
@@ -613,6 +614,7 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     a.slot_busy = D.slot_busy.p;
     a.abort_flag = S.abort_d + uidx;
     a.progress = S.progress.p + uidx;
+    a.gclaim = S.gclaim.p + uidx;
     a.na = na; a.nb = nbm;
     launch_k1(a, U.b1 - U.b0, db.groups[U.b1 - 1].ncols, P.pairs[U.pair].rows_padded, st,
               sm_cap > 0 ? std::min(sm_cap, D.n_sm) : D.n_sm);
@@ -874,6 +876,8 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       CK(cudaMemset(X.abort_dev.p, 0, sizeof(int32_t) * nu));
       X.progress.ensure(D.id, nu);
       CK(cudaMemset(X.progress.p, 0, sizeof(int32_t) * nu));
+      X.gclaim.ensure(D.id, nu);
+      CK(cudaMemset(X.gclaim.p, 0, sizeof(int32_t) * nu));
       X.abort_d = X.abort_dev.p;
       X.cancelled.assign(nu, 0);
       if (K > 0) {

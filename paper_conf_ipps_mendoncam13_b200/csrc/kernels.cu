@@ -213,19 +213,32 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   const int nb = (rows + BAND - 1) / BAND;
   const uint32_t koff = pk2(kOff), na = a.na, nbeta = a.nb;
   const int32_t *gprof = a.prof + P.prof_off;
-  // this block streams through groups gfirst, gfirst + gridDim.x, ... of the unit without
-  // draining the warp pipeline between them
-  const int gfirst = a.g0 + blockIdx.x, gend = a.g0 + a.n_groups, gstride = gridDim.x;
-  int total = 0;
-  for (int g = gfirst; g < gend; g += gstride) total += nb * ((a.groups[g].ncols + T - 1) / T);
+  // this block streams through the unit's groups without draining the warp pipeline between
+  // them, claiming them dynamically from the unit's counter: the groups are sorted by
+  // decreasing width, so claims go widest first and a block that took a wide group takes
+  // fewer (list scheduling; a static stride left the widest unit of each pack at 0.77 of
+  // the others).  The block's r-th group is gring[r & 3].  The next group is claimed late,
+  // when warp 0 enters the current group's second-to-last band (at the group's start when
+  // it has <= 2 bands), so a block claims only when it is about to need it, and every warp
+  // (lagging warp 0 by < one band) reads a slot written at least one band earlier.
+  const int gend = a.g0 + a.n_groups;
+  __shared__ int gring[4];
+  auto claim = [&]() -> int {
+    const int i = atomicAdd(a.gclaim, 1);
+    return i < a.n_groups ? a.g0 + i : gend;
+  };
 
   uint2 *border = nullptr;
-  if (nb > 1 && threadIdx.x == 0) {   // a border-row slot of this SM (released at exit)
-    const int base = (int)smid() * a.slots_per_sm;
-    int k = 0;
-    for (;; k = (k + 1) % a.slots_per_sm)
-      if (atomicCAS(&a.slot_busy[base + k], 0, 1) == 0) break;
-    slot_s = base + k;
+  if (threadIdx.x == 0) {
+    gring[0] = claim();
+    gring[1] = (nb <= 2 && gring[0] < gend) ? claim() : gend;   // nb > 2: claimed at band nb-2
+    if (nb > 1 && gring[0] < gend) {   // a border-row slot of this SM (released at exit)
+      const int base = (int)smid() * a.slots_per_sm;
+      int k = 0;
+      for (;; k = (k + 1) % a.slots_per_sm)
+        if (atomicCAS(&a.slot_busy[base + k], 0, 1) == 0) break;
+      slot_s = base + k;
+    }
   }
   auto load_band = [&](int b, int slot) {
     uint32_t *dst = prof_s + slot * kNCodes * S;
@@ -238,17 +251,20 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   if (nb > 1) load_band(1, 1);
   for (int k = threadIdx.x; k < T * 32; k += W * 32) kin[k] = make_uint2(koff, koff);
   __syncthreads();
+  const int gfirst = gring[0];
+  if (gfirst >= gend) return;   // nothing left for this block (uniform: read after the barrier)
   if (nb > 1) border = a.border + (size_t)slot_s * a.border_slot_cols * 32;
 
   // block-uniform tracker of warp 0's band starts: the profile of global band B+1 is
   // loaded into slot (B+1)&1 when warp W-1 leaves band B-1, i.e. W-1 steps after warp 0
   // starts band B (every band has nt >= W+1 steps, so warp 0 needs it later)
-  int t_g = gfirst, t_band = 0, t_nt = (a.groups[gfirst].ncols + T - 1) / T, t_start = 0, t_B = 0;
+  int t_r = 0, t_g = gfirst, t_band = 0, t_nt = (a.groups[gfirst].ncols + T - 1) / T, t_start = 0, t_B = 0;
+  int end_step = INT32_MAX;   // set when warp 0 runs out of groups: + W - 1 drains the pipeline
   int rl_step = -1, rl_band = 0, rl_slot = 0;
 
   // per-warp iterator over (group, band, tile); the queries of this warp's current slice
   // (per half) and the start mask of the slice below it
-  int g = gfirst, gk = 0, band = 0, tile = 0, gband = 0;
+  int g = gfirst, gr = 0, gk = 0, band = 0, tile = 0, gband = 0;
   int cq_lo = -1, cq_hi = -1;
   uint32_t omask = 0;
   const int nslices = P.rows_padded / 16;
@@ -259,34 +275,37 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
   uint32_t H[K], E[K];
   uint32_t best = koff, hprev_top = koff;
 
-  const int steps = total + W - 1;
-  for (int s = 0; s < steps; s++) {
-    if (nb > 2) {
-      if (s == t_start + t_nt) {   // warp 0 enters its next band at this step
-        t_start += t_nt;
-        t_B++;
-        if (++t_band == nb) {
-          t_band = 0;
-          t_g += gstride;
-          if (t_g < gend) t_nt = (a.groups[t_g].ncols + T - 1) / T;
-        }
-        // the band after this one: rows (t_band+1) mod nb, slot (t_B+1)&1
-        if (t_B + 1 >= 2) {
-          const bool last_overall = t_g >= gend || (t_band == nb - 1 && t_g + gstride >= gend);
-          if (!last_overall) {
-            rl_step = t_start + W - 1;
-            rl_band = t_band + 1 == nb ? 0 : t_band + 1;
-            rl_slot = (t_B + 1) & 1;
-          }
-        }
+  for (int s = 0; s < end_step; s++) {
+    if (s == t_start + t_nt) {   // warp 0 enters its next band at this step
+      t_start += t_nt;
+      t_B++;
+      if (++t_band == nb) {
+        t_band = 0;
+        t_g = gring[(++t_r) & 3];   // claimed at least one band ago
+        if (t_g < gend) t_nt = (a.groups[t_g].ncols + T - 1) / T;
+        else end_step = s + W - 1;
       }
-      if (s == rl_step) {
-        load_band(rl_band, rl_slot);
-        __syncthreads();
+      // claim the group after this one (only thread 0 writes; read no earlier than the
+      // next band transition)
+      if (threadIdx.x == 0 && t_g < gend && t_band == (nb > 2 ? nb - 2 : 0) && (nb > 2 || t_r > 0))
+        gring[(t_r + 1) & 3] = claim();
+      // the band after this one: rows (t_band+1) mod nb, slot (t_B+1)&1 (nb > 2: the
+      // group's bands rotate through two profile slots)
+      if (nb > 2 && t_B + 1 >= 2) {
+        const bool last_overall = t_g >= gend || (t_band == nb - 1 && gring[(t_r + 1) & 3] >= gend);
+        if (!last_overall) {
+          rl_step = t_start + W - 1;
+          rl_band = t_band + 1 == nb ? 0 : t_band + 1;
+          rl_slot = (t_B + 1) & 1;
+        }
       }
     }
+    if (nb > 2 && s == rl_step) {
+      load_band(rl_band, rl_slot);
+      __syncthreads();
+    }
     const int e = s - warp;
-    if (e >= 0 && e < total) {
+    if (e >= 0 && g < gend) {
       if (tile == 0) {
 #pragma unroll
         for (int i = 0; i < K; i++) { H[i] = koff; E[i] = koff; }
@@ -397,7 +416,7 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
           best = koff;
           cq_lo = cq_hi = -1;
           gk++;
-          g += gstride;
+          g = gring[(++gr) & 3];
           if (g < gend) {
             G = a.groups[g];
             nt = (G.ncols + T - 1) / T;

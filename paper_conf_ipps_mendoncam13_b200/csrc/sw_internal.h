@@ -101,6 +101,7 @@ struct K1Args {
   uint2 *border; int32_t border_slot_cols; int32_t slots_per_sm; int32_t *slot_busy;
   const volatile int32_t *abort_flag; // WA cancellation flag of the unit (polled in the loop)
   int32_t *progress;                 // unit's counter: groups completed (atomicAdd per block)
+  int32_t *gclaim;                   // unit's counter: groups claimed by its blocks (zeroed)
   uint32_t na, nb;                   // packed -alpha, -beta
 };
 struct K3Args {   // sequences [l0,l1) in sorted order (the long groups)

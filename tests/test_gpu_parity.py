@@ -237,16 +237,17 @@ def _digest(cfg, scores):
 
 def test_wa_beats_a_gpu_side_straggler():
     """workload adjustment against a genuinely slow GPU.  Two workers share the
-    B200; worker 1's DP kernels get ceil(148/24) SMs.  C2 with the paper's coarse tasks (one per
-    pack), one stream per worker: the slow worker takes its first task before the master knows
-    its rate, so without WA that task decides the end.  With WA on, the fast worker re-executes the
+    B200; worker 1's DP kernels get one SM's worth of blocks.  C2 with the paper's coarse tasks
+    (one per pack and kernel kind), one stream per worker: the slow worker takes its first task
+    before the master knows its rate, and that task outlives all the others, so without WA it
+    decides the end.  With WA on, the fast worker re-executes the
     straggler's last unit, the straggler's replica is cancelled IN its kernel (abort flag polled
     in the group/chunk loops) and abandoned with the cells it really computed; makespan and tail
     drop.  Both runs are bit-exact against the oracle's C2 digest."""
     w = seqgen.make_workload("C2")
     D = Database(w.db, devices=[0, 0])
-    kw = dict(top_k=10, target_unit_cells=2**62, straggler_mask=0b10, straggler_slowdown=24,
-              straggler_mode="sm_cap", streams=1, long_threshold=-1)
+    kw = dict(top_k=10, target_unit_cells=2**62, straggler_mask=0b10, straggler_slowdown=148,
+              straggler_mode="sm_cap", streams=1)
     D.search(w.queries, **kw)   # warm-up (lazy module loading, buffers)
     on = D.search(w.queries, workload_adjust=True, **kw)
     ok_on, e = _digest("C2", on.scores)
