@@ -1026,7 +1026,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         std::vector<int> completed_wait(depth, 0), slowed(depth, 0);
         std::vector<int32_t> k2_upto(depth, 0);   // saturated pairs handed to K2 per stream
         bool done = false, changed = true;
-        double last_req = 0;
+        double last_req = 0, req_gap = 2e-3;
         std::vector<double> stream_rate(depth, 0.0);
         int32_t buf[64];
         while (true) {
@@ -1107,6 +1107,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
             inflight[k] = -1;
             completed_wait[k] = 0;
             progressed = changed = true;
+            req_gap = 2e-3;
             // epilogue of a completed unit on the worker's high-priority epilogue stream, so
             // the stream goes straight on to its next unit: the int32 re-run of what the
             // stream's units saturated (K2), then (committed) the unit's top-k (K5u).  Both
@@ -1169,13 +1170,18 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
             int32_t r = 0;
             const double tq = now_s();
             if (n_inflight == 0) {
-              r = sreq_wait(wid, tq, buf, 64, 0.005);
+              // the master answers as soon as its table changes; the timeout only re-tests
+              // WA's time-dependent ETA condition (WA off: nothing to re-test)
+              r = sreq_wait(wid, tq, buf, 64, o.workload_adjust ? 0.005 : 0.25);
               last_req = tq;
               changed = false;
-            } else if (changed || tq - last_req > 2e-3) {
+            } else if (changed || tq - last_req > req_gap) {
               r = sreq(wid, tq, buf, 64);
               last_req = tq;
               changed = false;
+              // nothing granted while units still run here: ask again later and later
+              // (2 ms doubling to 64 ms; a completion or a grant resets it)
+              req_gap = r == 0 ? std::min(0.064, 2 * req_gap) : 2e-3;
             }
             if (r < 0) done = true;
             else {
