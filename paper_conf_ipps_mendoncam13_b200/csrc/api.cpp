@@ -896,7 +896,10 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       {
         int lo = 0, hi = 0;
         CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
-        if (!X.noise_st) CK(cudaStreamCreateWithPriority(&X.noise_st, cudaStreamNonBlocking, hi));
+        // (the local-load stream is created only when a worker emulates one: every stream
+        // takes one of the GPU's hardware work queues)
+        if (!X.noise_st && o.straggler_mode == SW_STRAGGLER_NOISE && o.straggler_mask)
+          CK(cudaStreamCreateWithPriority(&X.noise_st, cudaStreamNonBlocking, hi));
         while (X.epi.empty()) {   // one per worker (the hardware work queues are limited)
           cudaStream_t e;
           CK(cudaStreamCreateWithPriority(&e, cudaStreamNonBlocking, hi));

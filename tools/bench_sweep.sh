@@ -3,7 +3,7 @@
 # K1-alone roofline fraction.  Usage: tools/bench_sweep.sh "base" "w2 SW_K1_WAVES=2" ...
 for spec in "$@"; do
   label=${spec%% *}; envs=${spec#* }; [ "$envs" = "$spec" ] && envs=""
-  line=$(env $envs python bench.py --steps ${STEPS:-3} --warmup 2 --e2e-steps 0 --no-cpu-baseline 2>/dev/null | tail -1)
+  line=$(env $envs python bench.py --steps ${STEPS:-3} --warmup 2 --e2e-steps 0 --no-cpu-baseline ${BENCH_ARGS:-} 2>/dev/null | tail -1)
   python - "$label" "$line" <<'PY'
 import json, sys
 d = json.loads(sys.argv[2]); r = d["roofline"]
