@@ -202,6 +202,7 @@ inline DevSearch::~DevSearch() {
 struct sw_db {
   sw::PackedDB host;
   std::vector<std::unique_ptr<sw::Device>> devs;
+  std::vector<char> peer_ok;     // [i * n + j]: device of worker i can read worker j's memory
   std::atomic<int> busy{0};
   std::string unit_log;
   std::string sched_log;
@@ -724,16 +725,20 @@ int sw_db_create(const sw_seqset *dbs, const int *devices, int n_devices, sw_db 
       if (!H.sorted_len.empty()) CK(cudaMemcpy(D->sorted_len.p, H.sorted_len.data(), sizeof(int32_t) * H.sorted_len.size(), cudaMemcpyHostToDevice));
       db->devs.push_back(std::move(D));
     }
-    // the merge copies committed units' scores and hits between GPUs: direct over NVLink
-    for (int a : devs)
-      for (int b : devs) {
-        if (a == b) continue;
+    // the merge reads the other GPUs' committed scores directly over NVLink (peer access)
+    const size_t nd_ = devs.size();
+    db->peer_ok.assign(nd_ * nd_, 0);
+    for (size_t i = 0; i < nd_; i++)
+      for (size_t j = 0; j < nd_; j++) {
+        const int a = devs[i], b = devs[j];
+        if (a == b) { db->peer_ok[i * nd_ + j] = 1; continue; }
         int ok = 0;
         if (cudaDeviceCanAccessPeer(&ok, a, b) == cudaSuccess && ok) {
           CK(cudaSetDevice(a));
           const cudaError_t e = cudaDeviceEnablePeerAccess(b, 0);
           if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
           else CK(e);
+          db->peer_ok[i * nd_ + j] = 1;
         }
       }
     *out = db.release();
@@ -1252,7 +1257,9 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
           launch_fill(dst, nsc, -1, s0);
           launch_seg_copy(X.scores, dst, nd, D.perm.p, X.segs.p, (int)segs.size(), 2, s0);
           X.launches += segs.empty() ? 1 : 2;
-        } else if (!segs.empty()) {
+        } else if (!segs.empty() && !db->peer_ok[(size_t)w]) {
+          // device 0 cannot read this GPU's memory: pack the committed pairs densely for a
+          // (host-staged) peer copy
           X.compact.ensure(D.id, std::max<int64_t>(seg_total, 1));
           launch_seg_copy(X.scores, X.compact.p, nd, D.perm.p, X.segs.p, (int)segs.size(), 0, s0);
           X.launches++;
@@ -1311,9 +1318,10 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
     }
 
     // ---------------- merge (the paper's "the slaves send their results to the master, that
-    // merges them", P16 §IV).  In-process with several GPUs: every other GPU's committed
-    // units' scores (packed densely on that GPU) and its top-k lists are copied to the first
-    // GPU over NVLink (peer access enabled at sw_db_create) and merged there (scatter + K5m).
+    // merges them", P16 §IV).  In-process with several GPUs: a kernel on the first GPU reads
+    // every other GPU's committed units' scores over NVLink (peer access enabled at
+    // sw_db_create; without it they are packed densely and copied) and the top-k lists are
+    // copied and merged (K5m).
     // Multi-process: each rank keeps its committed pairs and hits; the binding gathers the
     // hits (NCCL) and merges them with sw_merge_hits.
     DevSearch &X0 = *S[0];
@@ -1336,14 +1344,20 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         if (sg_.empty()) continue;
         const int64_t total = sg_.back().off + (sg_.back().s1 - sg_.back().s0);
         CK(cudaStreamWaitEvent(s0, S[w]->ev_data, 0));
-        stage.ensure(dev0, std::max<int64_t>(total, 1));
-        CK(cudaMemcpyPeerAsync(stage.p, dev0, S[w]->compact.p, S[w]->D->id, sizeof(int32_t) * total, s0));
-        peer_bytes += sizeof(int32_t) * total;
         segs0.ensure(dev0, sg_.size());
         CK(cudaMemcpyAsync(segs0.p, sg_.data(), sizeof(SegInfo) * sg_.size(), cudaMemcpyHostToDevice, s0));
-        launch_seg_copy(stage.p, X0.scores, nd, X0.D->perm.p, segs0.p, (int)sg_.size(), 1, s0);
+        if (db->peer_ok[(size_t)w]) {
+          // one kernel on device 0 reads worker w's committed pairs over NVLink (peer loads)
+          // and writes them into the result: no staging buffer, no separate copy
+          launch_seg_copy(S[w]->scores, X0.scores, nd, X0.D->perm.p, segs0.p, (int)sg_.size(), 2, s0);
+        } else {
+          stage.ensure(dev0, std::max<int64_t>(total, 1));
+          CK(cudaMemcpyPeerAsync(stage.p, dev0, S[w]->compact.p, S[w]->D->id, sizeof(int32_t) * total, s0));
+          launch_seg_copy(stage.p, X0.scores, nd, X0.D->perm.p, segs0.p, (int)sg_.size(), 1, s0);
+        }
+        peer_bytes += sizeof(int32_t) * total;
         X0.launches++;
-        // the staging buffer is reused by the next worker: keep the copies ordered on s0
+        // segs0 / the staging buffer are reused by the next worker: ordered on s0
       }
       if (K > 0) {
         X0.all_hits.ensure(dev0, (size_t)nW * nq * K);

@@ -186,3 +186,27 @@ def test_bad_arguments():
         Scheduler(2, [1, 0])
     S = Scheduler(1, [])
     assert S.request(0, 0.0) is None
+
+
+def test_failed_worker_tasks_return_to_ready():
+    """R22: a worker that disappears (its connection closed) is failed: each unfinished task it
+    held that nobody else runs goes back to READY and is granted before the remaining ready
+    tasks; the failed worker gets nothing more, so the search completes with WA off too."""
+    from paper_conf_ipps_mendoncam13_b200 import Scheduler
+    S = Scheduler(2, [10, 10, 10, 10], policy="ss", wa=False)
+    assert S.request(0, 0.0) == [0]
+    assert S.request(1, 0.0) == [1]
+    S.fail_worker(1, 0.1)
+    assert S.state(1) == 0 and S.replicas(1) == 0          # READY again
+    assert S.request(1, 0.2) is None                        # a failed worker gets nothing
+    S.report(0, 0.3, 10, 0.1)
+    assert S.complete(0, 0, 0.3)
+    assert S.request(0, 0.3) == [1]                         # the re-queued task first
+    for u in (1,):
+        assert S.complete(0, u, 0.4)
+    got = S.request(0, 0.4) + S.request(0, 0.5)
+    assert sorted(got) == [2, 3]
+    for u in got:
+        assert S.complete(0, u, 0.6)
+    assert S.request(0, 0.7) is None
+    assert [e["ev"] for e in S.log()].count("F") == 1

@@ -58,7 +58,8 @@ for n in [int(x) for x in args.ns.split(",")]:
 g1 = rows[0]["gcups"]
 for row in rows:
     row["efficiency"] = row["gcups"] / (row["n"] * g1) if rows[0]["n"] == 1 else None
-    print(f"N={row['n']}: {row['gcups']:.1f} GCUPS, efficiency {row['efficiency']:.3f}, tail {row['tail_s']:.3f} s, "
+    eff = f"{row['efficiency']:.3f}" if row["efficiency"] is not None else "n/a"
+    print(f"N={row['n']}: {row['gcups']:.1f} GCUPS, efficiency {eff}, tail {row['tail_s']:.3f} s, "
           f"merge moved {row['peer_bytes'] / 1e6:.1f} MB, digest {row['digest_ok']}", flush=True)
 if args.out:
     json.dump(dict(config=args.config, sms_per_worker=sms, streams=args.streams, n_sm=n_sm,
