@@ -140,7 +140,7 @@ struct DevSearch {
   std::vector<char> cancelled;
   // data plane: per-unit top-k of committed units, merged per worker
   DBuf<int32_t> pack_q;          // queries of each pack (flattened, Plan::pack_q_off)
-  DBuf<int2> unit_hits;          // [units][max_pack_q][k]
+  DBuf<int2> unit_hits;          // [units][max_unit_q][k]
   DBuf<int2> worker_hits;        // [nq][k] top-k over this worker's committed units
   DBuf<int2> all_hits;           // device 0: [workers][nq][k]
   DBuf<int32_t> list_tab;        // merge tables: list_off[nq+1] then list_idx
@@ -228,6 +228,7 @@ struct Plan {
   std::vector<int32_t> pack_q;         // queries of each pack, flattened (ascending ids)
   std::vector<int32_t> pack_q_off;     // [packs + 1]
   int32_t max_pack_q = 1;              // most queries in one pack
+  int32_t max_unit_q = 1;              // most queries in one unit (a unit spans npk packs)
   uint64_t hash = 0;                   // FNV-1a of the unit table (multi-process handshake)
 };
 // sorted-sequence range [s0, s1) of a unit's pairs (K1: whole groups; K3: long sequences)
@@ -422,24 +423,16 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
       const int64_t per_pack = ((int64_t)n_workers * depth + n_packs - 1) / n_packs;
       if (per_pack > 1) k3_target = std::max<int64_t>(1, std::min<int64_t>(k3_target, (long_cells + per_pack - 1) / per_pack));
     }
-    // clustered K3 (k3_cluster > 1): each pack's long sequences in just enough units for
-    // every stream of every worker to get one (a launch holds one stream's share of the GPU)
-    int32_t k3_unit_seqs = 0;
-    if (k3_cluster > 1) {
-      const int64_t per_pack = std::max<int64_t>(1, ((int64_t)n_workers * depth + n_packs - 1) / n_packs);
-      k3_unit_seqs = (int32_t)std::max<int64_t>(kK3Warps, (P.n_long_seqs + per_pack - 1) / per_pack);
-      k3_unit_seqs = (k3_unit_seqs + kK3Warps - 1) / kK3Warps * kK3Warps;
-    }
-    for (int32_t s = 0; s < P.n_long_seqs;) {
+    // (clustered plans: K3 units span every pack, built after this loop)
+    for (int32_t s = 0; s < P.n_long_seqs && k3_cluster == 1;) {
       int32_t e = s;
       int64_t cells = 0, work = 0;
-      while (e < P.n_long_seqs && (k3_unit_seqs > 0 ? e - s < k3_unit_seqs
-                                                     : (cells < k3_target || e == s || (e - s) % kK3Warps))) {
+      while (e < P.n_long_seqs && (cells < k3_target || e == s || (e - s) % kK3Warps)) {
         cells += rows_eff * db.sorted_len[e];
         work += (int64_t)qp.rows_padded * db.sorted_len[e];
         e++;
       }
-      P.units.push_back({kUnitIntra, p, s, e, cells, work, k3_cluster, 0});
+      P.units.push_back({kUnitIntra, p, s, e, cells, work, 1, 1});
       P.max_k3_seqs = std::max(P.max_k3_seqs, e - s);
       s = e;
     }
@@ -476,9 +469,35 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
           work += rows_k1 * db.groups[e].ncols * kGroup;
           e++;
         }
-        P.units.push_back({kUnitInter, p, g, e, cells, work, 1, 0});
+        P.units.push_back({kUnitInter, p, g, e, cells, work, 1, 1});
         g = e;
       }
+    }
+  }
+  // clustered plans (long sequences carry the work, one worker's share is small): a K3 unit is
+  // every pack x a contiguous range of sequence blocks, cut at equal cells (units = workers x
+  // streams, or 4x an explicit target).  Its clusters claim (pack, block) tasks longest first,
+  // so every pack's longest pairs start at once and the streams' units take about as long --
+  // per-pack units finished in launch order (C5 at 1/8: 27 / 34 / 46 / 52 ms)
+  if (k3_cluster > 1 && P.n_long_seqs > 0 && !P.pairs.empty()) {
+    int64_t rows_all = 0, rows_pad = 0, long_res = 0;
+    for (size_t p = 0; p < P.pairs.size(); p++) { rows_all += P.real_rows[p]; rows_pad += P.pairs[p].rows_padded; }
+    for (int32_t s = 0; s < P.n_long_seqs; s++) long_res += db.sorted_len[s];
+    const int64_t k3_cells = rows_all * long_res;
+    const int64_t t4 = target > INT64_MAX / 4 ? INT64_MAX : 4 * target;
+    const int64_t unit_target = o.target_unit_cells > 0
+        ? t4 : std::max<int64_t>(1, k3_cells / std::max(1, n_workers * std::max(1, o.streams_per_device)));
+    for (int32_t s = 0; s < P.n_long_seqs;) {
+      int32_t e = s;
+      int64_t cells = 0, work = 0;
+      while (e < P.n_long_seqs && (cells < unit_target || e == s || (e - s) % kK3Warps)) {
+        cells += rows_all * db.sorted_len[e];
+        work += rows_pad * db.sorted_len[e];
+        e++;
+      }
+      P.units.push_back({kUnitIntra, 0, s, e, cells, work, k3_cluster, (int32_t)P.pairs.size()});
+      P.max_k3_seqs = std::max(P.max_k3_seqs, e - s);
+      s = e;
     }
   }
   // drop empty units (e.g. all-empty queries still produce valid zero scores: keep them
@@ -507,11 +526,21 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
   auto small3 = [](const Unit &u) {
     return interleave && u.kind == kUnitIntra && u.cluster == 1 && u.b1 - u.b0 < kK3UnitSeqs;
   };
+  auto may_ovf = [&](const Unit &u) {
+    for (int32_t p = u.pair; p < u.pair + u.npk; p++)
+      if (P.pack_may_ovf[p]) return 1;
+    return 0;
+  };
   std::stable_sort(P.units.begin(), P.units.end(), [&](const Unit &a, const Unit &b) {
     const int ra = a.kind == kUnitIntra ? (small3(a) ? 1 : 0) : 2;
     const int rb = b.kind == kUnitIntra ? (small3(b) ? 1 : 0) : 2;
     if (ra != rb) return ra < rb;
-    if (P.pack_may_ovf[a.pair] != P.pack_may_ovf[b.pair]) return P.pack_may_ovf[a.pair] > P.pack_may_ovf[b.pair];
+    if (may_ovf(a) != may_ovf(b)) return may_ovf(a) > may_ovf(b);
+    // clustered K3 units have about equal cells: the one holding the longest sequences (the
+    // critical path) goes first -- units launched earlier progress faster when several share
+    // the SMs (measured: finishing in launch order even with every CTA resident)
+    if (a.kind == kUnitIntra && b.kind == kUnitIntra && a.cluster > 1 && b.cluster > 1 && a.npk > 1 && b.npk > 1)
+      return a.b0 < b.b0;
     return a.work > b.work;
   });
   {
@@ -543,13 +572,17 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
     P.pack_q_off[p + 1] = (int32_t)P.pack_q.size();
     P.max_pack_q = std::max<int32_t>(P.max_pack_q, (int32_t)qs.size());
   }
+  for (const Unit &u : P.units)
+    P.max_unit_q = std::max(P.max_unit_q, P.pack_q_off[u.pair + u.npk] - P.pack_q_off[u.pair]);
   // unit-table hash: ranks of one multi-process search must agree on it (net.cpp handshake)
   uint64_t h = 1469598103934665603ull;
   auto mix = [&](int64_t v) {
     for (int b = 0; b < 8; b++) { h ^= (uint64_t)((v >> (8 * b)) & 0xff); h *= 1099511628211ull; }
   };
   mix(nq); mix(db.n); mix(db.residues); mix((int64_t)P.units.size());
-  for (const Unit &u : P.units) { mix(u.kind); mix(u.pair); mix(u.b0); mix(u.b1); mix(u.cells); mix(u.cluster); }
+  for (const Unit &u : P.units) {
+    mix(u.kind); mix(u.pair); mix(u.npk); mix(u.b0); mix(u.b1); mix(u.cells); mix(u.cluster);
+  }
   for (int32_t q : P.pack_q) mix(q);
   P.hash = h;
   return P;
@@ -623,7 +656,7 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     K3Args a;
     a.packed = D.packed.p; a.groups = D.groups.p; a.perm = D.perm.p; a.sorted_len = D.sorted_len.p;
     a.prof = S.prof.p; a.pairs = S.pairs.p; a.slices = S.slices.p;
-    a.pair = U.pair; a.l0 = U.b0; a.l1 = U.b1;
+    a.pair = U.pair; a.npk = U.npk; a.l0 = U.b0; a.l1 = U.b1;
     a.scores = S.scores; a.ndb = db.n;
     a.thresh = thresh;
     a.ovf = S.ovf.p + (size_t)stream_idx * S.ovf_cap; a.ovf_count = S.ovf_count.p + stream_idx;
@@ -645,11 +678,14 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     a.abort_flag = S.abort_d + uidx;
     a.progress = S.progress.p + uidx;
     a.na = na; a.nb = nbm;
-    // grid: cluster 1 -> a block per kK3Warps sequences; clustered -> an equal share of the
-    // resident CTAs per stream (the streams' units run side by side, each claiming its
-    // sequence blocks longest first); a slower PE -> its SM budget
+    // grid: cluster 1 -> a block per kK3Warps sequences; a slower PE -> its SM budget;
+    // clustered units spanning every pack (long sequences carry the work) -> up to the whole
+    // GPU (a later launch's queued clusters take the SMs an earlier unit frees: C5 at 1/4 of
+    // its database 5.02 -> 5.37 TCUPS over per-pack units with equal shares); a clustered
+    // per-pack unit beside K1 units (C4 at 1/8) -> its stream's share of the resident CTAs
     const int maxb = sm_cap > 0 ? std::min(D.n_sm, sm_cap) * k3_blocks_per_sm()
-                   : U.cluster > 1 ? std::max(U.cluster, k3_share(slots, (int)D.streams.size())) : INT32_MAX;
+                   : U.cluster > 1 ? (U.npk > 1 ? slots : std::max(U.cluster, k3_share(slots, (int)D.streams.size())))
+                                   : INT32_MAX;
     launch_k3(a, U.cluster, maxb, st);
   }
   S.launches++;
@@ -666,7 +702,8 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
 // progress units of a whole unit: K1 groups, K3 (sequence, chunk) pairs
 static int64_t unit_progress_total(const Plan &P, const Unit &U) {
   if (U.kind == kUnitInter) return U.b1 - U.b0;
-  const int64_t nch = (P.pairs[U.pair].rows + kK3Chunk - 1) / kK3Chunk;
+  int64_t nch = 0;
+  for (int32_t p = U.pair; p < U.pair + U.npk; p++) nch += (P.pairs[p].rows + kK3Chunk - 1) / kK3Chunk;
   return (int64_t)(U.b1 - U.b0) * nch;
 }
 
@@ -888,7 +925,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       if (K > 0) {
         X.pack_q.ensure(D.id, std::max<size_t>(P.pack_q.size(), 1));
         if (!P.pack_q.empty()) CK(cudaMemcpy(X.pack_q.p, P.pack_q.data(), sizeof(int32_t) * P.pack_q.size(), cudaMemcpyHostToDevice));
-        X.unit_hits.ensure(D.id, nu * P.max_pack_q * K);
+        X.unit_hits.ensure(D.id, nu * P.max_unit_q * K);
         X.worker_hits.ensure(D.id, (size_t)nq * K);
       }
       if (!X.one_h) {
@@ -1136,9 +1173,9 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
               if (K > 0) {
                 int32_t s0u, s1u;
                 unit_seq_range(U, nd, s0u, s1u);
-                const int32_t q0 = P.pack_q_off[U.pair], nqp = P.pack_q_off[U.pair + 1] - q0;
+                const int32_t q0 = P.pack_q_off[U.pair], nqp = P.pack_q_off[U.pair + U.npk] - q0;
                 launch_unit_topk(X.scores, nd, D.perm.p, s0u, s1u, X.pack_q.p + q0, nqp, K,
-                                 X.unit_hits.p + (size_t)u * P.max_pack_q * K, X.epi[0]);
+                                 X.unit_hits.p + (size_t)u * P.max_unit_q * K, X.epi[0]);
                 CK(cudaGetLastError());
                 X.launches++;
               }
@@ -1224,7 +1261,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
           for (int32_t u : X.committed) {
             int32_t s0u, s1u;
             unit_seq_range(P.units[u], nd, s0u, s1u);
-            for (int32_t j = P.pack_q_off[P.units[u].pair]; j < P.pack_q_off[P.units[u].pair + 1]; j++) {
+            for (int32_t j = P.pack_q_off[P.units[u].pair]; j < P.pack_q_off[P.units[u].pair + P.units[u].npk]; j++) {
               segs.push_back({P.pack_q[j], s0u, s1u, 0, seg_total});
               seg_total += s1u - s0u;
             }
@@ -1233,9 +1270,9 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         if (K > 0) {
           std::vector<std::vector<int32_t>> per_q(nq);
           for (int32_t u : X.committed) {
-            const int32_t p = P.units[u].pair;
-            for (int32_t j = P.pack_q_off[p]; j < P.pack_q_off[p + 1]; j++)
-              per_q[P.pack_q[j]].push_back(u * P.max_pack_q + (j - P.pack_q_off[p]));
+            const int32_t p = P.units[u].pair, p1 = p + P.units[u].npk;
+            for (int32_t j = P.pack_q_off[p]; j < P.pack_q_off[p1]; j++)
+              per_q[P.pack_q[j]].push_back(u * P.max_unit_q + (j - P.pack_q_off[p]));
           }
           tab.assign(nq + 1, 0);
           for (int32_t q = 0; q < nq; q++) tab[q + 1] = tab[q] + (int32_t)per_q[q].size();
@@ -1443,6 +1480,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         const UnitLog &L = ulog[k];
         const Unit &U = P.units[L.unit];
         js << (k ? "," : "") << "{\"unit\":" << L.unit << ",\"kind\":" << U.kind << ",\"pair\":" << U.pair
+           << ",\"npk\":" << U.npk
            << ",\"b0\":" << U.b0 << ",\"b1\":" << U.b1 << ",\"cluster\":" << U.cluster
            << ",\"worker\":" << L.worker << ",\"t_grant\":" << L.t_grant << ",\"t_start\":" << L.t_start
            << ",\"t_end\":" << L.t_end << ",\"cells\":" << L.cells << ",\"cells_done\":" << L.cells_done

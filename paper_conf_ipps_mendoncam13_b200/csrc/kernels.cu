@@ -584,15 +584,14 @@ __global__ void __launch_bounds__(kK3Warps * 32, 4) k3_kernel(const K3Args a) {
   uint2 *ring2 = reinterpret_cast<uint2 *>(ring4 + kK3Warps * 3);     // [warps][3][T]
   if (block_aborted(a.abort_flag)) return;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const QueryPair P = a.pairs[a.pair];
-  const int rows = P.rows;
-  const int nch = (rows + CH - 1) / CH;
-  const int nslices = P.rows_padded / 16;
   const uint32_t koff = pk2(kOff), na = a.na, nbeta = a.nb;
   const uint32_t padw = 0x01010101u * kPadCode;
-  const int32_t *gprof = a.prof + P.prof_off;
   uint32_t *prof_s = smem;
+  // tasks = (pack, sequence block of kK3Warps sequences); a unit spans packs [pair, pair + npk)
+  // (clustered units only), task t = pack pair + t % npk of block t / npk: longest blocks first,
+  // every pack's at once
   const int nsb = (a.l1 - a.l0 + kK3Warps - 1) / kK3Warps;
+  const int ntask = nsb * a.npk;
   const int crank = C > 1 ? (int)(blockIdx.x % C) : 0;     // CTA rank in the cluster
   const int cid = blockIdx.x / C, ncl = gridDim.x / C;
   // C > 1: this warp's (slot, buffer) border rows and progress counters are per grid slot
@@ -604,23 +603,29 @@ __global__ void __launch_bounds__(kK3Warps * 32, 4) k3_kernel(const K3Args a) {
   for (int b = 0; b < C; b++) cum[b] = 0;
   int done = 0;          // (sequence, chunk) pairs this warp completed
   bool aborted = false;
-  // C > 1: the clusters of a launch claim sequence blocks dynamically (longest first, the
+  // C > 1: the clusters of a launch claim tasks dynamically (longest blocks first, the
   // sorted order) from a per-launch counter; rank 0 claims and broadcasts over DSMEM
   __shared__ int sb_claim;
-  auto next_sb = [&](int prev) -> int {
+  auto next_task = [&](int prev) -> int {
     if (C == 1) return prev < 0 ? cid : prev + ncl;
     namespace cg = cooperative_groups;
     cg::cluster_group cl = cg::this_cluster();
     if (crank == 0 && threadIdx.x == 0)
-      sb_claim = (aborted || (a.abort_flag && *a.abort_flag != 0)) ? nsb : atomicAdd(a.claim, 1);
+      sb_claim = (aborted || (a.abort_flag && *a.abort_flag != 0)) ? ntask : atomicAdd(a.claim, 1);
     cl.sync();
     const int v = *cl.map_shared_rank(&sb_claim, 0);
     cl.sync();   // rank 0 may overwrite sb_claim only after every CTA read it
     return v;
   };
 
-  for (int sb = next_sb(-1); sb < nsb; sb = next_sb(sb)) {
+  for (int task = next_task(-1); task < ntask; task = next_task(task)) {
     if (aborted) continue;   // C > 1: go straight to the next claim (it returns the end)
+    const int sb = task / a.npk;
+    const QueryPair P = a.pairs[a.pair + task % a.npk];
+    const int rows = P.rows;
+    const int nch = (rows + CH - 1) / CH;
+    const int nslices = P.rows_padded / 16;
+    const int32_t *gprof = a.prof + P.prof_off;
     const int s = a.l0 + sb * kK3Warps + warp;
     const bool valid = s < a.l1;
     const int len = valid ? a.sorted_len[s] : 0;
@@ -815,7 +820,7 @@ static size_t k3_smem() {
 template <int T, int C>
 static void k3_go(const K3Args &a, int n, int max_blocks, cudaStream_t st) {
   const size_t smem = k3_smem<T>();
-  const int nsb = (n + kK3Warps - 1) / kK3Warps;
+  const int nsb = (n + kK3Warps - 1) / kK3Warps * std::max(1, a.npk);   // tasks
   auto fn = k3_kernel<kK3Rows, T, C>;
   cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared);

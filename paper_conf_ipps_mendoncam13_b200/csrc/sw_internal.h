@@ -67,7 +67,7 @@ struct Unit {
   int64_t cells;         // real cells (sum |q|*|d|), for GCUPS and PSS rates
   int64_t work;          // padded lane-cells (balancing)
   int32_t cluster = 1;   // K3: CTAs per thread-block cluster splitting each pair's chunks
-  int32_t pad_ = 0;
+  int32_t npk = 1;       // packs [pair, pair + npk) (> 1 only for clustered K3 units)
 };
 
 // ---- query packs ------------------------------------------------------------------------
@@ -104,10 +104,10 @@ struct K1Args {
   int32_t *gclaim;                   // unit's counter: groups claimed by its blocks (zeroed)
   uint32_t na, nb;                   // packed -alpha, -beta
 };
-struct K3Args {   // sequences [l0,l1) in sorted order (the long groups)
+struct K3Args {   // sequences [l0,l1) in sorted order (the long groups) x packs [pair, pair + npk)
   const uint4 *packed; const GroupInfo *groups; const int32_t *perm; const int32_t *sorted_len;
   const int32_t *prof; const QueryPair *pairs; const SliceInfo *slices;
-  int32_t pair; int32_t l0, l1;
+  int32_t pair; int32_t npk; int32_t l0, l1;
   int32_t *scores; int64_t ndb;
   int32_t thresh;
   int2 *ovf; int32_t *ovf_count; int32_t ovf_cap; uint32_t *ovf_bits;
