@@ -159,6 +159,10 @@ typedef struct {
   int64_t peer_bytes;       /* bytes copied between GPUs by the in-process merge */
   const char *sched_log_json;/* the master's event log with Φ and v̄ per grant (sw_sched.h);
                                in-process, or rank 0 in multi-process mode; owned by the sw_db */
+  double kernel_seconds_k2; /* summed device time of the int32 re-run launches (K2), from the
+                               launch being enqueued on its stream to its end (includes the
+                               wait for free SMs behind the DP kernels) */
+  int32_t n_k2_launches;    /* int32 re-run launches */
 } sw_stats;
 
 typedef struct sw_db sw_db; /* opaque: host index + packed replica on each device */

@@ -118,13 +118,14 @@ struct DevSearch {
   int32_t *scores = nullptr;
   DBuf<int2> ovf;              // [streams][kOvfCap] saturated pairs, one list per stream
   DBuf<int32_t> ovf_count;     // [streams]
-  DBuf<int32_t> ovf_cursor;    // [streams] entries taken by the int32 re-run
+  DBuf<int32_t> ovf_cursor;    // [streams][2] entries taken by the int32 re-run (small / big pairs)
   DBuf<uint32_t> ovf_bits;     // [nq*ndb] bits: pair already listed
   int32_t ovf_cap = 0;         // entries per stream list
   DBuf<uint2> k3_border;   // [streams][k3_rows][max_len]
   int64_t k3_rows = 0;
   DBuf<int32_t> k3_prog;   // [streams][k3 slots x warps]: clustered K3 progress counters
   DBuf<int32_t> k2_border;
+  DBuf<long long> k2_prog;   // [streams][kK2Blocks]: big-pair progress counters (K2 clusters)
   DBuf<int32_t> abort_dev;      // per-unit WA cancellation flags (device memory)
   DBuf<int32_t> progress;       // per-unit progress counters (K1 groups / K3 sequence-chunks)
   DBuf<int32_t> gclaim;         // per-unit K1 group claim counters
@@ -151,7 +152,8 @@ struct DevSearch {
   cudaEvent_t ev_start = nullptr, ev_end = nullptr, ev_data = nullptr;
   std::vector<cudaEvent_t> u_start, u_end;  // per stream
   int launches = 0;
-  double k1_sec = 0, k3_sec = 0;
+  double k1_sec = 0, k3_sec = 0, k2_sec = 0;
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> k2_ev;   // per K2 launch (rare), this search
   int64_t k1_cells = 0, k3_cells = 0;
   int64_t dup_cells = 0;
   int32_t n_cancelled = 0;
@@ -159,7 +161,9 @@ struct DevSearch {
   double last_dev = 0;           // device time of this worker's last unit completion (s)
   int32_t n_ovf = 0;
   void reset_counters() {
-    launches = 0; k1_sec = k3_sec = 0; k1_cells = k3_cells = 0; dup_cells = 0; n_cancelled = 0;
+    for (auto &e : k2_ev) { cudaEventDestroy(e.first); cudaEventDestroy(e.second); }
+    k2_ev.clear();
+    launches = 0; k1_sec = k3_sec = k2_sec = 0; k1_cells = k3_cells = 0; dup_cells = 0; n_cancelled = 0;
     finish_wall = 0; last_dev = 0; n_ovf = 0; scores = nullptr; committed.clear();
   }
   ~DevSearch();
@@ -191,6 +195,7 @@ inline DevSearch::~DevSearch() {
   for (auto e : epi) cudaStreamDestroy(e);
   if (ev_start) cudaEventDestroy(ev_start);
   if (ev_end) cudaEventDestroy(ev_end);
+  for (auto &e : k2_ev) { cudaEventDestroy(e.first); cudaEventDestroy(e.second); }
   if (ev_data) cudaEventDestroy(ev_data);
   for (auto e : u_start) cudaEventDestroy(e);
   for (auto e : u_end) cudaEventDestroy(e);
@@ -380,6 +385,26 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
   // worker's share of (pack, long-sequence block) tasks fills too few of the GPU's resident
   // K3 CTAs -- C5 at 8 GPUs: 256 blocks for 592 slots -- each pair's chunks are split over a
   // cluster of 4 (fill < 1/2) or 2 CTAs.  SW_K3_CLUSTER forces a size (tuning, tests).
+  // chunk balance: a cluster of C CTAs runs a pair's nch chunks in ceil(nch / C) rounds, and
+  // the CTAs idle at the cluster barrier for the rest of the last round; among C - 1, C, C + 1
+  // (instantiated sizes 2..5) take the best-balanced size over the packs [p0, p1), ties to
+  // the larger (fewer rounds).  C5's 5,000-row packs (10 chunks): 4 -> 5 CTAs, C5 at 1/8 of
+  // its database 4.30 -> 4.58 TCUPS, C4 at 1/8 6.16 -> 6.28
+  auto balance_cluster = [&](int base, int32_t p0, int32_t p1) {
+    int best = base;
+    double best_eff = -1.0;
+    for (int c = std::max(2, base - 1); c <= std::min(5, base + 1); c++) {
+      int64_t used = 0, slots = 0;
+      for (int32_t p = p0; p < p1; p++) {
+        const int64_t nch = (P.pairs[p].rows + kK3Chunk - 1) / kK3Chunk;
+        used += nch;
+        slots += (nch + c - 1) / c * c;
+      }
+      const double eff = slots > 0 ? (double)used / slots : 0.0;
+      if (eff > best_eff + 1e-9 || (eff > best_eff - 1e-9 && c > best)) { best = c; best_eff = eff; }
+    }
+    return best;
+  };
   int32_t k3_cluster = 1;
   {
     int64_t long_res = 0;
@@ -390,10 +415,11 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
     const double sb_per_worker = (double)P.pairs.size() * ((P.n_long_seqs + kK3Warps - 1) / kK3Warps) /
                                  std::max(1, n_workers);
     static const int forced = [] { const char *e = getenv("SW_K3_CLUSTER"); return e ? atoi(e) : 0; }();
-    if (forced == 1 || forced == 2 || forced == 4 || forced == 8) k3_cluster = forced;
+    if (forced >= 1 && forced <= 8 && forced != 6 && forced != 7) k3_cluster = forced;
     else if (o.target_unit_cells <= 0 && P.n_long_seqs > 0 && c3 >= c1 && k3_slots > 0) {
       const double fill = sb_per_worker / k3_slots;
       k3_cluster = fill < 0.5 ? 4 : fill < 1.0 ? 2 : 1;
+      if (k3_cluster > 1) k3_cluster = balance_cluster(k3_cluster, 0, (int32_t)P.pairs.size());
     }
   }
   int64_t target = o.target_unit_cells;
@@ -510,11 +536,12 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
   // costs 2 %)
   {
     static const int forced = [] { const char *e = getenv("SW_K3_CLUSTER"); return e ? atoi(e) : 0; }();
+    static const int mixc = [] { const char *e = getenv("SW_K3_MIXC"); return e && atoi(e) > 1 ? atoi(e) : 4; }();
     if (forced == 0 && k3_cluster == 1 && o.target_unit_cells <= 0 && k3_slots > 0)
       for (Unit &u : P.units)
         if (u.kind == kUnitIntra) {
           const double ratio = (double)((u.b1 - u.b0 + kK3Warps - 1) / kK3Warps) * depth / k3_slots;
-          if (ratio < 0.75) u.cluster = 4;
+          if (ratio < 0.75) u.cluster = getenv("SW_K3_MIXC") ? mixc : balance_cluster(4, u.pair, u.pair + u.npk);
         }
   }
   // LPT by expected duration: intra-task (long-sequence) units first -- each warp walks a
@@ -604,6 +631,9 @@ struct UnitLog {
 static const int kOvfCap = 1 << 20;
 
 
+// K2 border row stride (columns): whole 4-column tiles, 32-byte aligned rows (cp.async)
+static int64_t k2_stride(const Plan &P) { return (std::max<int64_t>(P.max_len, 1) + 3) / 4 * 4; }
+
 // K2 arguments for the saturated-pair list of one stream
 static K2Args k2_args(const Plan &P, const PackedDB &db, DevSearch &S, int stream_idx, int32_t alpha,
                       int32_t beta) {
@@ -613,9 +643,14 @@ static K2Args k2_args(const Plan &P, const PackedDB &db, DevSearch &S, int strea
   a.packed = D.packed.p; a.groups = D.groups.p; a.sorted_len = D.sorted_len.p; a.perm = D.perm.p;
   a.matrix = S.matrix.p;
   a.ovf = S.ovf.p + (size_t)stream_idx * S.ovf_cap; a.ovf_count = S.ovf_count.p + stream_idx;
-  a.ovf_cap = S.ovf_cap; a.ovf_cursor = S.ovf_cursor.p + stream_idx;
+  a.ovf_cap = S.ovf_cap; a.ovf_cursor = S.ovf_cursor.p + 2 * stream_idx;
+  // a pair of at least big_cells (SW_K2_BIG: tuning, tests) is split over a K2 cluster:
+  // 2^24 cells take ~1 ms on one SM
+  static const int64_t big = [] { const char *e = getenv("SW_K2_BIG"); return e && atoll(e) > 0 ? atoll(e) : (1LL << 24); }();
+  a.big_cells = big;
+  a.k2prog = S.k2_prog.p + (size_t)stream_idx * kK2Blocks;
   a.scores = S.scores; a.ndb = db.n; a.alpha = alpha; a.beta = beta; a.one = 1;
-  const int64_t stride = std::max<int64_t>(P.max_len, 1);
+  const int64_t stride = k2_stride(P);
   a.border = S.k2_border.p + (size_t)stream_idx * kK2Blocks * stride * 2;
   a.border_stride = stride;
   return a;
@@ -906,9 +941,10 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       X.ovf_cap = s16_ok ? kOvfCap : (int32_t)std::min<int64_t>((int64_t)nq * nd + 1, INT32_MAX / 2);
       X.ovf.ensure(D.id, (size_t)depth * X.ovf_cap);
       X.ovf_count.ensure(D.id, depth);
-      X.ovf_cursor.ensure(D.id, depth);
+      X.ovf_cursor.ensure(D.id, 2 * depth);
+      X.k2_prog.ensure(D.id, (size_t)depth * kK2Blocks);
       X.ovf_bits.ensure(D.id, ((size_t)nq * nd + 31) / 32);
-      X.k2_border.ensure(D.id, (size_t)depth * kK2Blocks * std::max<int64_t>(P.max_len, 1) * 2);
+      X.k2_border.ensure(D.id, (size_t)depth * kK2Blocks * k2_stride(P) * 2);
       const size_t k3b = (size_t)depth * k3_rows * ((std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16);
       if (P.n_long_seqs > 0) X.k3_border.ensure(D.id, k3b);
       if (any_cluster) X.k3_prog.ensure(D.id, (size_t)depth * (k3_slots * kK3Warps + 1));
@@ -1043,7 +1079,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         CK(cudaEventRecord(X.ev_start, s0));
         launch_fill(X.scores, (int64_t)nq * nd, -1, s0);
         CK(cudaMemsetAsync(X.ovf_count.p, 0, sizeof(int32_t) * depth, s0));
-        CK(cudaMemsetAsync(X.ovf_cursor.p, 0, sizeof(int32_t) * depth, s0));
+        CK(cudaMemsetAsync(X.ovf_cursor.p, 0, sizeof(int32_t) * 2 * depth, s0));
         CK(cudaMemsetAsync(X.ovf_bits.p, 0, sizeof(uint32_t) * (((size_t)nq * nd + 31) / 32), s0));
         launch_profile(X.qcodes.p, X.qoff.p, X.pairs.p, (int)P.pairs.size(), X.slices.p, X.matrix.p,
                        X.prof.p, P.prof_total, s0);
@@ -1162,7 +1198,15 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
             // a pair exactly, and the later partial maxima of its other slices are smaller.
             const int32_t seen = ((volatile int32_t *)X.ovf_seen_h)[k];
             if (seen > k2_upto[k]) {
-              launch_k2(k2_args(P, H, X, k, alpha, beta), kK2Blocks, X.epi[0]);
+              const K2Args k2a = k2_args(P, H, X, k, alpha, beta);
+              std::pair<cudaEvent_t, cudaEvent_t> ev;
+              CK(cudaEventCreate(&ev.first));
+              CK(cudaEventCreate(&ev.second));
+              X.k2_ev.push_back(ev);
+              CK(cudaMemsetAsync(k2a.k2prog, 0, sizeof(long long) * kK2Blocks, X.epi[0]));
+              CK(cudaEventRecord(ev.first, X.epi[0]));
+              launch_k2(k2a, kK2Blocks, X.epi[0]);
+              CK(cudaEventRecord(ev.second, X.epi[0]));
               CK(cudaGetLastError());
               X.launches++;
               k2_upto[k] = seen;
@@ -1242,14 +1286,20 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         // the int32 re-runs ran on each stream after the units that saturated; check the lists
         for (int k = 0; k < depth; k++) CK(cudaStreamSynchronize(D.streams[k]));
         CK(cudaStreamSynchronize(X.epi[0]));
-        std::vector<int32_t> novf(depth, 0), ncur(depth, 0);
+        for (auto &e : X.k2_ev) {
+          float ms = 0;
+          CK(cudaEventElapsedTime(&ms, e.first, e.second));
+          X.k2_sec += 1e-3 * ms;
+        }
+        std::vector<int32_t> novf(depth, 0), ncur(2 * depth, 0);
         CK(cudaMemcpy(novf.data(), X.ovf_count.p, sizeof(int32_t) * depth, cudaMemcpyDeviceToHost));
-        CK(cudaMemcpy(ncur.data(), X.ovf_cursor.p, sizeof(int32_t) * depth, cudaMemcpyDeviceToHost));
+        CK(cudaMemcpy(ncur.data(), X.ovf_cursor.p, sizeof(int32_t) * 2 * depth, cudaMemcpyDeviceToHost));
         X.n_ovf = 0;
         for (int k = 0; k < depth; k++) {
           if (novf[k] > X.ovf_cap) throw Error(SW_ENOMEM, "overflow list capacity exceeded");
           X.n_ovf += novf[k];
-          if (ncur[k] < novf[k]) throw Error(SW_ECUDA, "int32 re-run left saturated pairs");
+          if (ncur[2 * k] < novf[k] || ncur[2 * k + 1] < novf[k])
+            throw Error(SW_ECUDA, "int32 re-run left saturated pairs");
         }
         // ---- data plane, on this device: top-k over the units this worker committed
         // (K5m), and (in-process, device != first) the committed units' scores packed densely
@@ -1460,6 +1510,8 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         stats->kernel_launches += S[w]->launches;
         stats->kernel_seconds_k1 += S[w]->k1_sec;
         stats->kernel_seconds_k3 += S[w]->k3_sec;
+        stats->kernel_seconds_k2 += S[w]->k2_sec;
+        stats->n_k2_launches += (int32_t)S[w]->k2_ev.size();
         stats->cells_k1 += S[w]->k1_cells;
         stats->cells_k3 += S[w]->k3_cells;
         stats->n_cancelled += S[w]->n_cancelled;

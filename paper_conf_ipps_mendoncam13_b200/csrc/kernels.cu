@@ -26,6 +26,7 @@
 #include <algorithm>
 #include <mutex>
 #include "sw_internal.h"
+#include "../../include/sw.h"
 
 namespace sw {
 
@@ -856,7 +857,7 @@ int k3_blocks_per_sm() {
   });
   return v;
 }
-// cluster size 1, 2 or 4 (a.kprog: [grid slots][C] zeroed progress counters when C > 1).
+// cluster size 1, 2, 3, 4, 5 or 8 (3, 5, 8: 8-column tiles only; a.kprog: [grid slots][C] zeroed progress counters when C > 1).
 // max_blocks caps the grid (resident CTAs; an SM budget when emulating a slower PE);
 // C > 1 needs at most the resident clusters (persistent loop, sequence blocks claimed
 // through a.claim, zeroed), C == 1 one block per kK3Warps sequences
@@ -867,6 +868,8 @@ void launch_k3(const K3Args &a, int cluster, int max_blocks, cudaStream_t st) {
   switch (cluster) {
     case 2: if (t4) k3_go<4, 2>(a, n, max_blocks, st); else k3_go<8, 2>(a, n, max_blocks, st); break;
     case 4: if (t4) k3_go<4, 4>(a, n, max_blocks, st); else k3_go<8, 4>(a, n, max_blocks, st); break;
+    case 3: k3_go<8, 3>(a, n, max_blocks, st); break;
+    case 5: k3_go<8, 5>(a, n, max_blocks, st); break;
     case 8: k3_go<8, 8>(a, n, max_blocks, st); break;
     default: if (t4) k3_go<4, 1>(a, n, max_blocks, st); else k3_go<8, 1>(a, n, max_blocks, st); break;
   }
@@ -906,21 +909,171 @@ void launch_noise(const int32_t *stop, int n_blocks, uint64_t max_ns, uint32_t *
 
 // ------------------------------------------------------------------------------------
 // K2: int32 re-run of saturated (query, sequence) pairs.  Same recurrence as K1/K3 in
-// plain int32 (E and F floored at 0, exact for H: DESIGN.md §6), one BLOCK per pair:
-// thread L owns rows [L*K2R, (L+1)*K2R) of each chunk of kK2Threads*K2R query rows and
-// runs the wavefront of P14 §II.B (Fig. 3a) across the whole block -- at step t thread L
-// updates the K2C-column tile t - L and hands its bottom row (H, F) to thread L+1 through
-// a double-buffered shared-memory slot (one __syncthreads per step); the last active
-// thread writes the chunk's bottom row to a global border read by thread 0 in the next
-// chunk.  A single long saturated pair (C5: a 5,000-aa query inside a 10k-35k sequence)
-// therefore runs on a whole SM instead of one warp.  Scores come from the 25x25 matrix
-// replicated per lane in shared memory ([query code][db code][lane]: bank = lane, no
-// conflicts although every thread is at a different row and column).
+// plain int32 (E and F floored at 0, exact for H: DESIGN.md §6), run by a BLOCK:
+// thread L owns rows [L*K2R, (L+1)*K2R) of a chunk of query rows and runs the wavefront
+// of P14 §II.B (Fig. 3a) across the block -- at step t thread L updates the K2C-column
+// tile t - L and hands its bottom row (H, F) to thread L+1 through a double-buffered
+// shared-memory slot (one __syncthreads per step); the last active thread writes the
+// chunk's bottom row to a global border read by thread 0 of the next chunk.  Scores come
+// from the 25x25 matrix replicated per lane in shared memory ([query code][db code][lane]:
+// bank = lane, no conflicts although every thread is at a different row and column).
+// The CTAs of a launch form clusters of kK2Cluster:
+//  * big pairs (m*n >= big_cells; C5: a 5,000-aa query inside a 35k-residue sequence)
+//    are taken by a whole cluster: CTA r runs chunk r of about m / kK2Cluster rows, and
+//    chunk r+1 (the next CTA) follows it tile by tile through the border row in L2 (a
+//    per-(cluster, boundary) progress counter tagged with the pair's epoch, released
+//    every kK2Pub tiles and acquired before each prefetch; the cluster makes producer and
+//    consumer co-resident, so the wait cannot deadlock).  Round 1 ran such a pair on one
+//    SM (10.4 ms for C5's planted pair), the tail of a small per-GPU share of C5;
+//  * the other pairs are taken by single CTAs, chunks of kK2Threads*K2R rows in order.
+// Each list has its own cursor (small: ovf_cursor[0], big: ovf_cursor[1]); a cursor
+// skips the other kind's entries and never passes the count this launch saw.
 // ------------------------------------------------------------------------------------
 constexpr int K2R = 16;          // rows per thread
 constexpr int K2C = 4;           // columns per tile (one aligned 32-bit word of codes)
-constexpr int kK2Threads = 512;  // threads per block (chunk = 8,192 rows)
+constexpr int kK2Threads = 512;  // threads per block (chunk <= 8,192 rows)
+constexpr int kK2Pub = 8;        // tiles between a big pair's progress publications
+constexpr int kK2Ring = 8;       // border-row tiles in flight (thread 0's cp.async ring)
 constexpr size_t kK2Smem = sizeof(int32_t) * kNCodes * kNCodes * 32 + sizeof(int2) * 2 * kK2Threads * K2C;
+static_assert(kK2Cluster * kK2Threads * K2R > SW_MAX_QUERY_LEN, "a big pair is at most one chunk per CTA");
+
+__device__ __forceinline__ long long ld_acquire64(const long long *p) {
+  long long v;
+  asm volatile("ld.acquire.gpu.global.b64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release64(long long *p, long long v) {
+  asm volatile("st.release.gpu.global.b64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+// claim the next entry of one kind from cursor `cur` (thread 0); returns count when none
+__device__ __forceinline__ int k2_claim(const K2Args &a, int *cur_p, int count, bool big) {
+  int cur = *(volatile int32_t *)cur_p;
+  while (cur < count) {
+    const int2 e = a.ovf[cur];
+    const int64_t cells = (a.qoff[e.x + 1] - a.qoff[e.x]) * (int64_t)a.sorted_len[e.y];
+    const int seen = atomicCAS(cur_p, cur, cur + 1);
+    if (seen != cur) { cur = seen; continue; }          // someone else moved it: retry there
+    if ((cells >= a.big_cells) == big) return cur;      // ours
+    cur++;                                              // skipped (the other kind's)
+  }
+  return count;
+}
+
+// One chunk [r0, r0 + nact*R) (R rows per thread) of pair (qc, m) x (sequence of group G, lane gl) on this
+// block; returns this thread's maximum H.  bin / bout: border rows in / out (nullptr: the
+// first / last chunk); prog_in / prog_out: (big pairs) the producer's / this chunk's
+// progress counter, values (epoch << 32) + tiles.  bin == bout is allowed when the chunks
+// of a pair run in order on one block (the writer trails the reader by nact tiles).
+template <int R>
+__device__ __forceinline__ int k2_chunk(const K2Args &a, const int32_t *Ms, int2 *hand, const uint8_t *qc,
+                                        int m, int r0, int nact, const GroupInfo &G, int gl, int ntile,
+                                        const int2 *bin, int2 *bout, const long long *prog_in,
+                                        long long *prog_out, long long epoch, int2 *ring) {
+  const int L = threadIdx.x, lane = L & 31;
+  const uint32_t *words = reinterpret_cast<const uint32_t *>(a.packed);
+  const int na = -a.alpha, nb = -a.beta, one = a.one;
+  auto codes_of = [&](int tt) -> uint32_t {   // codes of columns tt*4 .. tt*4+3 (32-bit word)
+    const int col = tt * K2C;
+    return __ldg(words + ((G.word_off + (int64_t)(col >> 4) * kGroup + gl) * 4 + ((col & 15) >> 2)));
+  };
+  // big pairs: wait until the chunk above has published tile tt (thread 0 only)
+  long long seen = 0;
+  auto wait_tile = [&](int tt) {
+    if (!prog_in) return;
+    const long long want = (epoch << 32) + tt + 1;
+    if (seen >= want) return;
+    const long long t_wait = clock64();
+    while ((seen = ld_acquire64(prog_in)) < want)
+      if (clock64() - t_wait > (1ll << 36)) __trap();   // ~35 s: never hang the GPU
+  };
+  // thread 0 streams the border row of the chunk above into a kK2Ring-tile shared-memory
+  // ring with cp.async.cg (L2: never a stale L1 line), kK2Ring - 1 tiles ahead: an L2 round
+  // trip is longer than a step, so a one-step-ahead load would stall every step
+  auto fetch = [&](int tt) {
+    if (bin && tt < ntile) {
+      wait_tile(tt);
+      cp_async16_cg(&ring[(tt % kK2Ring) * K2C], bin + tt * K2C);
+      cp_async16_cg(&ring[(tt % kK2Ring) * K2C + 2], bin + tt * K2C + 2);
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  const bool active = L < nact;
+  int rowoff[R];
+#pragma unroll
+  for (int i = 0; i < R; i++) {
+    const int row = r0 + L * R + i;
+    rowoff[i] = (row < m ? (int)qc[row] : kPadCode) * (kNCodes * 32) + lane;
+  }
+  int H[R], E[R];
+#pragma unroll
+  for (int i = 0; i < R; i++) { H[i] = 0; E[i] = 0; }
+  int hprev_top = 0, best = 0;
+  const int steps = ntile + nact - 1;
+  // register prefetch, one step ahead: this thread's next codes word
+  uint32_t cw_next = (active && L == 0 && ntile > 0) ? codes_of(0) : 0u;
+  if (L == 0)
+    for (int tt = 0; tt < kK2Ring - 1; tt++) fetch(tt);
+  for (int t = 0; t < steps; t++) {
+    const int tile = t - L;
+    if (active && tile >= 0 && tile < ntile) {
+      const uint32_t cw = cw_next;
+      if (tile + 1 < ntile) cw_next = codes_of(tile + 1);
+      int2 in[K2C];
+      if (L == 0) {
+        fetch(tile + kK2Ring - 1);   // into the slot of tile - 1, consumed last step
+        asm volatile("cp.async.wait_group %0;" ::"n"(kK2Ring - 1) : "memory");   // tile landed
+#pragma unroll
+        for (int g = 0; g < K2C; g++) in[g] = bin ? ring[(tile % kK2Ring) * K2C + g] : make_int2(0, 0);
+      } else {
+#pragma unroll
+        for (int g = 0; g < K2C; g++) in[g] = hand[(((t - 1) & 1) * K2C + g) * kK2Threads + L - 1];
+      }
+      int coff[K2C], hd[K2C], f[K2C], oh[K2C];
+#pragma unroll
+      for (int g = 0; g < K2C; g++) {
+        coff[g] = (int)((cw >> (8 * g)) & 0xffu) * 32;
+        hd[g] = hprev_top;
+        f[g] = in[g].y;
+        hprev_top = in[g].x;
+      }
+      // skewed tile: at sub-step k column g updates row k - g (K2C independent chains)
+#pragma unroll
+      for (int k = 0; k < R + K2C - 1; k++) {
+#pragma unroll
+        for (int g = 0; g < K2C; g++) {
+          const int i = k - g;
+          if (i >= 0 && i < R) {
+            // x on the FMA pipe (IMAD by an opaque 1): a plain add would be fused by
+            // ptxas into a VIADDMNMX + VIMNMX pair, one more ALU op per cell
+            const int x = Ms[rowoff[i] + coff[g]] * one + hd[g];
+            const int h = __vimax3_s32(x, E[i], f[g]);      // >= 0: E, F floored at 0
+            const int tt = __viaddmax_s32(h, na, 0);        // max(H - alpha, 0)
+            E[i] = __viaddmax_s32(E[i], nb, tt);            // E(i, j+1)
+            f[g] = __viaddmax_s32(f[g], nb, tt);            // F(i+1, j)
+            hd[g] = H[i];
+            H[i] = h;
+            best = max(best, h);
+            if (i == R - 1) oh[g] = h;
+          }
+        }
+      }
+#pragma unroll
+      for (int g = 0; g < K2C; g++) hand[((t & 1) * K2C + g) * kK2Threads + L] = make_int2(oh[g], f[g]);
+      if (L == nact - 1 && bout) {
+#pragma unroll
+        for (int g = 0; g < K2C; g++) bout[tile * K2C + g] = make_int2(oh[g], f[g]);
+        if (prog_out && ((tile + 1) % kK2Pub == 0 || tile + 1 == ntile))
+          st_release64(prog_out, (epoch << 32) + tile + 1);   // orders this thread's border stores
+      }
+    } else if (active && L > 0 && tile == -1 && ntile > 0) {
+      cw_next = codes_of(0);   // first tile of this thread starts next step
+    }
+    __syncthreads();
+  }
+  if (L == 0) asm volatile("cp.async.wait_all;" ::: "memory");
+  return best;
+}
 
 __global__ void __launch_bounds__(kK2Threads, 1) k2_kernel(const K2Args a) {
   extern __shared__ __align__(16) int32_t k2s[];
@@ -928,148 +1081,112 @@ __global__ void __launch_bounds__(kK2Threads, 1) k2_kernel(const K2Args a) {
   int2 *hand = reinterpret_cast<int2 *>(k2s + kNCodes * kNCodes * 32);  // [2][K2C][threads]
   __shared__ int claim_s;
   __shared__ int red_s[kK2Threads / 32];
+  __shared__ __align__(16) int2 ring[kK2Ring * K2C];
   const int count = min(*a.ovf_count, a.ovf_cap);
-  if (*(volatile int32_t *)a.ovf_cursor >= count) return;   // nothing saturated (the usual case)
+  if (*(volatile int32_t *)a.ovf_cursor >= count && *(volatile int32_t *)(a.ovf_cursor + 1) >= count)
+    return;   // nothing saturated (the usual case)
   for (int k = threadIdx.x; k < kNCodes * kNCodes * 32; k += kK2Threads) {
     const int r = k / (kNCodes * 32), c = (k / 32) % kNCodes;   // query code, database slot
     Ms[k] = (r < 24 && c < 24) ? (int32_t)a.matrix[r * 24 + c_code_of_slot[c]] : kPadScore;
   }
   const int L = threadIdx.x, lane = L & 31;
-  const uint32_t *words = reinterpret_cast<const uint32_t *>(a.packed);
-  int32_t *border = a.border + (size_t)blockIdx.x * a.border_stride * 2;
-  const int na = -a.alpha, nb = -a.beta, one = a.one;
+  namespace cg = cooperative_groups;
+  cg::cluster_group cl = cg::this_cluster();
+  const int crank = (int)cl.block_rank(), cid = blockIdx.x / kK2Cluster;
+  auto block_max = [&](int best) {   // -> thread 0
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) best = max(best, __shfl_xor_sync(0xffffffffu, best, o));
+    if (lane == 0) red_s[L >> 5] = best;
+    __syncthreads();
+    int b = 0;
+    if (L == 0)
+      for (int w = 0; w < kK2Threads / 32; w++) b = max(b, red_s[w]);
+    return b;
+  };
+  // ---- big pairs: one cluster per pair, CTA r = chunk r
+  // border row of boundary r (chunk r -> r+1) of this cluster = block (cid*C + r)'s row
+  int2 *cborder = reinterpret_cast<int2 *>(a.border) + (size_t)cid * kK2Cluster * a.border_stride;
+  long long *cprog = a.k2prog + (size_t)cid * kK2Cluster;
+  for (long long epoch = 1;; epoch++) {
+    if (crank == 0 && L == 0) claim_s = k2_claim(a, a.ovf_cursor + 1, count, true);
+    cl.sync();
+    const int p = *cl.map_shared_rank(&claim_s, 0);
+    cl.sync();   // rank 0 may overwrite claim_s only after every CTA read it
+    if (p >= count) break;
+    const int q = a.ovf[p].x, s = a.ovf[p].y;
+    const int m = (int)(a.qoff[q + 1] - a.qoff[q]);
+    const int len = a.sorted_len[s];
+    const int ntile = (len + K2C - 1) / K2C;   // columns up to ntile*4 <= G.ncols are pad codes
+    // rows per thread: a CTA holds only m / kK2Cluster rows, so with few threads a step is
+    // latency-bound and fewer rows per thread shorten its dependency chain; the most rows
+    // per thread that still leave <= 192 threads (5,000 x 35,000: 16 -> 4 rows, 7.1 -> 4.9
+    // ms; 30,000 x 20,000: 16 rows, 7.9 ms, 8 rows 9.7 ms)
+    const int per_cta = (m + kK2Cluster - 1) / kK2Cluster;
+    const int R = per_cta <= 4 * 192 ? 4 : per_cta <= 8 * 192 ? 8 : K2R;
+    const int rc = ((m + kK2Cluster - 1) / kK2Cluster + R - 1) / R * R;   // rows per chunk
+    const int nch = (m + rc - 1) / rc;
+    int best = 0;
+    if (crank < nch && len > 0) {
+      const int r0 = crank * rc;
+      const int nact = (min(rc, m - r0) + R - 1) / R;
+      const uint8_t *qc = a.qcodes + a.qoff[q];
+      const GroupInfo G = a.groups[s / kGroup];
+      int2 *bi = crank > 0 ? cborder + (size_t)(crank - 1) * a.border_stride : nullptr;
+      int2 *bo = crank < nch - 1 ? cborder + (size_t)crank * a.border_stride : nullptr;
+      const long long *pi = crank > 0 ? cprog + crank - 1 : nullptr;
+      long long *po = crank < nch - 1 ? cprog + crank : nullptr;
+      if (R == 4) best = k2_chunk<4>(a, Ms, hand, qc, m, r0, nact, G, s % kGroup, ntile, bi, bo, pi, po, epoch, ring);
+      else if (R == 8) best = k2_chunk<8>(a, Ms, hand, qc, m, r0, nact, G, s % kGroup, ntile, bi, bo, pi, po, epoch, ring);
+      else best = k2_chunk<K2R>(a, Ms, hand, qc, m, r0, nact, G, s % kGroup, ntile, bi, bo, pi, po, epoch, ring);
+    }
+    const int b = block_max(best);
+    if (L == 0 && crank < nch) atomicMax(a.scores + (int64_t)q * a.ndb + a.perm[s], b);   // max over chunks
+    __syncthreads();   // red_s / hand reused
+  }
+  // ---- the other pairs: one block per pair, chunks in order
+  int2 *border = reinterpret_cast<int2 *>(a.border) + (size_t)blockIdx.x * a.border_stride;
   constexpr int CH = kK2Threads * K2R;
   while (true) {
-    // claim the next entry; the cursor never passes the count (a later re-run on this
-    // stream must still find the entries appended after this one)
-    if (L == 0) {
-      int p = count;
-      int cur = *(volatile int32_t *)a.ovf_cursor;
-      while (cur < count) {
-        const int seen = atomicCAS(a.ovf_cursor, cur, cur + 1);
-        if (seen == cur) { p = cur; break; }
-        cur = seen;
-      }
-      claim_s = p;
-    }
+    if (L == 0) claim_s = k2_claim(a, a.ovf_cursor, count, false);
     __syncthreads();
     const int p = claim_s;
     if (p >= count) break;
     const int q = a.ovf[p].x, s = a.ovf[p].y;
     const int m = (int)(a.qoff[q + 1] - a.qoff[q]);
-    const uint8_t *qc = a.qcodes + a.qoff[q];
     const int len = a.sorted_len[s];
-    const GroupInfo G = a.groups[s / kGroup];
-    const int gl = s % kGroup;
-    // the 32-bit word of codes of tile tt (columns tt*4 .. tt*4+3 of this lane's sequence)
-    auto codes_of = [&](int tt) -> uint32_t {
-      const int col = tt * K2C;
-      return __ldg(words + ((G.word_off + (int64_t)(col >> 4) * kGroup + gl) * 4 + ((col & 15) >> 2)));
-    };
-    const int ntile = (len + K2C - 1) / K2C;   // columns up to ntile*4 <= G.ncols are pad codes
+    const int ntile = (len + K2C - 1) / K2C;
     const int nch = (m + CH - 1) / CH;
     int best = 0;
     for (int ch = 0; ch < nch && len > 0; ch++) {
       const int r0 = ch * CH;
       const int nact = min(kK2Threads, (m - r0 + K2R - 1) / K2R);   // threads with real rows
-      const bool active = L < nact;
-      int rowoff[K2R];
-#pragma unroll
-      for (int i = 0; i < K2R; i++) {
-        const int row = r0 + L * K2R + i;
-        rowoff[i] = (row < m ? (int)qc[row] : kPadCode) * (kNCodes * 32) + lane;
-      }
-      int H[K2R], E[K2R];
-#pragma unroll
-      for (int i = 0; i < K2R; i++) { H[i] = 0; E[i] = 0; }
-      int hprev_top = 0;
-      const int steps = ntile + nact - 1;
-      // register prefetch, one step ahead: this thread's next codes word and (thread 0 of
-      // a later chunk) the next border entries
-      uint32_t cw_next = (active && L == 0 && ntile > 0) ? codes_of(0) : 0u;
-      int2 bnext[K2C];
-#pragma unroll
-      for (int g = 0; g < K2C; g++)
-        bnext[g] = (L == 0 && ch > 0) ? make_int2(border[2 * g], border[2 * g + 1]) : make_int2(0, 0);
-      for (int t = 0; t < steps; t++) {
-        const int tile = t - L;
-        if (active && tile >= 0 && tile < ntile) {
-          const uint32_t cw = cw_next;
-          if (tile + 1 < ntile) cw_next = codes_of(tile + 1);
-          int2 in[K2C];
-          if (L == 0) {
-#pragma unroll
-            for (int g = 0; g < K2C; g++) in[g] = bnext[g];
-            if (ch > 0 && tile + 1 < ntile)
-#pragma unroll
-              for (int g = 0; g < K2C; g++) {
-                const int col = (tile + 1) * K2C + g;
-                bnext[g] = make_int2(border[2 * col], border[2 * col + 1]);
-              }
-          } else {
-#pragma unroll
-            for (int g = 0; g < K2C; g++) in[g] = hand[(((t - 1) & 1) * K2C + g) * kK2Threads + L - 1];
-          }
-          int coff[K2C], hd[K2C], f[K2C], oh[K2C];
-#pragma unroll
-          for (int g = 0; g < K2C; g++) {
-            coff[g] = (int)((cw >> (8 * g)) & 0xffu) * 32;
-            hd[g] = hprev_top;
-            f[g] = in[g].y;
-            hprev_top = in[g].x;
-          }
-          // skewed tile: at sub-step k column g updates row k - g (K2C independent chains)
-#pragma unroll
-          for (int k = 0; k < K2R + K2C - 1; k++) {
-#pragma unroll
-            for (int g = 0; g < K2C; g++) {
-              const int i = k - g;
-              if (i >= 0 && i < K2R) {
-                // x on the FMA pipe (IMAD by an opaque 1): a plain add would be fused by
-                // ptxas into a VIADDMNMX + VIMNMX pair, one more ALU op per cell
-                const int x = Ms[rowoff[i] + coff[g]] * one + hd[g];
-                const int h = __vimax3_s32(x, E[i], f[g]);      // >= 0: E, F floored at 0
-                const int tt = __viaddmax_s32(h, na, 0);        // max(H - alpha, 0)
-                E[i] = __viaddmax_s32(E[i], nb, tt);            // E(i, j+1)
-                f[g] = __viaddmax_s32(f[g], nb, tt);            // F(i+1, j)
-                hd[g] = H[i];
-                H[i] = h;
-                best = max(best, h);
-                if (i == K2R - 1) oh[g] = h;
-              }
-            }
-          }
-#pragma unroll
-          for (int g = 0; g < K2C; g++) hand[((t & 1) * K2C + g) * kK2Threads + L] = make_int2(oh[g], f[g]);
-          if (L == nact - 1 && ch < nch - 1)
-#pragma unroll
-            for (int g = 0; g < K2C; g++) {
-              const int col = tile * K2C + g;
-              border[2 * col] = oh[g];
-              border[2 * col + 1] = f[g];
-            }
-        } else if (active && L > 0 && tile == -1 && ntile > 0) {
-          cw_next = codes_of(0);   // first tile of this thread starts next step
-        }
-        __syncthreads();
-      }
+      best = max(best, k2_chunk<K2R>(a, Ms, hand, a.qcodes + a.qoff[q], m, r0, nact, a.groups[s / kGroup], s % kGroup,
+                                ntile, ch > 0 ? border : nullptr, ch < nch - 1 ? border : nullptr, nullptr,
+                                nullptr, 0, ring));
     }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) best = max(best, __shfl_xor_sync(0xffffffffu, best, o));
-    if (lane == 0) red_s[L >> 5] = best;
-    __syncthreads();
-    if (L == 0) {
-      int b = 0;
-      for (int w = 0; w < kK2Threads / 32; w++) b = max(b, red_s[w]);
-      a.scores[(int64_t)q * a.ndb + a.perm[s]] = b;
-    }
+    const int b = block_max(best);
+    if (L == 0) a.scores[(int64_t)q * a.ndb + a.perm[s]] = b;
     __syncthreads();   // claim_s / red_s / hand reused by the next pair
   }
 }
 
+// blocks: a multiple of kK2Cluster (clusters of kK2Cluster CTAs); a.k2prog: blocks int64
+// counters, zeroed before the launch on its stream
 void launch_k2(const K2Args &a, int blocks, cudaStream_t st) {
   cudaFuncSetAttribute(k2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kK2Smem);
-  k2_kernel<<<blocks, kK2Threads, kK2Smem, st>>>(a);
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3((blocks + kK2Cluster - 1) / kK2Cluster * kK2Cluster);
+  cfg.blockDim = dim3(kK2Threads);
+  cfg.dynamicSmemBytes = kK2Smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = kK2Cluster;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  cudaLaunchKernelEx(&cfg, k2_kernel, a);
 }
 
 // ------------------------------------------------------------------------------------

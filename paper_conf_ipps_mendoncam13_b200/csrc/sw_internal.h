@@ -122,16 +122,19 @@ struct K3Args {   // sequences [l0,l1) in sorted order (the long groups) x packs
 };
 constexpr int kMaxStreams = 64;    // sw_opts.streams_per_device limit
 constexpr int kK2Blocks = 16;      // K2 blocks per launch (one block per saturated pair at a time)
+constexpr int kK2Cluster = 8;      // K2 CTAs that split one big saturated pair (kK2Blocks / kK2Cluster clusters)
 struct K2Args {   // int32 re-run of saturated pairs (block per pair)
   const uint8_t *qcodes; const int64_t *qoff;
   const uint4 *packed; const GroupInfo *groups; const int32_t *sorted_len; const int32_t *perm;
   const int8_t *matrix;                   // 24x24 (device)
   const int2 *ovf; const int32_t *ovf_count; int32_t ovf_cap;
-  int32_t *ovf_cursor;                    // blocks take entries with atomicCAS
+  int32_t *ovf_cursor;                    // [2]: small / big pairs, taken with atomicCAS
+  int64_t big_cells;                      // m*n at which a pair is split over a cluster
   int32_t *scores; int64_t ndb;
   int32_t alpha, beta;
   int32_t one;                              // = 1 (opaque to the compiler, see k2_kernel)
   int32_t *border; int64_t border_stride;   // per-block border row (2 x int32 per column)
+  long long *k2prog;                        // per-block progress counters (big pairs), zeroed
 };
 
 struct TbPair {     // one pair of a traceback batch

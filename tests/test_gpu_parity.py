@@ -548,7 +548,7 @@ print("ok", r.stats["n_cancelled"], r.stats["n_wa_grants"])
 """
 
 
-@pytest.mark.parametrize("cluster", ["2", "4"])
+@pytest.mark.parametrize("cluster", ["2", "3", "4", "5", "8"])
 def test_k3_cluster_split(cluster):
     """K3 with each pair's chunks split over a thread-block cluster (SW_K3_CLUSTER forces the
     size; auto picks it for small long-sequence shares): bit-exact on C5-shaped pairs with an
@@ -581,3 +581,39 @@ def test_traceback_gaps_across_chunks():
         _check_alignment(qs.seq(int(qi[k])).decode(), db.seq(int(di[k])).decode(), a)
     assert "I" * 40 in al[0]["ops"]
     D.close()
+
+
+_K2_SCRIPT = """
+import os, sys; sys.path.insert(0, %r); sys.path.insert(0, os.path.join(sys.path[0], "tests"))
+import test_gpu_parity as T
+T.test_overflow_rerun_int32()
+T.test_big_matrix_forces_many_overflows()
+T.test_overflow_rerun_multi_chunk()
+T.test_precision_routing_large_gaps()
+# every pair through K2 (alpha + beta > 16384): queries whose cluster chunks use 4, 8 and
+# 16 rows per thread, against short, ragged and empty sequences
+import numpy as np, oracle, seqgen
+qs = seqgen.SeqSet.from_list([seqgen.residues(71, 0, L).tobytes() for L in (40000, 20000, 9000, 4000, 33)])
+db = seqgen.SeqSet.from_list([seqgen.residues(72, k, L).tobytes() for k, L in enumerate((1500, 7, 0, 2001, 640))])
+ref = oracle.search(qs, db, gap_open=20000, gap_extend=3)
+r = T._search(db, qs, gap_open=20000, gap_extend=3, top_k=2)
+assert (r.scores == ref).all(), np.argwhere(r.scores != ref)[:5]
+print("ok")
+"""
+
+
+@pytest.mark.parametrize("big", ["1", "2000000"])
+def test_k2_cluster_split(big):
+    """K2 splits a big saturated pair over a cluster of 8 CTAs (chunk r on CTA r, borders
+    through L2 with epoch-tagged progress counters).  SW_K2_BIG lowers the size at which a
+    pair counts as big: "1" sends every re-run pair (down to a 4-aa query, fewer chunks
+    than CTAs) through the cluster path, "2000000" mixes both paths in one launch.  Every
+    overflow / int32-routing case stays bit-exact against the oracle."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, SW_K2_BIG=big)
+    out = subprocess.run([sys.executable, "-c", _K2_SCRIPT % root], env=env, capture_output=True,
+                         text=True, timeout=900, cwd=root)
+    assert out.returncode == 0 and "ok" in out.stdout, (out.stdout[-2000:], out.stderr[-3000:])

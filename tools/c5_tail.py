@@ -19,9 +19,10 @@ ap.add_argument("--config", default="C5")
 ap.add_argument("--unit-cells", type=int, nargs="*", default=[0])
 ap.add_argument("--streams", type=int, nargs="*", default=[4])
 ap.add_argument("--reps", type=int, default=3)
+ap.add_argument("--n-db", type=int, default=None)
 args = ap.parse_args()
 
-w = seqgen.make_workload(args.config)
+w = seqgen.make_workload(args.config, n_db=args.n_db) if args.n_db else seqgen.make_workload(args.config)
 D = Database(w.db, devices=[0])
 cells = int(w.meta["cells"])
 for uc in args.unit_cells:
@@ -40,7 +41,8 @@ for uc in args.unit_cells:
         print(json.dumps({"unit_cells": uc, "streams": ns, "sec": best["seconds_device"],
                           "gcups": cells / best["seconds_device"] / 1e9, "units": len(log),
                           "last_start_ms": 1e3 * last_start, "end_ms": 1e3 * end,
-                          "k3_kernel_s": best["kernel_seconds_k3"], "k1_kernel_s": best["kernel_seconds_k1"],
+                          "k3_kernel_s": best["kernel_seconds_k3"], "k2_kernel_s": best["kernel_seconds_k2"],
+                          "last_unit_end_dev_ms": max(e["dev_t1"] for e in log), "k1_kernel_s": best["kernel_seconds_k1"],
                           "longest_units_ms": [round(d, 1) for d, _, _ in durs[-6:]],
                           "shortest_units_ms": [round(d, 1) for d, _, _ in durs[:3]]}), flush=True)
 D.close()
