@@ -125,13 +125,16 @@ struct DevSearch {
   int64_t k3_rows = 0;
   DBuf<int32_t> k3_prog;   // [streams][k3 slots x warps]: clustered K3 progress counters
   DBuf<int32_t> k2_border;
-  DBuf<long long> k2_prog;   // [streams][kK2Blocks]: big-pair progress counters (K2 clusters)
+  DBuf<K2Ctl> k2_ctl;        // [streams]: big-pair tickets, slots and progress counters (K2)
   DBuf<int32_t> abort_dev;      // per-unit WA cancellation flags (device memory)
   DBuf<int32_t> progress;       // per-unit progress counters (K1 groups / K3 sequence-chunks)
   DBuf<int32_t> gclaim;         // per-unit K1 group claim counters
   int32_t *abort_d = nullptr;
   int32_t *one_h = nullptr;      // pinned constant 1, source of the cancellation copies
   int32_t *ovf_seen_h = nullptr; // pinned [kMaxStreams]: ovf_count copied after each unit
+  int32_t *ovf_early_h = nullptr;// pinned, mapped [kMaxStreams]: entries listed, written by the
+                                 // DP kernels as they list them (early int32 re-run launch)
+  int32_t *ovf_early_d = nullptr;// its device address
   int32_t *prog_h = nullptr;     // pinned [kMaxStreams]: the unit's progress after it ran
   cudaStream_t cancel_st = nullptr;
   cudaStream_t noise_st = nullptr;   // high priority: the local-load kernel (straggler mode 2)
@@ -189,6 +192,7 @@ struct Device {
 inline DevSearch::~DevSearch() {
   if (one_h) cudaFreeHost(one_h);
   if (ovf_seen_h) cudaFreeHost(ovf_seen_h);
+  if (ovf_early_h) cudaFreeHost(ovf_early_h);
   if (prog_h) cudaFreeHost(prog_h);
   if (cancel_st) cudaStreamDestroy(cancel_st);
   if (noise_st) cudaStreamDestroy(noise_st);
@@ -648,10 +652,10 @@ static K2Args k2_args(const Plan &P, const PackedDB &db, DevSearch &S, int strea
   // 2^24 cells take ~1 ms on one SM
   static const int64_t big = [] { const char *e = getenv("SW_K2_BIG"); return e && atoll(e) > 0 ? atoll(e) : (1LL << 24); }();
   a.big_cells = big;
-  a.k2prog = S.k2_prog.p + (size_t)stream_idx * kK2Blocks;
+  a.ctl = S.k2_ctl.p + stream_idx;
   a.scores = S.scores; a.ndb = db.n; a.alpha = alpha; a.beta = beta; a.one = 1;
   const int64_t stride = k2_stride(P);
-  a.border = S.k2_border.p + (size_t)stream_idx * kK2Blocks * stride * 2;
+  a.border = S.k2_border.p + (size_t)stream_idx * kK2Rows * stride * 2;
   a.border_stride = stride;
   return a;
 }
@@ -679,6 +683,7 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     a.thresh = thresh;
     a.ovf = S.ovf.p + (size_t)stream_idx * S.ovf_cap; a.ovf_count = S.ovf_count.p + stream_idx;
     a.ovf_cap = S.ovf_cap; a.ovf_bits = S.ovf_bits.p;
+    a.ovf_early = S.ovf_early_d + stream_idx;
     a.border = D.k1_border.p; a.border_slot_cols = D.slot_cols; a.slots_per_sm = D.slots_per_sm;
     a.slot_busy = D.slot_busy.p;
     a.abort_flag = S.abort_d + uidx;
@@ -696,6 +701,7 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     a.thresh = thresh;
     a.ovf = S.ovf.p + (size_t)stream_idx * S.ovf_cap; a.ovf_count = S.ovf_count.p + stream_idx;
     a.ovf_cap = S.ovf_cap; a.ovf_bits = S.ovf_bits.p;
+    a.ovf_early = S.ovf_early_d + stream_idx;
     const int64_t stride = (std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16;  // >= tiles * T
     a.border = S.k3_border.p + (size_t)stream_idx * S.k3_rows * stride;
     a.border_stride = stride;
@@ -942,9 +948,9 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       X.ovf.ensure(D.id, (size_t)depth * X.ovf_cap);
       X.ovf_count.ensure(D.id, depth);
       X.ovf_cursor.ensure(D.id, 2 * depth);
-      X.k2_prog.ensure(D.id, (size_t)depth * kK2Blocks);
+      X.k2_ctl.ensure(D.id, (size_t)depth);
       X.ovf_bits.ensure(D.id, ((size_t)nq * nd + 31) / 32);
-      X.k2_border.ensure(D.id, (size_t)depth * kK2Blocks * k2_stride(P) * 2);
+      X.k2_border.ensure(D.id, (size_t)depth * kK2Rows * k2_stride(P) * 2);
       const size_t k3b = (size_t)depth * k3_rows * ((std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16);
       if (P.n_long_seqs > 0) X.k3_border.ensure(D.id, k3b);
       if (any_cluster) X.k3_prog.ensure(D.id, (size_t)depth * (k3_slots * kK3Warps + 1));
@@ -969,7 +975,10 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         *X.one_h = 1;
         CK(cudaHostAlloc((void **)&X.ovf_seen_h, sizeof(int32_t) * kMaxStreams, cudaHostAllocDefault));
         CK(cudaHostAlloc((void **)&X.prog_h, sizeof(int32_t) * kMaxStreams, cudaHostAllocDefault));
+        CK(cudaHostAlloc((void **)&X.ovf_early_h, sizeof(int32_t) * kMaxStreams, cudaHostAllocMapped));
+        CK(cudaHostGetDevicePointer((void **)&X.ovf_early_d, X.ovf_early_h, 0));
       }
+      for (int k = 0; k < kMaxStreams; k++) ((volatile int32_t *)X.ovf_early_h)[k] = 0;
       if (!X.cancel_st) CK(cudaStreamCreateWithFlags(&X.cancel_st, cudaStreamNonBlocking));
       {
         int lo = 0, hi = 0;
@@ -1080,6 +1089,9 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         launch_fill(X.scores, (int64_t)nq * nd, -1, s0);
         CK(cudaMemsetAsync(X.ovf_count.p, 0, sizeof(int32_t) * depth, s0));
         CK(cudaMemsetAsync(X.ovf_cursor.p, 0, sizeof(int32_t) * 2 * depth, s0));
+        // list slots read (-1, -1) until written: a K2 running beside the unit that lists an
+        // entry may see it counted before it is stored
+        CK(cudaMemsetAsync(X.ovf.p, 0xff, sizeof(int2) * (size_t)depth * X.ovf_cap, s0));
         CK(cudaMemsetAsync(X.ovf_bits.p, 0, sizeof(uint32_t) * (((size_t)nq * nd + 31) / 32), s0));
         launch_profile(X.qcodes.p, X.qoff.p, X.pairs.p, (int)P.pairs.size(), X.slices.p, X.matrix.p,
                        X.prof.p, P.prof_total, s0);
@@ -1106,6 +1118,23 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         std::vector<double> hold_until(depth, 0);
         std::vector<int> completed_wait(depth, 0), slowed(depth, 0);
         std::vector<int32_t> k2_upto(depth, 0);   // saturated pairs handed to K2 per stream
+        // the int32 re-run (K2) of stream k's saturated pairs once `seen` of them are listed,
+        // on the epilogue stream
+        auto launch_rerun = [&](int k, int32_t seen) {
+          if (seen <= k2_upto[k]) return;
+          const K2Args k2a = k2_args(P, H, X, k, alpha, beta);
+          std::pair<cudaEvent_t, cudaEvent_t> ev;
+          CK(cudaEventCreate(&ev.first));
+          CK(cudaEventCreate(&ev.second));
+          X.k2_ev.push_back(ev);
+          CK(cudaMemsetAsync(k2a.ctl, 0, sizeof(K2Ctl), X.epi[0]));
+          CK(cudaEventRecord(ev.first, X.epi[0]));
+          launch_k2(k2a, kK2Blocks, X.epi[0]);
+          CK(cudaEventRecord(ev.second, X.epi[0]));
+          CK(cudaGetLastError());
+          X.launches++;
+          k2_upto[k] = seen;
+        };
         bool done = false, changed = true;
         double last_req = 0, req_gap = 2e-3;
         std::vector<double> stream_rate(depth, 0.0);
@@ -1124,6 +1153,13 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
             CK(cudaGetLastError());
             noise_on = true;
           }
+          // saturated pairs listed by running units (published by the DP kernels as they list
+          // them): their int32 re-run starts now, beside the unit, instead of after it -- a
+          // long pair's re-run was the tail of C5 at 1/8 of its database (SW_K2_EARLY=0: after
+          // the unit; C5 at 1/8 5.05 vs 4.85 TCUPS, full C5 6.06 vs 6.03)
+          static const bool early = [] { const char *e = getenv("SW_K2_EARLY"); return !(e && atoi(e) == 0); }();
+          if (early)
+            for (int k = 0; k < depth; k++) launch_rerun(k, ((volatile int32_t *)X.ovf_early_h)[k]);
           // completions
           for (int k = 0; k < depth; k++) {
             if (inflight[k] < 0) continue;
@@ -1196,21 +1232,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
             // own stream they delayed its next unit (C4 at 1/8 of its database: 16 % idle).
             // K2 may see entries a later unit on the stream is appending: it recomputes such
             // a pair exactly, and the later partial maxima of its other slices are smaller.
-            const int32_t seen = ((volatile int32_t *)X.ovf_seen_h)[k];
-            if (seen > k2_upto[k]) {
-              const K2Args k2a = k2_args(P, H, X, k, alpha, beta);
-              std::pair<cudaEvent_t, cudaEvent_t> ev;
-              CK(cudaEventCreate(&ev.first));
-              CK(cudaEventCreate(&ev.second));
-              X.k2_ev.push_back(ev);
-              CK(cudaMemsetAsync(k2a.k2prog, 0, sizeof(long long) * kK2Blocks, X.epi[0]));
-              CK(cudaEventRecord(ev.first, X.epi[0]));
-              launch_k2(k2a, kK2Blocks, X.epi[0]);
-              CK(cudaEventRecord(ev.second, X.epi[0]));
-              CK(cudaGetLastError());
-              X.launches++;
-              k2_upto[k] = seen;
-            }
+            launch_rerun(k, ((volatile int32_t *)X.ovf_seen_h)[k]);
             if (committed) {
               X.committed.push_back(u);
               // K5u: this unit's top-k per query of its pack (after its int32 re-run)

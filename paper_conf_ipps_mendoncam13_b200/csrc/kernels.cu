@@ -125,17 +125,26 @@ struct Cell {
 
 // One half of a lane's running maximum (offset representation) for query q: saturated
 // halves go to the int32 re-run list, the others raise the score with atomicMax (a query
-// spans several warps / lanes / bands, each contributes the maximum over its rows).
+// spans several warps / lanes / bands, each contributes the maximum over its rows).  A
+// listed entry is published to the host (ovf_early, host-mapped) so that the worker can
+// start the int32 re-run while the unit still runs; list slots hold (-1, -1) until written.
 __device__ __forceinline__ void flush_half(int q, int v, int ss, int orig, int32_t *scores,
                                            int64_t ndb, int thresh, int2 *ovf, int32_t *ovf_count,
-                                           int ovf_cap, uint32_t *ovf_bits) {
+                                           int ovf_cap, uint32_t *ovf_bits, int32_t *ovf_early) {
   if (q < 0) return;
   if (v >= thresh) {   // several warps / lanes may saturate on one pair: list it once
     const int64_t bit = (int64_t)q * ndb + orig;
     const uint32_t m = 1u << (bit & 31);
     if (!(atomicOr(ovf_bits + (bit >> 5), m) & m)) {
       const int k = atomicAdd(ovf_count, 1);
-      if (k < ovf_cap) ovf[k] = make_int2(q, ss);
+      if (k < ovf_cap) {
+        ovf[k] = make_int2(q, ss);
+        if (ovf_early) {   // a hint: two writers may land out of order (the worker also reads
+                           // the device count after every unit), so a plain store, no host atomics
+          __threadfence_system();   // the entry before the host sees its count
+          *(volatile int32_t *)ovf_early = k + 1;
+        }
+      }
     }
   } else {
     atomicMax(scores + (int64_t)q * ndb + orig, v - kOff);
@@ -318,9 +327,9 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
           if (lane < G.count) {
             const int ss = G.first + lane, orig = a.perm[ss];
             if (si.q_lo != cq_lo)
-              flush_half(cq_lo, lo16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
+              flush_half(cq_lo, lo16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits, a.ovf_early);
             if (si.q_hi != cq_hi)
-              flush_half(cq_hi, hi16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
+              flush_half(cq_hi, hi16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits, a.ovf_early);
           }
           if (si.q_lo != cq_lo) best = (best & 0xffff0000u) | (koff & 0xffffu);
           if (si.q_hi != cq_hi) best = (best & 0x0000ffffu) | (koff & 0xffff0000u);
@@ -411,8 +420,8 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
           band = 0;
           if (lane < G.count) {   // end of the group: flush both halves
             const int ss = G.first + lane, orig = a.perm[ss];
-            flush_half(cq_lo, lo16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
-            flush_half(cq_hi, hi16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
+            flush_half(cq_lo, lo16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits, a.ovf_early);
+            flush_half(cq_hi, hi16(best), ss, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits, a.ovf_early);
           }
           best = koff;
           cq_lo = cq_hi = -1;
@@ -659,12 +668,12 @@ __global__ void __launch_bounds__(kK3Warps * 32, 4) k3_kernel(const K3Args a) {
         const int sidx = ch * 32 + lane;
         const SliceInfo si = a.slices[P.slice_off + sidx];
         if (si.q_lo != cq_lo) {
-          flush_half(cq_lo, lo16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
+          flush_half(cq_lo, lo16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits, a.ovf_early);
           best = (best & 0xffff0000u) | (koff & 0xffffu);
           cq_lo = si.q_lo;
         }
         if (si.q_hi != cq_hi) {
-          flush_half(cq_hi, hi16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
+          flush_half(cq_hi, hi16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits, a.ovf_early);
           best = (best & 0x0000ffffu) | (koff & 0xffff0000u);
           cq_hi = si.q_hi;
         }
@@ -801,8 +810,8 @@ __global__ void __launch_bounds__(kK3Warps * 32, 4) k3_kernel(const K3Args a) {
     for (int b = 0; b < C; b++)
       if (C > 1 && nch - 1 > b) cum[b] += ((nch - 1 - b + C - 1) / C) * ntile;
     if (valid && !aborted) {   // every lane flushes what it holds
-      flush_half(cq_lo, lo16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
-      flush_half(cq_hi, hi16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits);
+      flush_half(cq_lo, lo16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits, a.ovf_early);
+      flush_half(cq_hi, hi16(best), s, orig, a.scores, a.ndb, a.thresh, a.ovf, a.ovf_count, a.ovf_cap, a.ovf_bits, a.ovf_early);
     }
     if (C == 1 && aborted) break;   // (C > 1: every CTA of the cluster reaches the claim, which ends)
   }
@@ -909,33 +918,36 @@ void launch_noise(const int32_t *stop, int n_blocks, uint64_t max_ns, uint32_t *
 
 // ------------------------------------------------------------------------------------
 // K2: int32 re-run of saturated (query, sequence) pairs.  Same recurrence as K1/K3 in
-// plain int32 (E and F floored at 0, exact for H: DESIGN.md §6), run by a BLOCK:
-// thread L owns rows [L*K2R, (L+1)*K2R) of a chunk of query rows and runs the wavefront
-// of P14 §II.B (Fig. 3a) across the block -- at step t thread L updates the K2C-column
-// tile t - L and hands its bottom row (H, F) to thread L+1 through a double-buffered
-// shared-memory slot (one __syncthreads per step); the last active thread writes the
-// chunk's bottom row to a global border read by thread 0 of the next chunk.  Scores come
-// from the 25x25 matrix replicated per lane in shared memory ([query code][db code][lane]:
-// bank = lane, no conflicts although every thread is at a different row and column).
-// The CTAs of a launch form clusters of kK2Cluster:
-//  * big pairs (m*n >= big_cells; C5: a 5,000-aa query inside a 35k-residue sequence)
-//    are taken by a whole cluster: CTA r runs chunk r of about m / kK2Cluster rows, and
-//    chunk r+1 (the next CTA) follows it tile by tile through the border row in L2 (a
-//    per-(cluster, boundary) progress counter tagged with the pair's epoch, released
-//    every kK2Pub tiles and acquired before each prefetch; the cluster makes producer and
-//    consumer co-resident, so the wait cannot deadlock).  Round 1 ran such a pair on one
-//    SM (10.4 ms for C5's planted pair), the tail of a small per-GPU share of C5;
-//  * the other pairs are taken by single CTAs, chunks of kK2Threads*K2R rows in order.
+// plain int32 (E and F floored at 0, exact for H: DESIGN.md §6), run by a BLOCK of
+// kK2Threads: thread L owns rows [L*R, (L+1)*R) of a chunk of 128*R query rows and runs
+// the wavefront of P14 §II.B (Fig. 3a) across the block -- at step t thread L updates the
+// K2C-column tile t - L and hands its bottom row (H, F) and the tile's residue codes to
+// thread L+1 through a double-buffered shared-memory slot (one __syncthreads per step);
+// thread 0 streams the codes and the border row of the chunk above through a cp.async ring.
+// Scores come from a per-chunk int8 profile [code][thread][R] in shared memory: one LDS of
+// R bytes per column and thread, bank = thread (no conflicts).
+// A block is the size of a K3 block (128 threads, <= 128 registers, ~60 KB of shared
+// memory), so it starts in the SM slot that one K3 block leaves: a 512-thread block that
+// needed a whole SM waited behind the persistent K3 blocks until the step's end.
+// Two kinds of pairs:
+//  * big pairs (m*n >= big_cells; C5: a 5,000-aa query inside a 35k-residue sequence) are
+//    split into chunks run by as many blocks at once: chunk r+1 follows chunk r tile by
+//    tile through a border row in L2 (a progress counter tagged with the pair's number,
+//    released every kK2Pub tiles and acquired before each prefetch).  Blocks take chunk
+//    tickets in order, so a chunk only waits for chunks whose blocks already run (no
+//    co-scheduling needed).  One block per pair ran C5's planted pair in 12.3 ms;
+//  * the other pairs are taken by single blocks, chunks of 128*kK2RSmall rows in order.
 // Each list has its own cursor (small: ovf_cursor[0], big: ovf_cursor[1]); a cursor
 // skips the other kind's entries and never passes the count this launch saw.
 // ------------------------------------------------------------------------------------
-constexpr int K2R = 16;          // rows per thread
 constexpr int K2C = 4;           // columns per tile (one aligned 32-bit word of codes)
-constexpr int kK2Threads = 512;  // threads per block (chunk <= 8,192 rows)
+constexpr int kK2RSmall = 16;    // rows per thread of a single-block pair (2,048-row chunks)
+constexpr int kK2MaxR = 16;
 constexpr int kK2Pub = 8;        // tiles between a big pair's progress publications
-constexpr int kK2Ring = 8;       // border-row tiles in flight (thread 0's cp.async ring)
-constexpr size_t kK2Smem = sizeof(int32_t) * kNCodes * kNCodes * 32 + sizeof(int2) * 2 * kK2Threads * K2C;
-static_assert(kK2Cluster * kK2Threads * K2R > SW_MAX_QUERY_LEN, "a big pair is at most one chunk per CTA");
+constexpr int kK2Ring = 8;       // tiles in flight (thread 0's cp.async ring)
+constexpr size_t kK2Smem = (size_t)kNCodes * kK2Threads * kK2MaxR + sizeof(int2) * 2 * kK2Threads * K2C +
+                           sizeof(uint32_t) * 2 * kK2Threads;
+static_assert(kK2Span * kK2Threads * kK2MaxR > SW_MAX_QUERY_LEN, "a big pair is at most kK2Span chunks");
 
 __device__ __forceinline__ long long ld_acquire64(const long long *p) {
   long long v;
@@ -946,36 +958,82 @@ __device__ __forceinline__ void st_release64(long long *p, long long v) {
   asm volatile("st.release.gpu.global.b64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-// claim the next entry of one kind from cursor `cur` (thread 0); returns count when none
-__device__ __forceinline__ int k2_claim(const K2Args &a, int *cur_p, int count, bool big) {
+// claim the next entry of one kind from cursor `cur` (thread 0); returns count when none.
+// An entry counted but not yet written (its writer is between the atomicAdd and the store:
+// K2 can run beside the unit that lists it) still holds (-1, -1): wait for it
+__device__ __forceinline__ int k2_claim(const K2Args &a, int *cur_p, int count, bool big, int2 &entry) {
   int cur = *(volatile int32_t *)cur_p;
   while (cur < count) {
-    const int2 e = a.ovf[cur];
+    int2 e;
+    const long long t_wait = clock64();
+    while (true) {
+      const long long v = *(const volatile long long *)(a.ovf + cur);   // one 8-byte load
+      e = make_int2((int)(v & 0xffffffffll), (int)(v >> 32));
+      if (e.x >= 0) break;
+      if (clock64() - t_wait > (1ll << 36)) __trap();
+    }
     const int64_t cells = (a.qoff[e.x + 1] - a.qoff[e.x]) * (int64_t)a.sorted_len[e.y];
     const int seen = atomicCAS(cur_p, cur, cur + 1);
     if (seen != cur) { cur = seen; continue; }          // someone else moved it: retry there
-    if ((cells >= a.big_cells) == big) return cur;      // ours
+    if ((cells >= a.big_cells) == big) { entry = e; return cur; }   // ours
     cur++;                                              // skipped (the other kind's)
   }
   return count;
 }
 
-// One chunk [r0, r0 + nact*R) (R rows per thread) of pair (qc, m) x (sequence of group G, lane gl) on this
+template <int R> struct K2Word;
+template <> struct K2Word<4> { typedef uint32_t T; };
+template <> struct K2Word<8> { typedef uint2 T; };
+template <> struct K2Word<16> { typedef uint4 T; };
+template <int R>
+__device__ __forceinline__ int k2_score(const typename K2Word<R>::T &w, int i) {   // signed byte i
+  uint32_t v;
+  if constexpr (R == 4) v = w;
+  else if constexpr (R == 8) v = (i < 4) ? w.x : w.y;
+  else v = (i < 4) ? w.x : (i < 8) ? w.y : (i < 12) ? w.z : w.w;
+  return (int)(int8_t)(v >> (8 * (i & 3)));
+}
+
+// One chunk [r0, r0 + nact*R) of pair (qc, m) x (sequence of group G, lane gl) on this
 // block; returns this thread's maximum H.  bin / bout: border rows in / out (nullptr: the
 // first / last chunk); prog_in / prog_out: (big pairs) the producer's / this chunk's
 // progress counter, values (epoch << 32) + tiles.  bin == bout is allowed when the chunks
 // of a pair run in order on one block (the writer trails the reader by nact tiles).
 template <int R>
-__device__ __forceinline__ int k2_chunk(const K2Args &a, const int32_t *Ms, int2 *hand, const uint8_t *qc,
+__device__ __forceinline__ int k2_chunk(const K2Args &a, const int8_t *Ms, int8_t *prof, int2 *hand,
+                                        uint32_t *handc, int2 *ring, uint32_t *cring, const uint8_t *qc,
                                         int m, int r0, int nact, const GroupInfo &G, int gl, int ntile,
                                         const int2 *bin, int2 *bout, const long long *prog_in,
-                                        long long *prog_out, long long epoch, int2 *ring) {
-  const int L = threadIdx.x, lane = L & 31;
+                                        long long *prog_out, long long epoch) {
+  typedef typename K2Word<R>::T W;
+  const int L = threadIdx.x;
   const uint32_t *words = reinterpret_cast<const uint32_t *>(a.packed);
-  const int na = -a.alpha, nb = -a.beta, one = a.one;
-  auto codes_of = [&](int tt) -> uint32_t {   // codes of columns tt*4 .. tt*4+3 (32-bit word)
+  const int na = -a.alpha, nb = -a.beta;
+  // this chunk's profile: byte i of prof[c][L] = S[q(r0 + L*R + i)][code of slot c]
+  __syncthreads();   // the previous chunk's profile is no longer read
+  {
+    uint32_t pw[R / 4];
+    for (int c = 0; c < kNCodes; c++) {
+#pragma unroll
+      for (int k = 0; k < R / 4; k++) {
+        uint32_t v = 0;
+#pragma unroll
+        for (int b = 0; b < 4; b++) {
+          const int row = r0 + L * R + k * 4 + b;
+          const int sc = (row < m && c < 24) ? (int)Ms[qc[row] * 24 + c_code_of_slot[c]] : kPadScore;
+          v |= (uint32_t)(uint8_t)(int8_t)sc << (8 * b);
+        }
+        pw[k] = v;
+      }
+      uint32_t *dst = reinterpret_cast<uint32_t *>(prof + ((size_t)c * kK2Threads + L) * R);
+#pragma unroll
+      for (int k = 0; k < R / 4; k++) dst[k] = pw[k];
+    }
+  }
+  __syncthreads();
+  auto codes_at = [&](int tt) -> const uint32_t * {   // codes of columns tt*4 .. tt*4+3
     const int col = tt * K2C;
-    return __ldg(words + ((G.word_off + (int64_t)(col >> 4) * kGroup + gl) * 4 + ((col & 15) >> 2)));
+    return words + ((G.word_off + (int64_t)(col >> 4) * kGroup + gl) * 4 + ((col & 15) >> 2));
   };
   // big pairs: wait until the chunk above has published tile tt (thread 0 only)
   long long seen = 0;
@@ -987,52 +1045,51 @@ __device__ __forceinline__ int k2_chunk(const K2Args &a, const int32_t *Ms, int2
     while ((seen = ld_acquire64(prog_in)) < want)
       if (clock64() - t_wait > (1ll << 36)) __trap();   // ~35 s: never hang the GPU
   };
-  // thread 0 streams the border row of the chunk above into a kK2Ring-tile shared-memory
-  // ring with cp.async.cg (L2: never a stale L1 line), kK2Ring - 1 tiles ahead: an L2 round
-  // trip is longer than a step, so a one-step-ahead load would stall every step
+  // thread 0 streams the tile inputs -- the residue codes and the border row of the chunk
+  // above (cp.async.cg: L2, never a stale L1 line) -- into a kK2Ring-tile shared-memory ring,
+  // kK2Ring - 1 tiles ahead: an L2 round trip is longer than a step
   auto fetch = [&](int tt) {
-    if (bin && tt < ntile) {
-      wait_tile(tt);
-      cp_async16_cg(&ring[(tt % kK2Ring) * K2C], bin + tt * K2C);
-      cp_async16_cg(&ring[(tt % kK2Ring) * K2C + 2], bin + tt * K2C + 2);
+    if (tt < ntile) {
+      const unsigned d = (unsigned)__cvta_generic_to_shared(&cring[tt % kK2Ring]);
+      asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(d), "l"(codes_at(tt)) : "memory");
+      if (bin) {
+        wait_tile(tt);
+        cp_async16_cg(&ring[(tt % kK2Ring) * K2C], bin + tt * K2C);
+        cp_async16_cg(&ring[(tt % kK2Ring) * K2C + 2], bin + tt * K2C + 2);
+      }
     }
     asm volatile("cp.async.commit_group;" ::: "memory");
   };
   const bool active = L < nact;
-  int rowoff[R];
-#pragma unroll
-  for (int i = 0; i < R; i++) {
-    const int row = r0 + L * R + i;
-    rowoff[i] = (row < m ? (int)qc[row] : kPadCode) * (kNCodes * 32) + lane;
-  }
   int H[R], E[R];
 #pragma unroll
   for (int i = 0; i < R; i++) { H[i] = 0; E[i] = 0; }
   int hprev_top = 0, best = 0;
   const int steps = ntile + nact - 1;
-  // register prefetch, one step ahead: this thread's next codes word
-  uint32_t cw_next = (active && L == 0 && ntile > 0) ? codes_of(0) : 0u;
   if (L == 0)
     for (int tt = 0; tt < kK2Ring - 1; tt++) fetch(tt);
+  const W *pbase = reinterpret_cast<const W *>(prof) + L;   // + c * kK2Threads
   for (int t = 0; t < steps; t++) {
     const int tile = t - L;
     if (active && tile >= 0 && tile < ntile) {
-      const uint32_t cw = cw_next;
-      if (tile + 1 < ntile) cw_next = codes_of(tile + 1);
+      uint32_t cw;
       int2 in[K2C];
       if (L == 0) {
         fetch(tile + kK2Ring - 1);   // into the slot of tile - 1, consumed last step
         asm volatile("cp.async.wait_group %0;" ::"n"(kK2Ring - 1) : "memory");   // tile landed
+        cw = cring[tile % kK2Ring];
 #pragma unroll
         for (int g = 0; g < K2C; g++) in[g] = bin ? ring[(tile % kK2Ring) * K2C + g] : make_int2(0, 0);
       } else {
+        cw = handc[((t - 1) & 1) * kK2Threads + L - 1];
 #pragma unroll
         for (int g = 0; g < K2C; g++) in[g] = hand[(((t - 1) & 1) * K2C + g) * kK2Threads + L - 1];
       }
-      int coff[K2C], hd[K2C], f[K2C], oh[K2C];
+      W sw[K2C];
+      int hd[K2C], f[K2C], oh[K2C];
 #pragma unroll
       for (int g = 0; g < K2C; g++) {
-        coff[g] = (int)((cw >> (8 * g)) & 0xffu) * 32;
+        sw[g] = pbase[((cw >> (8 * g)) & 0xffu) * kK2Threads];
         hd[g] = hprev_top;
         f[g] = in[g].y;
         hprev_top = in[g].x;
@@ -1044,9 +1101,7 @@ __device__ __forceinline__ int k2_chunk(const K2Args &a, const int32_t *Ms, int2
         for (int g = 0; g < K2C; g++) {
           const int i = k - g;
           if (i >= 0 && i < R) {
-            // x on the FMA pipe (IMAD by an opaque 1): a plain add would be fused by
-            // ptxas into a VIADDMNMX + VIMNMX pair, one more ALU op per cell
-            const int x = Ms[rowoff[i] + coff[g]] * one + hd[g];
+            const int x = k2_score<R>(sw[g], i) + hd[g];
             const int h = __vimax3_s32(x, E[i], f[g]);      // >= 0: E, F floored at 0
             const int tt = __viaddmax_s32(h, na, 0);        // max(H - alpha, 0)
             E[i] = __viaddmax_s32(E[i], nb, tt);            // E(i, j+1)
@@ -1060,14 +1115,13 @@ __device__ __forceinline__ int k2_chunk(const K2Args &a, const int32_t *Ms, int2
       }
 #pragma unroll
       for (int g = 0; g < K2C; g++) hand[((t & 1) * K2C + g) * kK2Threads + L] = make_int2(oh[g], f[g]);
+      handc[(t & 1) * kK2Threads + L] = cw;
       if (L == nact - 1 && bout) {
 #pragma unroll
         for (int g = 0; g < K2C; g++) bout[tile * K2C + g] = make_int2(oh[g], f[g]);
         if (prog_out && ((tile + 1) % kK2Pub == 0 || tile + 1 == ntile))
           st_release64(prog_out, (epoch << 32) + tile + 1);   // orders this thread's border stores
       }
-    } else if (active && L > 0 && tile == -1 && ntile > 0) {
-      cw_next = codes_of(0);   // first tile of this thread starts next step
     }
     __syncthreads();
   }
@@ -1075,24 +1129,22 @@ __device__ __forceinline__ int k2_chunk(const K2Args &a, const int32_t *Ms, int2
   return best;
 }
 
-__global__ void __launch_bounds__(kK2Threads, 1) k2_kernel(const K2Args a) {
+__global__ void __launch_bounds__(kK2Threads) k2_kernel(const K2Args a) {
   extern __shared__ __align__(16) int32_t k2s[];
-  int32_t *Ms = k2s;                                              // [qc][dc][lane]
-  int2 *hand = reinterpret_cast<int2 *>(k2s + kNCodes * kNCodes * 32);  // [2][K2C][threads]
-  __shared__ int claim_s;
-  __shared__ int red_s[kK2Threads / 32];
+  int2 *hand = reinterpret_cast<int2 *>(k2s);                                // [2][K2C][threads]
+  uint32_t *handc = reinterpret_cast<uint32_t *>(hand + 2 * K2C * kK2Threads);   // [2][threads]
+  int8_t *prof = reinterpret_cast<int8_t *>(handc + 2 * kK2Threads);          // [codes][threads][R]
+  __shared__ __align__(16) uint32_t cring[kK2Ring];
   __shared__ __align__(16) int2 ring[kK2Ring * K2C];
+  __shared__ int8_t Ms[24 * 24];
+  __shared__ int claim_s;
+  __shared__ int2 claim_e;
+  __shared__ int red_s[kK2Threads / 32];
   const int count = min(*a.ovf_count, a.ovf_cap);
   if (*(volatile int32_t *)a.ovf_cursor >= count && *(volatile int32_t *)(a.ovf_cursor + 1) >= count)
     return;   // nothing saturated (the usual case)
-  for (int k = threadIdx.x; k < kNCodes * kNCodes * 32; k += kK2Threads) {
-    const int r = k / (kNCodes * 32), c = (k / 32) % kNCodes;   // query code, database slot
-    Ms[k] = (r < 24 && c < 24) ? (int32_t)a.matrix[r * 24 + c_code_of_slot[c]] : kPadScore;
-  }
+  for (int k = threadIdx.x; k < 24 * 24; k += kK2Threads) Ms[k] = a.matrix[k];
   const int L = threadIdx.x, lane = L & 31;
-  namespace cg = cooperative_groups;
-  cg::cluster_group cl = cg::this_cluster();
-  const int crank = (int)cl.block_rank(), cid = blockIdx.x / kK2Cluster;
   auto block_max = [&](int best) {   // -> thread 0
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) best = max(best, __shfl_xor_sync(0xffffffffu, best, o));
@@ -1103,55 +1155,97 @@ __global__ void __launch_bounds__(kK2Threads, 1) k2_kernel(const K2Args a) {
       for (int w = 0; w < kK2Threads / 32; w++) b = max(b, red_s[w]);
     return b;
   };
-  // ---- big pairs: one cluster per pair, CTA r = chunk r
-  // border row of boundary r (chunk r -> r+1) of this cluster = block (cid*C + r)'s row
-  int2 *cborder = reinterpret_cast<int2 *>(a.border) + (size_t)cid * kK2Cluster * a.border_stride;
-  long long *cprog = a.k2prog + (size_t)cid * kK2Cluster;
-  for (long long epoch = 1;; epoch++) {
-    if (crank == 0 && L == 0) claim_s = k2_claim(a, a.ovf_cursor + 1, count, true);
-    cl.sync();
-    const int p = *cl.map_shared_rank(&claim_s, 0);
-    cl.sync();   // rank 0 may overwrite claim_s only after every CTA read it
-    if (p >= count) break;
-    const int q = a.ovf[p].x, s = a.ovf[p].y;
+  auto spin_until = [](const volatile int32_t *p, int want) {   // acquire
+    const long long t_wait = clock64();
+    while (true) {
+      int v;
+      asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+      if (v >= want) break;
+      if (clock64() - t_wait > (1ll << 36)) __trap();   // ~35 s: never hang the GPU
+    }
+  };
+  // ---- big pairs: blocks take chunk tickets in order (ticket t = chunk t % kK2Span of big
+  // pair t / kK2Span), so a chunk only ever waits for chunks with earlier tickets, whose
+  // blocks are already running.  Ticket 0 of a pair finds it in the list and publishes it;
+  // pairs alternate between two slots of border rows and progress counters, and a pair
+  // starts only when the pair two before it (same slot) has finished every ticket.
+  K2Ctl *ctl = a.ctl;
+  int2 *bbase = reinterpret_cast<int2 *>(a.border) + (size_t)kK2Blocks * a.border_stride;
+  while (true) {
+    if (L == 0) claim_s = atomicAdd(&ctl->tickets, 1);
+    __syncthreads();
+    const int t = claim_s;
+    const int j = t / kK2Span, c = t % kK2Span, sl = j & 1;
+    K2Pair *pp = &ctl->pairs[j & 7];
+    if (L == 0) {
+      if (c == 0) {
+        spin_until(&ctl->slot_done[sl], j / 2);   // the pair two before has finished
+        int2 e = make_int2(-1, -1);
+        if (k2_claim(a, a.ovf_cursor + 1, count, true, e) >= count) e = make_int2(-1, -1);
+        pp->q = e.x;
+        pp->s = e.y;
+        asm volatile("st.release.gpu.global.b32 [%0], %1;" ::"l"(&pp->tag), "r"(j + 1) : "memory");
+        claim_e = e;
+      } else {
+        spin_until(&pp->tag, j + 1);
+        claim_e = make_int2(*(volatile int32_t *)&pp->q, *(volatile int32_t *)&pp->s);
+      }
+    }
+    __syncthreads();
+    const int q = claim_e.x, s = claim_e.y;
+    auto finish_ticket = [&]() {   // thread 0: this ticket is done with pair j's slot
+      if (atomicAdd(&ctl->chunks_done[sl], 1) == kK2Span - 1) {
+        ctl->chunks_done[sl] = 0;
+        __threadfence();
+        atomicAdd(&ctl->slot_done[sl], 1);
+      }
+    };
+    if (q < 0) {   // no big pair left (every later ticket finds none too)
+      if (L == 0) finish_ticket();
+      break;
+    }
     const int m = (int)(a.qoff[q + 1] - a.qoff[q]);
     const int len = a.sorted_len[s];
     const int ntile = (len + K2C - 1) / K2C;   // columns up to ntile*4 <= G.ncols are pad codes
-    // rows per thread: a CTA holds only m / kK2Cluster rows, so with few threads a step is
-    // latency-bound and fewer rows per thread shorten its dependency chain; the most rows
-    // per thread that still leave <= 192 threads (5,000 x 35,000: 16 -> 4 rows, 7.1 -> 4.9
-    // ms; 30,000 x 20,000: 16 rows, 7.9 ms, 8 rows 9.7 ms)
-    const int per_cta = (m + kK2Cluster - 1) / kK2Cluster;
-    const int R = per_cta <= 4 * 192 ? 4 : per_cta <= 8 * 192 ? 8 : K2R;
-    const int rc = ((m + kK2Cluster - 1) / kK2Cluster + R - 1) / R * R;   // rows per chunk
+    // rows per thread: fewer rows shorten a step's dependency chain (a block is
+    // latency-bound), more rows mean fewer chunks, each adding a pipeline lag of ~nact steps
+    const int R = m <= kK2Threads * 4 * 12 ? 4 : m <= kK2Threads * 8 * 16 ? 8 : 16;
+    const int rc = kK2Threads * R;   // rows per chunk
     const int nch = (m + rc - 1) / rc;
     int best = 0;
-    if (crank < nch && len > 0) {
-      const int r0 = crank * rc;
+    if (c < nch && len > 0) {
+      const int r0 = c * rc;
       const int nact = (min(rc, m - r0) + R - 1) / R;
       const uint8_t *qc = a.qcodes + a.qoff[q];
       const GroupInfo G = a.groups[s / kGroup];
-      int2 *bi = crank > 0 ? cborder + (size_t)(crank - 1) * a.border_stride : nullptr;
-      int2 *bo = crank < nch - 1 ? cborder + (size_t)crank * a.border_stride : nullptr;
-      const long long *pi = crank > 0 ? cprog + crank - 1 : nullptr;
-      long long *po = crank < nch - 1 ? cprog + crank : nullptr;
-      if (R == 4) best = k2_chunk<4>(a, Ms, hand, qc, m, r0, nact, G, s % kGroup, ntile, bi, bo, pi, po, epoch, ring);
-      else if (R == 8) best = k2_chunk<8>(a, Ms, hand, qc, m, r0, nact, G, s % kGroup, ntile, bi, bo, pi, po, epoch, ring);
-      else best = k2_chunk<K2R>(a, Ms, hand, qc, m, r0, nact, G, s % kGroup, ntile, bi, bo, pi, po, epoch, ring);
+      int2 *bi = c > 0 ? bbase + (size_t)(sl * kK2Span + c - 1) * a.border_stride : nullptr;
+      int2 *bo = c < nch - 1 ? bbase + (size_t)(sl * kK2Span + c) * a.border_stride : nullptr;
+      const long long *pi = c > 0 ? &ctl->prog[sl][c - 1] : nullptr;
+      long long *po = c < nch - 1 ? &ctl->prog[sl][c] : nullptr;
+      const long long ep = j + 1;
+      if (R == 4)
+        best = k2_chunk<4>(a, Ms, prof, hand, handc, ring, cring, qc, m, r0, nact, G, s % kGroup, ntile, bi, bo, pi, po, ep);
+      else if (R == 8)
+        best = k2_chunk<8>(a, Ms, prof, hand, handc, ring, cring, qc, m, r0, nact, G, s % kGroup, ntile, bi, bo, pi, po, ep);
+      else
+        best = k2_chunk<16>(a, Ms, prof, hand, handc, ring, cring, qc, m, r0, nact, G, s % kGroup, ntile, bi, bo, pi, po, ep);
     }
     const int b = block_max(best);
-    if (L == 0 && crank < nch) atomicMax(a.scores + (int64_t)q * a.ndb + a.perm[s], b);   // max over chunks
-    __syncthreads();   // red_s / hand reused
+    if (L == 0) {
+      if (c < nch) atomicMax(a.scores + (int64_t)q * a.ndb + a.perm[s], b);   // max over chunks
+      finish_ticket();
+    }
+    __syncthreads();   // claim_s / claim_e / red_s reused
   }
   // ---- the other pairs: one block per pair, chunks in order
   int2 *border = reinterpret_cast<int2 *>(a.border) + (size_t)blockIdx.x * a.border_stride;
-  constexpr int CH = kK2Threads * K2R;
+  constexpr int CH = kK2Threads * kK2RSmall;
   while (true) {
-    if (L == 0) claim_s = k2_claim(a, a.ovf_cursor, count, false);
+    if (L == 0) claim_s = k2_claim(a, a.ovf_cursor, count, false, claim_e);
     __syncthreads();
     const int p = claim_s;
     if (p >= count) break;
-    const int q = a.ovf[p].x, s = a.ovf[p].y;
+    const int q = claim_e.x, s = claim_e.y;
     const int m = (int)(a.qoff[q + 1] - a.qoff[q]);
     const int len = a.sorted_len[s];
     const int ntile = (len + K2C - 1) / K2C;
@@ -1159,34 +1253,21 @@ __global__ void __launch_bounds__(kK2Threads, 1) k2_kernel(const K2Args a) {
     int best = 0;
     for (int ch = 0; ch < nch && len > 0; ch++) {
       const int r0 = ch * CH;
-      const int nact = min(kK2Threads, (m - r0 + K2R - 1) / K2R);   // threads with real rows
-      best = max(best, k2_chunk<K2R>(a, Ms, hand, a.qcodes + a.qoff[q], m, r0, nact, a.groups[s / kGroup], s % kGroup,
-                                ntile, ch > 0 ? border : nullptr, ch < nch - 1 ? border : nullptr, nullptr,
-                                nullptr, 0, ring));
+      const int nact = min(kK2Threads, (m - r0 + kK2RSmall - 1) / kK2RSmall);   // threads with real rows
+      best = max(best, k2_chunk<kK2RSmall>(a, Ms, prof, hand, handc, ring, cring, a.qcodes + a.qoff[q], m, r0, nact,
+                                           a.groups[s / kGroup], s % kGroup, ntile, ch > 0 ? border : nullptr,
+                                           ch < nch - 1 ? border : nullptr, nullptr, nullptr, 0));
     }
     const int b = block_max(best);
     if (L == 0) a.scores[(int64_t)q * a.ndb + a.perm[s]] = b;
-    __syncthreads();   // claim_s / red_s / hand reused by the next pair
+    __syncthreads();   // claim_s / red_s reused by the next pair
   }
 }
 
-// blocks: a multiple of kK2Cluster (clusters of kK2Cluster CTAs); a.k2prog: blocks int64
-// counters, zeroed before the launch on its stream
+// a.ctl zeroed before the launch on its stream; a.border: kK2Rows rows
 void launch_k2(const K2Args &a, int blocks, cudaStream_t st) {
   cudaFuncSetAttribute(k2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kK2Smem);
-  cudaLaunchConfig_t cfg{};
-  cfg.gridDim = dim3((blocks + kK2Cluster - 1) / kK2Cluster * kK2Cluster);
-  cfg.blockDim = dim3(kK2Threads);
-  cfg.dynamicSmemBytes = kK2Smem;
-  cfg.stream = st;
-  cudaLaunchAttribute at[1];
-  at[0].id = cudaLaunchAttributeClusterDimension;
-  at[0].val.clusterDim.x = kK2Cluster;
-  at[0].val.clusterDim.y = 1;
-  at[0].val.clusterDim.z = 1;
-  cfg.attrs = at;
-  cfg.numAttrs = 1;
-  cudaLaunchKernelEx(&cfg, k2_kernel, a);
+  k2_kernel<<<blocks, kK2Threads, kK2Smem, st>>>(a);
 }
 
 // ------------------------------------------------------------------------------------

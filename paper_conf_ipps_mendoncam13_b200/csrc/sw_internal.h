@@ -98,6 +98,7 @@ struct K1Args {
   int32_t *scores; int64_t ndb;      // [nq][ndb]
   int32_t thresh;                    // overflow threshold on best~ (offset repr)
   int2 *ovf; int32_t *ovf_count; int32_t ovf_cap; uint32_t *ovf_bits;
+  int32_t *ovf_early;                // host-mapped: entries listed so far (early K2 launch)
   uint2 *border; int32_t border_slot_cols; int32_t slots_per_sm; int32_t *slot_busy;
   const volatile int32_t *abort_flag; // WA cancellation flag of the unit (polled in the loop)
   int32_t *progress;                 // unit's counter: groups completed (atomicAdd per block)
@@ -111,6 +112,7 @@ struct K3Args {   // sequences [l0,l1) in sorted order (the long groups) x packs
   int32_t *scores; int64_t ndb;
   int32_t thresh;
   int2 *ovf; int32_t *ovf_count; int32_t ovf_cap; uint32_t *ovf_bits;
+  int32_t *ovf_early;                // host-mapped: entries listed so far (early K2 launch)
   uint2 *border; int64_t border_stride;   // border rows (>= max long len): per sequence (C = 1)
                                           // or per (grid slot, buffer) (cluster C > 1)
   int32_t *kprog;                         // C > 1: per (grid slot, buffer) progress counters (zeroed)
@@ -121,8 +123,19 @@ struct K3Args {   // sequences [l0,l1) in sorted order (the long groups) x packs
   uint32_t na, nb;
 };
 constexpr int kMaxStreams = 64;    // sw_opts.streams_per_device limit
-constexpr int kK2Blocks = 16;      // K2 blocks per launch (one block per saturated pair at a time)
-constexpr int kK2Cluster = 8;      // K2 CTAs that split one big saturated pair (kK2Blocks / kK2Cluster clusters)
+constexpr int kK2Blocks = 32;      // K2 blocks per launch
+constexpr int kK2Threads = 128;    // K2 block size (the size of a K3 block)
+constexpr int kK2Span = 32;        // chunk tickets per big saturated pair (at most kK2Span chunks)
+constexpr int kK2Rows = kK2Blocks + 2 * kK2Span;   // K2 border rows per stream
+struct K2Pair { int32_t tag, q, s, pad; };   // a published big pair (tag = pair number + 1)
+struct K2Ctl {                     // per stream, zeroed before each K2 launch
+  int32_t tickets;                 // chunk tickets taken: ticket t = chunk t % kK2Span of big pair t / kK2Span
+  int32_t chunks_done[2];          // per pair slot (pair % 2): tickets of its current pair finished
+  int32_t slot_done[2];            // per pair slot: pairs finished in it
+  int32_t pad[3];
+  long long prog[2][kK2Span];      // per pair slot and chunk: (pair + 1) << 32 | tiles published
+  K2Pair pairs[8];                 // ring of published pairs (pair % 8)
+};
 struct K2Args {   // int32 re-run of saturated pairs (block per pair)
   const uint8_t *qcodes; const int64_t *qoff;
   const uint4 *packed; const GroupInfo *groups; const int32_t *sorted_len; const int32_t *perm;
@@ -133,8 +146,9 @@ struct K2Args {   // int32 re-run of saturated pairs (block per pair)
   int32_t *scores; int64_t ndb;
   int32_t alpha, beta;
   int32_t one;                              // = 1 (opaque to the compiler, see k2_kernel)
-  int32_t *border; int64_t border_stride;   // per-block border row (2 x int32 per column)
-  long long *k2prog;                        // per-block progress counters (big pairs), zeroed
+  int32_t *border; int64_t border_stride;   // border rows (2 x int32 per column): one per block,
+                                            // then 2 x kK2Span for the big pairs' pair slots
+  struct K2Ctl *ctl;                        // big pairs' tickets and slots, zeroed per launch
 };
 
 struct TbPair {     // one pair of a traceback batch

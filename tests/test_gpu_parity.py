@@ -603,12 +603,13 @@ print("ok")
 
 
 @pytest.mark.parametrize("big", ["1", "2000000"])
-def test_k2_cluster_split(big):
-    """K2 splits a big saturated pair over a cluster of 8 CTAs (chunk r on CTA r, borders
-    through L2 with epoch-tagged progress counters).  SW_K2_BIG lowers the size at which a
-    pair counts as big: "1" sends every re-run pair (down to a 4-aa query, fewer chunks
-    than CTAs) through the cluster path, "2000000" mixes both paths in one launch.  Every
-    overflow / int32-routing case stays bit-exact against the oracle."""
+def test_k2_split(big):
+    """K2 splits a big saturated pair into chunks run by several blocks at once (chunk tickets
+    taken in order, borders through L2 with pair-tagged progress counters, two pair slots).
+    SW_K2_BIG lowers the size at which a pair counts as big: "1" sends every re-run pair
+    (down to a 4-aa query, one chunk) through the split path -- many pairs, slot reuse --
+    "2000000" mixes both paths in one launch.  Queries of 33 to 40,000 aa cover 4, 8 and
+    16 rows per thread.  Every overflow / int32-routing case stays bit-exact."""
     import os
     import subprocess
     import sys
