@@ -118,11 +118,14 @@ typedef struct {
   int32_t straggler_after_ms;/* the straggler slows down only after this many ms (local
                                 load introduced mid-run, P24 §V.C); 0 = from the start */
   int32_t straggler_mode;    /* SW_STRAGGLER_* (default SW_STRAGGLER_SM_CAP) */
-  int32_t worker_sms;        /* experiments: > 0 caps EVERY worker's DP kernels to this many SMs'
-                                worth of resident blocks (split over its streams), so several
-                                workers sharing one GPU behave like separate smaller GPUs; a
-                                straggler (SW_STRAGGLER_SM_CAP) then gets ceil(worker_sms / s).
-                                0 = no partition (default) */
+  int32_t worker_sms;        /* experiments: > 0 makes several workers sharing one GPU behave like
+                                separate smaller GPUs.  Each worker gets a green-context SM
+                                partition of worker_sms rounded down to a multiple of 8 (its
+                                kernels run on those SMs only) when the device splits into
+                                enough of them; otherwise its DP kernels are capped to worker_sms
+                                SMs' worth of resident blocks (split over its streams).  A
+                                straggler (SW_STRAGGLER_SM_CAP) then gets ceil(SMs / s).  See
+                                sw_stats.partition_mode.  0 = no partition (default) */
   int32_t reserved[5];
 } sw_opts;
 
@@ -163,6 +166,10 @@ typedef struct {
                                launch being enqueued on its stream to its end (includes the
                                wait for free SMs behind the DP kernels) */
   int32_t n_k2_launches;    /* int32 re-run launches */
+  int32_t partition_mode;   /* emulated GPUs (sw_opts.worker_sms > 0): 2 = each worker on its own
+                               green-context SM partition, 1 = CTA caps (its blocks share SMs
+                               with other workers'), 0 = off */
+  int32_t partition_sms;    /* SMs per emulated GPU (mode 2: the partition's, a multiple of 8) */
 } sw_stats;
 
 typedef struct sw_db sw_db; /* opaque: host index + packed replica on each device */

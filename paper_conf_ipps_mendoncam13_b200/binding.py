@@ -70,7 +70,8 @@ class sw_stats(ctypes.Structure):
                 ("unit_log_json", ctypes.c_char_p), ("n_grant_messages", ctypes.c_int32),
                 ("n_cancelled", ctypes.c_int32), ("seconds_last_unit", ctypes.c_double),
                 ("peer_bytes", ctypes.c_int64), ("sched_log_json", ctypes.c_char_p),
-                ("kernel_seconds_k2", ctypes.c_double), ("n_k2_launches", ctypes.c_int32)]
+                ("kernel_seconds_k2", ctypes.c_double), ("n_k2_launches", ctypes.c_int32),
+                ("partition_mode", ctypes.c_int32), ("partition_sms", ctypes.c_int32)]
 
 
 # every symbol include/*.h declares (tests check the library exports all of them)

@@ -22,6 +22,7 @@
 #include <string>
 #include <thread>
 #include <vector>
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include "sw_internal.h"
 #include "net.h"
@@ -172,9 +173,63 @@ struct DevSearch {
   ~DevSearch();
 };
 
+// ---------------------------------------------------------------- green contexts
+// Emulated GPUs (sw_opts.worker_sms, experiments): the workers sharing one B200 each get a
+// disjoint SM partition through a green context (driver API, reached through the runtime's
+// entry-point table: no link-time libcuda), and their streams are created in it, so a
+// worker's kernels run on its SMs only.  Partitions are multiples of 8 SMs on sm_100.
+struct GreenApi {
+  CUresult (*get_res)(CUdevice, CUdevResource *, CUdevResourceType) = nullptr;
+  CUresult (*split)(CUdevResource *, unsigned *, const CUdevResource *, CUdevResource *, unsigned, unsigned) = nullptr;
+  CUresult (*gen_desc)(CUdevResourceDesc *, CUdevResource *, unsigned) = nullptr;
+  CUresult (*create)(CUgreenCtx *, CUdevResourceDesc, CUdevice, unsigned) = nullptr;
+  CUresult (*destroy)(CUgreenCtx) = nullptr;
+  CUresult (*stream)(CUstream *, CUgreenCtx, unsigned, int) = nullptr;
+  bool ok = false;
+};
+static const GreenApi &green_api() {
+  static GreenApi g;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    auto get = [](const char *name, auto &fn) {
+      void *p = nullptr;
+      cudaDriverEntryPointQueryResult q;
+      if (cudaGetDriverEntryPoint(name, &p, cudaEnableDefault, &q) == cudaSuccess && q == cudaDriverEntryPointSuccess)
+        fn = reinterpret_cast<std::remove_reference_t<decltype(fn)>>(p);
+      return fn != nullptr;
+    };
+    g.ok = get("cuDeviceGetDevResource", g.get_res) && get("cuDevSmResourceSplitByCount", g.split) &&
+           get("cuDevResourceGenerateDesc", g.gen_desc) && get("cuGreenCtxCreate", g.create) &&
+           get("cuGreenCtxDestroy", g.destroy) && get("cuGreenCtxStreamCreate", g.stream);
+  });
+  return g;
+}
+struct GreenSet {   // one device split into n partitions of sms SMs
+  int dev = -1, sms = 0, n = 0;
+  std::vector<CUgreenCtx> ctx;
+  ~GreenSet() {
+    for (CUgreenCtx c : ctx)
+      if (c) green_api().destroy(c);
+  }
+};
+// a stream in green context g (nullptr: the device's primary context)
+static cudaStream_t make_stream(CUgreenCtx g, int prio) {
+  cudaStream_t st;
+  if (g) {
+    CUstream cs;
+    if (green_api().stream(&cs, g, CU_STREAM_NON_BLOCKING, prio) != CUDA_SUCCESS)
+      throw Error(SW_ECUDA, "cuGreenCtxStreamCreate failed");
+    return (cudaStream_t)cs;
+  }
+  CK(cudaStreamCreateWithPriority(&st, cudaStreamNonBlocking, prio));
+  return st;
+}
+
 struct Device {
   int id = 0;
   int n_sm = 0;
+  int n_eff = 0;                // SMs its kernels are sized for: n_sm, or its green partition's
+  CUgreenCtx gctx = nullptr;    // the green context its streams belong to (emulated GPUs)
   DBuf<uint4> packed;
   DBuf<GroupInfo> groups;
   DBuf<int32_t> perm, sorted_len;
@@ -210,6 +265,7 @@ inline DevSearch::~DevSearch() {
 
 struct sw_db {
   sw::PackedDB host;
+  std::vector<std::unique_ptr<sw::GreenSet>> green;   // emulated GPUs (destroyed after devs)
   std::vector<std::unique_ptr<sw::Device>> devs;
   std::vector<char> peer_ok;     // [i * n + j]: device of worker i can read worker j's memory
   std::atomic<int> busy{0};
@@ -691,7 +747,7 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     a.gclaim = S.gclaim.p + uidx;
     a.na = na; a.nb = nbm;
     launch_k1(a, U.b1 - U.b0, db.groups[U.b1 - 1].ncols, P.pairs[U.pair].rows_padded, st,
-              sm_cap > 0 ? std::min(sm_cap, D.n_sm) : D.n_sm);
+              sm_cap > 0 ? std::min(sm_cap, D.n_eff) : D.n_eff);
   } else {
     K3Args a;
     a.packed = D.packed.p; a.groups = D.groups.p; a.perm = D.perm.p; a.sorted_len = D.sorted_len.p;
@@ -710,7 +766,7 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     // tiles between a clustered chunk's progress publications (SW_K3_PUB: tuning)
     static const int pub = [] { const char *e = getenv("SW_K3_PUB"); return e && atoi(e) > 0 ? atoi(e) : 8; }();
     a.pub_every = pub;
-    const int slots = D.n_sm * k3_blocks_per_sm();
+    const int slots = D.n_eff * k3_blocks_per_sm();
     if (U.cluster > 1) {   // counters + the launch's claim counter, zeroed on its stream
       a.kprog = S.k3_prog.p + (size_t)stream_idx * (slots * kK3Warps + 1);
       a.claim = a.kprog + slots * kK3Warps;
@@ -724,7 +780,7 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     // GPU (a later launch's queued clusters take the SMs an earlier unit frees: C5 at 1/4 of
     // its database 5.02 -> 5.37 TCUPS over per-pack units with equal shares); a clustered
     // per-pack unit beside K1 units (C4 at 1/8) -> its stream's share of the resident CTAs
-    const int maxb = sm_cap > 0 ? std::min(D.n_sm, sm_cap) * k3_blocks_per_sm()
+    const int maxb = sm_cap > 0 ? std::min(D.n_eff, sm_cap) * k3_blocks_per_sm()
                    : U.cluster > 1 ? (U.npk > 1 ? slots : std::max(U.cluster, k3_share(slots, (int)D.streams.size())))
                                    : INT32_MAX;
     launch_k3(a, U.cluster, maxb, st);
@@ -793,6 +849,7 @@ int sw_db_create(const sw_seqset *dbs, const int *devices, int n_devices, sw_db 
       D->id = d;
       CK(cudaSetDevice(d));
       CK(cudaDeviceGetAttribute(&D->n_sm, cudaDevAttrMultiProcessorCount, d));
+      D->n_eff = D->n_sm;
       D->packed.alloc(d, std::max<size_t>(H.packed.size(), 1));
       D->groups.alloc(d, std::max<size_t>(H.groups.size(), 1));
       D->perm.alloc(d, std::max<size_t>(H.perm.size(), 1));
@@ -880,12 +937,110 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
     const PackedDB &H = db->host;
     const int32_t nq = queries->n, nd = H.n;
     const int nW = dist ? 1 : (int)db->devs.size();
+    // emulated GPUs (worker_sms > 0, in-process): every worker on a device gets a green SM
+    // partition of worker_sms SMs rounded down to a multiple of 8 when the device splits
+    // into enough of them, otherwise (or without green contexts) its DP grids are capped
+    // to worker_sms SMs' worth of blocks (CTA caps: blocks of several workers share SMs)
+    int32_t partition_mode = 0, partition_sms = 0;
+    if (!dist && !db->devs.empty()) {
+      std::vector<int> want_n;   // workers per device id
+      for (auto &d : db->devs) {
+        if ((int)want_n.size() <= d->id) want_n.resize(d->id + 1, 0);
+        want_n[d->id]++;
+      }
+      const int sms8 = o.worker_sms / 8 * 8;
+      bool green_ok = o.worker_sms > 0 && sms8 >= 8 && green_api().ok;
+      auto reset_streams = [&](int dev_id) {   // the streams of every worker on dev_id
+        for (auto &d : db->devs) {
+          if (d->id != dev_id) continue;
+          CK(cudaSetDevice(d->id));
+          CK(cudaDeviceSynchronize());
+          for (auto st : d->streams) cudaStreamDestroy(st);
+          d->streams.clear();
+          if (d->ws) {
+            DevSearch &X = *d->ws;
+            for (auto e : X.epi) cudaStreamDestroy(e);
+            X.epi.clear();
+            if (X.cancel_st) cudaStreamDestroy(X.cancel_st);
+            if (X.noise_st) cudaStreamDestroy(X.noise_st);
+            X.cancel_st = X.noise_st = nullptr;
+          }
+          d->gctx = nullptr;
+        }
+      };
+      for (int dev = 0; green_ok && dev < (int)want_n.size(); dev++) {
+        if (want_n[dev] == 0) continue;
+        GreenSet *gs = nullptr;
+        for (auto &g : db->green)
+          if (g->dev == dev) gs = g.get();
+        if (gs && gs->sms == sms8 && gs->n >= want_n[dev]) continue;
+        reset_streams(dev);   // before the old contexts go
+        db->green.erase(std::remove_if(db->green.begin(), db->green.end(),
+                                       [&](const std::unique_ptr<GreenSet> &g) { return g->dev == dev; }),
+                        db->green.end());
+        const GreenApi &ga = green_api();
+        CK(cudaSetDevice(dev));
+        CK(cudaFree(nullptr));   // the primary context exists
+        CUdevResource all, rem;
+        unsigned n = 0;
+        if (ga.get_res(dev, &all, CU_DEV_RESOURCE_TYPE_SM) != CUDA_SUCCESS ||
+            ga.split(nullptr, &n, &all, nullptr, 0, sms8) != CUDA_SUCCESS || (int)n < want_n[dev]) {
+          green_ok = false;
+          break;
+        }
+        std::vector<CUdevResource> parts(n);
+        auto ng = std::make_unique<GreenSet>();
+        ng->dev = dev;
+        if (ga.split(parts.data(), &n, &all, &rem, 0, sms8) != CUDA_SUCCESS || (int)n < want_n[dev]) {
+          green_ok = false;
+          break;
+        }
+        ng->sms = (int)parts[0].sm.smCount;
+        for (int i = 0; i < want_n[dev]; i++) {
+          CUdevResourceDesc desc;
+          CUgreenCtx gc = nullptr;
+          if (ga.gen_desc(&desc, &parts[i], 1) != CUDA_SUCCESS ||
+              ga.create(&gc, desc, dev, CU_GREEN_CTX_DEFAULT_STREAM) != CUDA_SUCCESS) {
+            green_ok = false;
+            break;
+          }
+          ng->ctx.push_back(gc);
+        }
+        ng->n = (int)ng->ctx.size();
+        db->green.push_back(std::move(ng));
+      }
+      // each worker's context (in order on its device) and SM count; a device whose workers
+      // change context gets all its streams rebuilt (lazily, in the setup below)
+      std::vector<int> used(want_n.size(), 0);
+      std::vector<CUgreenCtx> want(db->devs.size(), nullptr);
+      std::vector<int> neff(db->devs.size(), 0);
+      for (size_t w = 0; w < db->devs.size(); w++) {
+        Device &d = *db->devs[w];
+        neff[w] = d.n_sm;
+        if (!green_ok) continue;
+        for (auto &g : db->green)
+          if (g->dev == d.id && used[d.id] < g->n) {
+            want[w] = g->ctx[used[d.id]++];
+            neff[w] = g->sms;
+          }
+      }
+      for (size_t w = 0; w < db->devs.size(); w++)
+        if (db->devs[w]->gctx != want[w]) reset_streams(db->devs[w]->id);
+      for (size_t w = 0; w < db->devs.size(); w++) {
+        db->devs[w]->gctx = want[w];
+        db->devs[w]->n_eff = neff[w];
+      }
+      if (o.worker_sms > 0) {
+        partition_mode = green_ok ? 2 : 1;
+        partition_sms = green_ok ? db->devs[0]->n_eff : o.worker_sms;
+      }
+    }
     // one wave of K1 blocks on the (first) GPU: SMs x resident K1 blocks per SM
     int32_t k1_wave = 0, k3_slots = 0;
     if (!db->devs.empty()) {
       CK(cudaSetDevice(db->devs[0]->id));
-      k1_wave = db->devs[0]->n_sm * k1_blocks_per_sm();
-      k3_slots = db->devs[0]->n_sm * k3_blocks_per_sm();
+      k1_wave = db->devs[0]->n_eff * k1_blocks_per_sm();
+      k3_slots = db->devs[0]->n_eff * k3_blocks_per_sm();
     }
     Plan P = make_plan(queries, H, o, dist ? o.dist_world : nW, M, thresh, k1_wave, k3_slots);
     bool any_cluster = false;
@@ -909,11 +1064,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       X.D = &D;
       X.reset_counters();
       const int depth = o.streams_per_device;
-      while ((int)D.streams.size() < depth) {
-        cudaStream_t st;
-        CK(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
-        D.streams.push_back(st);
-      }
+      while ((int)D.streams.size() < depth) D.streams.push_back(make_stream(D.gctx, 0));
       if (D.slots_per_sm == 0) {
         D.slots_per_sm = k1_blocks_per_sm();
         D.sm_slots = 256;  // %smid < 256
@@ -979,19 +1130,15 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         CK(cudaHostGetDevicePointer((void **)&X.ovf_early_d, X.ovf_early_h, 0));
       }
       for (int k = 0; k < kMaxStreams; k++) ((volatile int32_t *)X.ovf_early_h)[k] = 0;
-      if (!X.cancel_st) CK(cudaStreamCreateWithFlags(&X.cancel_st, cudaStreamNonBlocking));
+      if (!X.cancel_st) X.cancel_st = make_stream(D.gctx, 0);
       {
         int lo = 0, hi = 0;
         CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
         // (the local-load stream is created only when a worker emulates one: every stream
         // takes one of the GPU's hardware work queues)
         if (!X.noise_st && o.straggler_mode == SW_STRAGGLER_NOISE && o.straggler_mask)
-          CK(cudaStreamCreateWithPriority(&X.noise_st, cudaStreamNonBlocking, hi));
-        while (X.epi.empty()) {   // one per worker (the hardware work queues are limited)
-          cudaStream_t e;
-          CK(cudaStreamCreateWithPriority(&e, cudaStreamNonBlocking, hi));
-          X.epi.push_back(e);
-        }
+          X.noise_st = make_stream(D.gctx, hi);
+        while (X.epi.empty()) X.epi.push_back(make_stream(D.gctx, hi));   // one per worker
       }
       if (!X.ev_start) CK(cudaEventCreate(&X.ev_start));
       if (!X.ev_end) CK(cudaEventCreate(&X.ev_end));
@@ -1105,12 +1252,13 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         const bool straggler = (o.straggler_mask >> wid) & 1ull;
         const int slow = std::max(1, o.straggler_slowdown);
         // the worker's SM budget: the whole GPU, or its partition (worker_sms, experiments)
-        const int budget = o.worker_sms > 0 ? std::min(o.worker_sms, D.n_sm) : D.n_sm;
+        const int budget = D.gctx ? D.n_eff : o.worker_sms > 0 ? std::min(o.worker_sms, D.n_sm) : D.n_sm;
         const int sm_cap = (budget + slow - 1) / slow;     // ceil(budget / slowdown)
         // a budget is split over the worker's streams (up to `depth` units run at once), so
         // the whole worker holds ~budget SMs' worth of blocks
         const int sm_share = std::max(1, (sm_cap + depth - 1) / depth);
-        const int part_share = o.worker_sms > 0 ? std::max(1, (budget + depth - 1) / depth) : 0;
+        // (a green partition needs no cap: its kernels cannot leave its SMs)
+        const int part_share = (o.worker_sms > 0 && !D.gctx) ? std::max(1, (budget + depth - 1) / depth) : 0;
         const double t_after = 1e-3 * std::max(0, o.straggler_after_ms);
         std::deque<int32_t> pending;
         std::vector<int32_t> inflight(depth, -1);
@@ -1147,9 +1295,9 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
           if (slow_now && o.straggler_mode == SW_STRAGGLER_NOISE && !noise_on) {
             // local load: SM-filling blocks on all but ceil(n_sm / slowdown) SMs
             X.noise_flag.ensure(D.id, 1);
-            X.noise_sink.ensure(D.id, D.n_sm);
+            X.noise_sink.ensure(D.id, D.n_eff);
             CK(cudaMemsetAsync(X.noise_flag.p, 0, sizeof(int32_t), X.noise_st));
-            launch_noise(X.noise_flag.p, D.n_sm - sm_cap, 60ull * 1000000000ull, X.noise_sink.p, X.noise_st);
+            launch_noise(X.noise_flag.p, D.n_eff - sm_cap, 60ull * 1000000000ull, X.noise_sink.p, X.noise_st);
             CK(cudaGetLastError());
             noise_on = true;
           }
@@ -1534,6 +1682,8 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         stats->kernel_seconds_k3 += S[w]->k3_sec;
         stats->kernel_seconds_k2 += S[w]->k2_sec;
         stats->n_k2_launches += (int32_t)S[w]->k2_ev.size();
+        stats->partition_mode = partition_mode;
+        stats->partition_sms = partition_sms;
         stats->cells_k1 += S[w]->k1_cells;
         stats->cells_k3 += S[w]->k3_cells;
         stats->n_cancelled += S[w]->n_cancelled;

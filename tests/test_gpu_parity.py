@@ -618,3 +618,25 @@ def test_k2_split(big):
     out = subprocess.run([sys.executable, "-c", _K2_SCRIPT % root], env=env, capture_output=True,
                          text=True, timeout=900, cwd=root)
     assert out.returncode == 0 and "ok" in out.stdout, (out.stdout[-2000:], out.stderr[-3000:])
+
+
+def test_green_partitions_emulated_gpus():
+    """Emulated GPUs (worker_sms): four workers on one B200, each on its own green-context SM
+    partition (32 SMs: 37 rounded down to a multiple of 8); then back to the whole GPU, and
+    to 16-SM partitions with a GPU-side straggler and WA.  C2 stays bit-exact (digest) in
+    every layout; the stats report the partition."""
+    w = seqgen.make_workload("C2")
+    D = Database(w.db, devices=[0, 0, 0, 0])
+    try:
+        r = D.search(w.queries, top_k=10, worker_sms=37, streams=2)
+        assert r.stats["partition_mode"] == 2 and r.stats["partition_sms"] == 32
+        assert _digest("C2", r.scores)[0]
+        r = D.search(w.queries, top_k=10, streams=2)
+        assert r.stats["partition_mode"] == 0
+        assert _digest("C2", r.scores)[0]
+        r = D.search(w.queries, top_k=10, worker_sms=18, streams=2, straggler_mask=0b1000, straggler_slowdown=4,
+                     target_unit_cells=2**62)
+        assert r.stats["partition_mode"] == 2 and r.stats["partition_sms"] == 16
+        assert _digest("C2", r.scores)[0]
+    finally:
+        D.close()

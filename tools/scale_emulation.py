@@ -1,6 +1,7 @@
 """Strong-scaling emulation on one B200 (no multi-GPU node available): N workers share the
-GPU, each capped to the same SM budget (sw_opts.worker_sms = n_SM // 8 by default), i.e. N
-emulated GPUs of 18 SMs.  For N = 1, 2, 4, 8 it reports device-timed GCUPS of the whole
+GPU, each on its own green-context SM partition (sw_opts.worker_sms = n_SM // 8 by default,
+rounded down to a multiple of 8: 16 SMs), i.e. N emulated GPUs of 16 SMs whose kernels cannot
+leave their SMs (they share the L2 and HBM).  For N = 1, 2, 4, 8 it reports device-timed GCUPS of the whole
 search (PSS + WA, the in-process data plane: committed segments and hit lists copied to the
 first worker and merged), the efficiency GCUPS(N) / (N x GCUPS(1)), units per worker,
 request messages and the bytes the merge moved.  Scores are checked against the oracle's digest.
@@ -51,7 +52,7 @@ for n in [int(x) for x in args.ns.split(",")]:
     row = dict(n=n, sms_per_worker=sms, gcups=st["gcups"], seconds=st["seconds_device"], units=st["n_units"],
                committed_per_worker=per, tail_s=st["tail_seconds"], wa_grants=st["n_wa_grants"],
                cancelled=st["n_cancelled"], request_messages=st["n_requests"], peer_bytes=st["peer_bytes"],
-               digest_ok=ok)
+               digest_ok=ok, partition_mode=st["partition_mode"], partition_sms=st["partition_sms"])
     rows.append(row)
     print(json.dumps(row), flush=True)
     D.close()
@@ -63,5 +64,6 @@ for row in rows:
           f"merge moved {row['peer_bytes'] / 1e6:.1f} MB, digest {row['digest_ok']}", flush=True)
 if args.out:
     json.dump(dict(config=args.config, sms_per_worker=sms, streams=args.streams, n_sm=n_sm,
-                   note="N workers on one B200, each capped to sms_per_worker SMs (worker_sms): N emulated GPUs",
+                   note="N workers on one B200, each on its own green-context partition of partition_sms SMs "
+                        "(partition_mode 2; 1 = CTA caps): N emulated GPUs",
                    rows=rows), open(args.out, "w"), indent=1)

@@ -48,7 +48,8 @@ def main():
     ap.add_argument("--scenarios", default="homogeneous,straggler,local_load_midrun")
     ap.add_argument("--out", default=None)
     ap.add_argument("--partition", action="store_true",
-                    help="each worker gets n_SM / workers SMs (worker_sms): the workers behave like separate GPUs")
+                    help="each worker gets n_SM / workers SMs (worker_sms): its own green-context SM partition "
+                         "(a multiple of 8 SMs), so the workers behave like separate GPUs")
     ap.add_argument("--unit-cells", type=int, default=0,
                     help="target_unit_cells (0 = auto; 2**62 = the paper's very coarse tasks, one per pack)")
     args = ap.parse_args()
@@ -93,6 +94,7 @@ def main():
                     d["last_dev_ms"] = max(d["last_dev_ms"], e["dev_t1"])
                 grants = grant_timeline(best["sched_log"])
                 row = dict(scenario=name, policy=policy, wa=wa, makespan_s=best["seconds_device"],
+                           partition_mode=best["partition_mode"], partition_sms=best["partition_sms"],
                            last_unit_s=best["seconds_last_unit"], tail_s=best["tail_seconds"],
                            gcups=best["gcups"], duplicated_cells=best["duplicated_cells"],
                            wa_grants=best["n_wa_grants"], cancelled=best["n_cancelled"],
@@ -124,7 +126,9 @@ def main():
     out = dict(config=args.config, workers=args.workers, streams=args.streams, slowdown=args.slowdown,
                mode=args.mode, unit_cells=args.unit_cells, oracle_digest_checked=bool(gold), worker_sms=wsms,
                note="P workers share one B200 (separate streams/replicas); the straggler is the last worker"
-                    + (f"; each worker is capped to {wsms} SMs (worker_sms), i.e. P emulated GPUs" if wsms else ""),
+                    + (f"; worker_sms={wsms}: each worker on its own green-context partition of "
+                       f"{base.stats['partition_sms']} SMs (partition_mode {base.stats['partition_mode']}: 2 = green "
+                       f"contexts, 1 = CTA caps), i.e. P emulated GPUs" if wsms else ""),
                summary=summary, runs=rows)
     if args.out:
         with open(args.out, "w") as f:
