@@ -15,6 +15,7 @@ pinned host memory) timed by the host clock around the call.
 from __future__ import annotations
 
 import argparse
+import hashlib
 import json
 import os
 import statistics
@@ -182,6 +183,10 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--ref-seconds", type=float, default=12.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--emulated-scaling", default="1,2,4,8",
+                    help="N=1 runs only: N emulated GPUs on disjoint green-context SM partitions of "
+                         "n_SM // 8 SMs (rounded to 8) for each listed N, one device-timed search each; "
+                         "'' = skip")
     ap.add_argument("--policy", default="pss")
     ap.add_argument("--no-wa", action="store_true")
     ap.add_argument("--straggler-mask", type=int, default=0)
@@ -368,6 +373,33 @@ def main():
             cpu = {"value": g, "unit": "GCUPS", "cores": cores, "kind": "oracle", "sample": desc,
                    "single_core": {"value": g1, "sample": desc1}, "cpu_model": cpu_model()}
 
+    # ---- emulated multi-GPU strong scaling (no multi-GPU node in this pool): N workers on
+    # one B200, each on its own green-context SM partition (sw_opts.worker_sms), the same
+    # workload; one device-timed search per N (libsw's CUDA events), scores of every N equal
+    emulated = None
+    if world == 1 and args.emulated_scaling:
+        nsm_all = torch.cuda.get_device_properties(local).multi_processor_count
+        sms = nsm_all // 8
+        rows, ref_digest = [], None
+        for n in [int(x) for x in args.emulated_scaling.split(",") if x]:
+            De = Database(w.db, devices=[local] * n)
+            flush_l2()
+            r = De.search(w.queries, top_k=args.top_k, worker_sms=sms, **kw)
+            dg = hashlib.sha256(np.ascontiguousarray(r.scores, dtype="<i4").tobytes()).hexdigest()
+            ref_digest = ref_digest or dg
+            rows.append({"n": n, "gcups": r.stats["gcups"], "seconds": r.stats["seconds_device"],
+                         "partition_mode": r.stats["partition_mode"], "partition_sms": r.stats["partition_sms"],
+                         "tail_s": r.stats["tail_seconds"], "peer_bytes": r.stats["peer_bytes"],
+                         "scores_equal_n1": dg == ref_digest})
+            De.close()
+        g1 = next((x["gcups"] for x in rows if x["n"] == 1), None)
+        for x in rows:
+            x["efficiency"] = x["gcups"] / (x["n"] * g1) if g1 else None
+        emulated = {"rows": rows, "kind": "strong scaling, N emulated GPUs on one B200",
+                    "note": "each worker on a disjoint green-context SM partition (partition_mode 2; its kernels "
+                            "cannot leave its partition_sms SMs; L2/HBM shared); PSS + WA, in-process data "
+                            "plane; efficiency = GCUPS(N) / (N x GCUPS(1))"}
+
     if rank == 0:
         line = {"metric": "GCUPS", "value": value, "unit": "GCUPS", "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
@@ -392,7 +424,7 @@ def main():
                            "db_create_s": db_create_s, "generate_s": gen_s,
                            "wall_s_timed": wall, "parallelism": f"dp{world} (PSS/WA units)"},
                 "gpu_launches": launches, "clocks": clocks, "e2e": e2e, "roofline": roofline,
-                "cpu_baseline": cpu, "context": PAPER_CONTEXT}
+                "cpu_baseline": cpu, "emulated_scaling": emulated, "context": PAPER_CONTEXT}
         print(json.dumps(line), flush=True)
     if world > 1:
         tdist.barrier()
