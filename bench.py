@@ -171,6 +171,36 @@ def load_traffic():
         return None, None
 
 
+def emulated_scaling(args, w, kw, local, flush_l2):
+    """N emulated GPUs on one B200 (no multi-GPU node in this pool): N workers, each on its own
+    green-context SM partition (sw_opts.worker_sms), the same workload; one device-timed search
+    per N (libsw's CUDA events); the scores of every N must equal N = 1's."""
+    import torch
+    from paper_conf_ipps_mendoncam13_b200 import Database
+    nsm_all = torch.cuda.get_device_properties(local).multi_processor_count
+    sms = nsm_all // 8
+    rows, ref_digest = [], None
+    for n in [int(x) for x in args.emulated_scaling.split(",") if x]:
+        De = Database(w.db, devices=[local] * n)
+        flush_l2()
+        r = De.search(w.queries, top_k=args.top_k, worker_sms=sms, **kw)
+        dg = hashlib.sha256(np.ascontiguousarray(r.scores, dtype="<i4").tobytes()).hexdigest()
+        ref_digest = ref_digest or dg
+        rows.append({"n": n, "gcups": r.stats["gcups"], "seconds": r.stats["seconds_device"],
+                     "partition_mode": r.stats["partition_mode"], "partition_sms": r.stats["partition_sms"],
+                     "tail_s": r.stats["tail_seconds"], "peer_bytes": r.stats["peer_bytes"],
+                     "scores_equal_n1": dg == ref_digest})
+        De.close()
+    g1 = next((x["gcups"] for x in rows if x["n"] == 1), None)
+    for x in rows:
+        x["efficiency"] = x["gcups"] / (x["n"] * g1) if g1 else None
+    emulated = {"rows": rows, "kind": "strong scaling, N emulated GPUs on one B200",
+                "note": "each worker on a disjoint green-context SM partition (partition_mode 2; its kernels "
+                        "cannot leave its partition_sms SMs; L2/HBM shared); PSS + WA, in-process data "
+                        "plane; efficiency = GCUPS(N) / (N x GCUPS(1))"}
+    return emulated
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -378,27 +408,10 @@ def main():
     # workload; one device-timed search per N (libsw's CUDA events), scores of every N equal
     emulated = None
     if world == 1 and args.emulated_scaling:
-        nsm_all = torch.cuda.get_device_properties(local).multi_processor_count
-        sms = nsm_all // 8
-        rows, ref_digest = [], None
-        for n in [int(x) for x in args.emulated_scaling.split(",") if x]:
-            De = Database(w.db, devices=[local] * n)
-            flush_l2()
-            r = De.search(w.queries, top_k=args.top_k, worker_sms=sms, **kw)
-            dg = hashlib.sha256(np.ascontiguousarray(r.scores, dtype="<i4").tobytes()).hexdigest()
-            ref_digest = ref_digest or dg
-            rows.append({"n": n, "gcups": r.stats["gcups"], "seconds": r.stats["seconds_device"],
-                         "partition_mode": r.stats["partition_mode"], "partition_sms": r.stats["partition_sms"],
-                         "tail_s": r.stats["tail_seconds"], "peer_bytes": r.stats["peer_bytes"],
-                         "scores_equal_n1": dg == ref_digest})
-            De.close()
-        g1 = next((x["gcups"] for x in rows if x["n"] == 1), None)
-        for x in rows:
-            x["efficiency"] = x["gcups"] / (x["n"] * g1) if g1 else None
-        emulated = {"rows": rows, "kind": "strong scaling, N emulated GPUs on one B200",
-                    "note": "each worker on a disjoint green-context SM partition (partition_mode 2; its kernels "
-                            "cannot leave its partition_sms SMs; L2/HBM shared); PSS + WA, in-process data "
-                            "plane; efficiency = GCUPS(N) / (N x GCUPS(1))"}
+        try:
+            emulated = emulated_scaling(args, w, kw, local, flush_l2)
+        except Exception as e:   # an experiment: never lose the bench line for it
+            emulated = {"error": f"{type(e).__name__}: {e}"}
 
     if rank == 0:
         line = {"metric": "GCUPS", "value": value, "unit": "GCUPS", "n_gpus": world,
