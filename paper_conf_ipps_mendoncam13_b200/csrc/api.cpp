@@ -21,6 +21,7 @@
 #include <stdexcept>
 #include <string>
 #include <thread>
+#include <type_traits>
 #include <vector>
 #include <cuda.h>
 #include <cuda_runtime.h>
@@ -204,8 +205,8 @@ static const GreenApi &green_api() {
   });
   return g;
 }
-struct GreenSet {   // one device split into n partitions of sms SMs
-  int dev = -1, sms = 0, n = 0;
+struct GreenSet {   // one device split into n partitions of sms SMs (asked for: req)
+  int dev = -1, req = 0, sms = 0, n = 0;
   std::vector<CUgreenCtx> ctx;
   ~GreenSet() {
     for (CUgreenCtx c : ctx)
@@ -973,7 +974,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         GreenSet *gs = nullptr;
         for (auto &g : db->green)
           if (g->dev == dev) gs = g.get();
-        if (gs && gs->sms == sms8 && gs->n >= want_n[dev]) continue;
+        if (gs && gs->req == sms8 && gs->n >= want_n[dev]) continue;
         reset_streams(dev);   // before the old contexts go
         db->green.erase(std::remove_if(db->green.begin(), db->green.end(),
                                        [&](const std::unique_ptr<GreenSet> &g) { return g->dev == dev; }),
@@ -991,6 +992,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
         std::vector<CUdevResource> parts(n);
         auto ng = std::make_unique<GreenSet>();
         ng->dev = dev;
+        ng->req = sms8;
         if (ga.split(parts.data(), &n, &all, &rem, 0, sms8) != CUDA_SUCCESS || (int)n < want_n[dev]) {
           green_ok = false;
           break;
