@@ -37,6 +37,8 @@ PAPER_CONTEXT = ("paper: 7,190 s on 1 SSE core (Core i7 3.4 GHz) vs 112 s on 4x 
 DPX_RATE = 64.0   # measured lane-ops/clk/SM of VIMNMX3.S16x2 / VIADDMNMX.S16x2 (tools/dpx_peak)
 DPX_PER_CELL = 2.0  # K1/K3 inner loop: 4 three-input DPX per s16x2 lane word = 2 per cell
 DPX_FORMULATION = 2.25  # + the running maximum (0.5 VIMNMX3 per word): the kernel's own ALU ops/cell
+MICROBENCH_CELLS_PER_CLK = 24.5  # the same cell update in a register-only loop (tools/dp_variants.cu,
+                                 # profiles/r01_dp_variants.txt): no barriers, borders or profile staging
 
 
 def env_rank():
@@ -388,6 +390,10 @@ def main():
                     "peak_at_max_clock": peak_max,
                     "formulation_peak": peak_form,
                     "k1_frac_of_formulation": (k1_alone / peak_form) if k1_alone else None,
+                    "microbench_ceiling": nsm * sm_mhz * 1e6 * MICROBENCH_CELLS_PER_CLK / 1e9,
+                    "k1_frac_of_microbench": (k1_alone / (nsm * sm_mhz * 1e6 * MICROBENCH_CELLS_PER_CLK / 1e9))
+                                             if k1_alone else None,
+                    "step_frac_of_microbench": per_gpu / (nsm * sm_mhz * 1e6 * MICROBENCH_CELLS_PER_CLK / 1e9),
                     "step_frac_of_formulation": per_gpu / peak_form,
                     "derivation": f"{nsm} SMs x {sm_mhz:.0f} MHz (median under load) x {DPX_RATE:.0f} "
                                   f"DPX lane-ops/clk/SM (measured, tools/dpx_peak.cu) / "
