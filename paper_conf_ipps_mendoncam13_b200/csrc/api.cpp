@@ -548,6 +548,7 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
         if (forced > 0) per_unit = forced * k1_wave;
         else if (2 * gpu >= k1_wave) per_unit = (gpu + k1_wave - 1) / k1_wave * k1_wave;
       }
+      static const double crit = [] { const char *e = getenv("SW_K1_CRIT"); return e ? atof(e) : 1.5; }();
       while (g < seg_end) {
         int32_t e = g;
         int64_t cells = 0, work = 0;
@@ -555,6 +556,18 @@ static Plan make_plan(const sw_seqset *q, const PackedDB &db, const sw_opts &o, 
           cells += rows_eff * grp_res[e];
           work += rows_k1 * db.groups[e].ncols * kGroup;
           e++;
+        }
+        // a block runs a whole group: a unit whose per-block share (work / wave) is not well
+        // above its widest group's work ends on that group's block alone (the widest C4 unit
+        // of a pack: groups of 872-3,048 columns, 2 waves -> 5.2 TCUPS alone vs 6.3 typical);
+        // such a unit takes more whole waves until the share is >= crit x the widest group
+        // (SW_K1_CRIT, tuning: 0 / 1.5 / 2.5 -> K1 alone 6,102 / 6,177 / 6,002 GCUPS on C4)
+        const int64_t w_first = rows_k1 * (int64_t)db.groups[g].ncols * kGroup;
+        while (per_unit > 0 && crit > 0 && e < seg_end && (double)work / k1_wave < crit * (double)w_first) {
+          for (int32_t k = 0; k < k1_wave && e < seg_end; k++, e++) {
+            cells += rows_eff * grp_res[e];
+            work += rows_k1 * db.groups[e].ncols * kGroup;
+          }
         }
         P.units.push_back({kUnitInter, p, g, e, cells, work, 1, 1});
         g = e;
