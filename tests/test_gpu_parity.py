@@ -93,6 +93,7 @@ def test_overflow_rerun_int32():
         r = _search(db, qs, top_k=3, long_threshold=thr)
         assert (r.scores == ref).all()
         assert r.stats["n_overflow_pairs"] >= 1
+        assert r.stats["n_k2_launches"] >= 1 and r.stats["kernel_seconds_k2"] > 0
 
 
 def test_big_matrix_forces_many_overflows():
