@@ -139,8 +139,10 @@ __device__ __forceinline__ void flush_half(int q, int v, int ss, int orig, int32
       const int k = atomicAdd(ovf_count, 1);
       if (k < ovf_cap) {
         ovf[k] = make_int2(q, ss);
-        if (ovf_early) {   // a hint: two writers may land out of order (the worker also reads
-                           // the device count after every unit), so a plain store, no host atomics
+        // a hint: two writers may land out of order (the worker also reads the device count
+        // after every unit), so a plain store, no host atomics; only at counts 1, 2, 4, 8, ...
+        // (a search routed to int32 lists every pair: no system fence per pair)
+        if (ovf_early && ((k + 1) & k) == 0) {
           __threadfence_system();   // the entry before the host sees its count
           *(volatile int32_t *)ovf_early = k + 1;
         }
