@@ -92,10 +92,11 @@ def lib():
     global _lib
     if _lib is not None:
         return _lib
-    path = _build.LIB
+    checked = os.environ.get("SW_CHECKED") == "1"   # the bounds-asserting build (tests)
+    path = _build.LIB_CHECKED if checked else _build.LIB
     try:
-        if _build._stale():
-            _build.build()
+        if _build._stale(checked):
+            _build.build(checked=checked)
     except Exception as e:  # nvcc missing etc.: only fatal if there is no library at all
         if not os.path.exists(path):
             raise ImportError(f"libsw.so is missing and could not be built: {e}") from e

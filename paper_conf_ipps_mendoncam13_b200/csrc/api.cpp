@@ -775,6 +775,7 @@ static void launch_unit(const Plan &P, const PackedDB &db, DevSearch &S, const U
     const int64_t stride = (std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16;  // >= tiles * T
     a.border = S.k3_border.p + (size_t)stream_idx * S.k3_rows * stride;
     a.border_stride = stride;
+    a.border_rows = S.k3_rows;
     a.kprog = nullptr;
     a.claim = nullptr;
     // tiles between a clustered chunk's progress publications (SW_K3_PUB: tuning)

@@ -28,6 +28,23 @@
 #include "sw_internal.h"
 #include "../../include/sw.h"
 
+// Checked build (SW_CHECKED=1 at build / load time: libsw_checked.so): bounds of the border
+// rows, ring slots, profile codes and list entries are asserted in the kernels; a violation
+// prints where and traps.  compute-sanitizer is closed on this GPU pool, so the GPU tests run
+// the split paths on this build too (tests/test_gpu_parity.py::test_checked_build).
+#ifdef SW_CHECKED
+#define SW_CHECK(c)                                                                          \
+  do {                                                                                       \
+    if (!(c)) {                                                                              \
+      printf("SW_CHECK failed %s:%d: %s (block %d thread %d)\n", __FILE__, __LINE__, #c,      \
+             (int)blockIdx.x, (int)threadIdx.x);                                             \
+      __trap();                                                                              \
+    }                                                                                        \
+  } while (0)
+#else
+#define SW_CHECK(c) do { } while (0)
+#endif
+
 namespace sw {
 
 constexpr bool kK1PairLoads = true;   // K1 reads two profile rows per LDS.64
@@ -411,6 +428,7 @@ __global__ void __launch_bounds__(W * 32, MINB) k1_kernel(const K1Args a) {
         for (int j = 0; j < GS; j++) outp[(q * GS + j) * 32 + lane] = make_uint2(oh[j], fc[j]);
       }
       if (warp == W - 1 && band < nb - 1) {
+        SW_CHECK(tile * T + T <= a.border_slot_cols);
 #pragma unroll
         for (int jj = 0; jj < T; jj++) border[(size_t)(tile * T + jj) * 32 + lane] = outp[jj * 32 + lane];
       }
@@ -690,6 +708,7 @@ __global__ void __launch_bounds__(kK3Warps * 32, 4) k3_kernel(const K3Args a) {
                                       : a.border + (size_t)(gslot * C + bin) * a.border_stride;
       uint2 *border_out = C == 1 ? a.border + (size_t)(sb * kK3Warps + warp) * a.border_stride
                                  : a.border + (size_t)(gslot * C + bout) * a.border_stride;
+      SW_CHECK(C > 1 ? (int64_t)gslot * C + C <= a.border_rows : (int64_t)sb * kK3Warps + warp < a.border_rows);
       const int *prog_in = a.kprog + gslot * C + bin;
       int *prog_out = a.kprog + gslot * C + bout;
       // counters count tiles written into a buffer since the launch: earlier sequence blocks
@@ -729,6 +748,7 @@ __global__ void __launch_bounds__(kK3Warps * 32, 4) k3_kernel(const K3Args a) {
                   }
                 }
               }
+              SW_CHECK((int64_t)tt * T + T <= a.border_stride);
 #pragma unroll
               for (int jj = 0; jj < T; jj += 2) cp_async16_cg(&bring[sl * T + jj], &border_in[tt * T + jj]);
             } else {
@@ -797,6 +817,7 @@ __global__ void __launch_bounds__(kK3Warps * 32, 4) k3_kernel(const K3Args a) {
 #pragma unroll
           for (int q = 0; q < NW; q++) out_c[q] = in_c[q];
           if (lane == 31 && ch < nch - 1) {
+            SW_CHECK((int64_t)tile * T + T <= a.border_stride);
 #pragma unroll
             for (int jj = 0; jj < T; jj++) border_out[tile * T + jj] = make_uint2(out_h[jj], out_f[jj]);
             if (C > 1 && ((tile + 1) % a.pub_every == 0 || tile + 1 == ntile))
@@ -1055,6 +1076,7 @@ __device__ __forceinline__ int k2_chunk(const K2Args &a, const int8_t *Ms, int8_
       const unsigned d = (unsigned)__cvta_generic_to_shared(&cring[tt % kK2Ring]);
       asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(d), "l"(codes_at(tt)) : "memory");
       if (bin) {
+        SW_CHECK((int64_t)tt * K2C + K2C <= a.border_stride);
         wait_tile(tt);
         cp_async16_cg(&ring[(tt % kK2Ring) * K2C], bin + tt * K2C);
         cp_async16_cg(&ring[(tt % kK2Ring) * K2C + 2], bin + tt * K2C + 2);
@@ -1091,6 +1113,7 @@ __device__ __forceinline__ int k2_chunk(const K2Args &a, const int8_t *Ms, int8_
       int hd[K2C], f[K2C], oh[K2C];
 #pragma unroll
       for (int g = 0; g < K2C; g++) {
+        SW_CHECK(((cw >> (8 * g)) & 0xffu) < (uint32_t)kNCodes);
         sw[g] = pbase[((cw >> (8 * g)) & 0xffu) * kK2Threads];
         hd[g] = hprev_top;
         f[g] = in[g].y;
@@ -1119,6 +1142,7 @@ __device__ __forceinline__ int k2_chunk(const K2Args &a, const int8_t *Ms, int8_
       for (int g = 0; g < K2C; g++) hand[((t & 1) * K2C + g) * kK2Threads + L] = make_int2(oh[g], f[g]);
       handc[(t & 1) * kK2Threads + L] = cw;
       if (L == nact - 1 && bout) {
+        SW_CHECK((int64_t)tile * K2C + K2C <= a.border_stride);
 #pragma unroll
         for (int g = 0; g < K2C; g++) bout[tile * K2C + g] = make_int2(oh[g], f[g]);
         if (prog_out && ((tile + 1) % kK2Pub == 0 || tile + 1 == ntile))
@@ -1195,6 +1219,7 @@ __global__ void __launch_bounds__(kK2Threads) k2_kernel(const K2Args a) {
     }
     __syncthreads();
     const int q = claim_e.x, s = claim_e.y;
+    SW_CHECK(q < 0 || (s >= 0 && (int64_t)s < a.ndb));
     auto finish_ticket = [&]() {   // thread 0: this ticket is done with pair j's slot
       if (atomicAdd(&ctl->chunks_done[sl], 1) == kK2Span - 1) {
         ctl->chunks_done[sl] = 0;
@@ -1220,6 +1245,7 @@ __global__ void __launch_bounds__(kK2Threads) k2_kernel(const K2Args a) {
       const int nact = (min(rc, m - r0) + R - 1) / R;
       const uint8_t *qc = a.qcodes + a.qoff[q];
       const GroupInfo G = a.groups[s / kGroup];
+      SW_CHECK(nch <= kK2Span && R * kK2Threads >= (m + kK2Span - 1) / kK2Span);
       int2 *bi = c > 0 ? bbase + (size_t)(sl * kK2Span + c - 1) * a.border_stride : nullptr;
       int2 *bo = c < nch - 1 ? bbase + (size_t)(sl * kK2Span + c) * a.border_stride : nullptr;
       const long long *pi = c > 0 ? &ctl->prog[sl][c - 1] : nullptr;

@@ -115,6 +115,7 @@ struct K3Args {   // sequences [l0,l1) in sorted order (the long groups) x packs
   int32_t *ovf_early;                // host-mapped: entries listed so far (early K2 launch)
   uint2 *border; int64_t border_stride;   // border rows (>= max long len): per sequence (C = 1)
                                           // or per (grid slot, buffer) (cluster C > 1)
+  int64_t border_rows;                    // rows allocated (checked build)
   int32_t *kprog;                         // C > 1: per (grid slot, buffer) progress counters (zeroed)
   int32_t *claim;                         // C > 1: sequence blocks claimed so far (zeroed)
   int32_t pub_every;                      // C > 1: tiles between progress publications

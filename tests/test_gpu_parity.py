@@ -641,3 +641,23 @@ def test_green_partitions_emulated_gpus():
         assert _digest("C2", r.scores)[0]
     finally:
         D.close()
+
+
+@pytest.mark.parametrize("script,extra", [("k2", {"SW_K2_BIG": "1"}), ("k2", {}), ("cluster", {"SW_K3_CLUSTER": "5"}),
+                                          ("cluster", {"SW_K3_CLUSTER": "2"})])
+def test_checked_build(script, extra):
+    """The same bit-exact cases on libsw_checked.so (SW_CHECKED=1: bounds of border rows, ring
+    slots, profile codes and list entries asserted inside K1/K2/K3; a violation traps and the
+    subprocess fails).  compute-sanitizer is closed on this GPU pool; these asserts stand in."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, SW_CHECKED="1", **extra)
+    src = (_K2_SCRIPT if script == "k2" else _CLUSTER_SCRIPT) % root
+    src += ("\nimport paper_conf_ipps_mendoncam13_b200 as _P\n"
+            "assert _P.lib()._name.endswith('libsw_checked.so'), _P.lib()._name\nprint('checked lib ok')\n")
+    out = subprocess.run([sys.executable, "-c", src], env=env, capture_output=True, text=True, timeout=1200, cwd=root)
+    assert "checked lib ok" in out.stdout, (out.stdout[-2000:], out.stderr[-3000:])
+    assert out.returncode == 0 and "ok" in out.stdout, (out.stdout[-2000:], out.stderr[-3000:])
+    assert "SW_CHECK failed" not in out.stdout + out.stderr
