@@ -639,6 +639,10 @@ def test_green_partitions_emulated_gpus():
                      target_unit_cells=2**62)
         assert r.stats["partition_mode"] == 2 and r.stats["partition_sms"] == 16
         assert _digest("C2", r.scores)[0]
+        # under the 8-SM partition granularity: CTA caps (blocks of the workers share SMs)
+        r = D.search(w.queries, top_k=10, worker_sms=6, streams=2)
+        assert r.stats["partition_mode"] == 1 and r.stats["partition_sms"] == 6
+        assert _digest("C2", r.scores)[0]
     finally:
         D.close()
 
