@@ -1317,9 +1317,18 @@ void launch_k2(const K2Args &a, int blocks, cudaStream_t st) {
 constexpr int K6R = 8;
 constexpr int K6CH = 32 * K6R;   // rows per chunk
 static_assert(K6CH == kTbChunk, "host and kernel chunk heights");
+constexpr int K6C = 4;   // columns per lane step: 4 independent skewed chains (a lane is latency-bound)
+// One 256-row chunk of a pair, columns [0, ncols): forward (score only; checkpoint row out,
+// highest cell) or backtrack recompute (one direction byte per cell, [column][256 rows]: a
+// lane's 8 bytes of a column are one 8-byte store).  At step t lane l updates the K6C-column
+// tile t - l, skewed like K2 (at sub-step k column g updates row k - g), and hands each
+// column's bottom (H, F) and residue code to lane l+1 by shuffles.
+// prog_in / prog_out (forward, several warps): shared-memory counters of the checkpoint
+// columns the chunk above has written / this chunk has written (nullptr: in order on one warp)
 __device__ __forceinline__ void tb_chunk(const TbArgs &a, const TbPair &T, const int32_t *Ms, const uint8_t *qc,
                                          const uint8_t *bytes, const GroupInfo &G, int gl, int ch, int ncols,
-                                         bool fwd, int &bv, int &bi, int &bj) {
+                                         bool fwd, int &bv, int &bi, int &bj,
+                                         const volatile int *prog_in = nullptr, volatile int *prog_out = nullptr) {
   constexpr int NEG = -(1 << 29);
   const int lane = threadIdx.x & 31;
   const int m = T.m, n = T.n;
@@ -1327,65 +1336,121 @@ __device__ __forceinline__ void tb_chunk(const TbArgs &a, const TbPair &T, const
   int2 *ckpt = reinterpret_cast<int2 *>(a.border) + T.ckpt_off;   // [nch - 1][n]
   const int2 *top = ch > 0 ? ckpt + (size_t)(ch - 1) * n : nullptr;
   int2 *bottom = (fwd && ch < nch - 1) ? ckpt + (size_t)ch * n : nullptr;
-  uint8_t *dir = a.dir + T.dir_off;   // [K6CH][n] (backtrack only)
+  uint8_t *dir = a.dir + T.dir_off;   // [n][K6CH] (backtrack only)
   int qr[K6R];
 #pragma unroll
   for (int i = 0; i < K6R; i++) {
     const int row = ch * K6CH + lane * K6R + i;
-    qr[i] = row < m ? qc[row] : kPadCode;
+    qr[i] = (row < m ? qc[row] : kPadCode) * 32;
   }
   int H[K6R], E[K6R];
 #pragma unroll
   for (int i = 0; i < K6R; i++) { H[i] = 0; E[i] = NEG; }
-  int hprev_top = 0, out_h = 0, out_f = NEG, out_c = kPadCode;
-  for (int t = 0; t < ncols + 31; t++) {
-    int in_h = __shfl_up_sync(0xffffffffu, out_h, 1);
-    int in_f = __shfl_up_sync(0xffffffffu, out_f, 1);
-    int in_c = __shfl_up_sync(0xffffffffu, out_c, 1);
-    if (lane == 0 && t < ncols) {
-      in_c = bytes[(G.word_off + (int64_t)(t >> 4) * kGroup + gl) * 16 + (t & 15)];
-      if (top) { const int2 v = top[t]; in_h = v.x; in_f = v.y; }
-      else { in_h = 0; in_f = NEG; }
-    }
-    const int col = t - lane;
-    if (col >= 0 && col < ncols) {
-      int hd = hprev_top, hup = in_h, f = in_f;
-      hprev_top = in_h;
+  int hprev_top = 0;
+  int out_h[K6C], out_f[K6C], out_c[K6C];
 #pragma unroll
-      for (int i = 0; i < K6R; i++) {
-        const int row = ch * K6CH + lane * K6R + i;   // 0-based query row
-        const int eo = H[i] - a.alpha, ee = E[i] - a.beta;
-        const int e = max(ee, eo);                        // E(i,j)
-        const int fo = hup - a.alpha, fe = f - a.beta;
-        f = max(fe, fo);                                  // F(i,j)
-        const int dg = hd + Ms[qr[i] * 32 + in_c];        // diagonal
-        const int h = __vimax3_s32(max(dg, 0), e, f);     // H(i,j)
-        if (row < m) {
-          if (fwd) {
-            if (h > bv || (h == bv && h > 0 && (row + 1 < bi || (row + 1 == bi && col + 1 < bj)))) {
-              bv = h; bi = row + 1; bj = col + 1;
+  for (int g = 0; g < K6C; g++) { out_h[g] = 0; out_f[g] = NEG; out_c[g] = kPadCode; }
+  const int ntile = (ncols + K6C - 1) / K6C;
+  for (int t = 0; t < ntile + 31; t++) {
+    int in_h[K6C], in_f[K6C], in_c[K6C];
+#pragma unroll
+    for (int g = 0; g < K6C; g++) {
+      in_h[g] = __shfl_up_sync(0xffffffffu, out_h[g], 1);
+      in_f[g] = __shfl_up_sync(0xffffffffu, out_f[g], 1);
+      in_c[g] = __shfl_up_sync(0xffffffffu, out_c[g], 1);
+    }
+    if (lane == 0 && t < ntile) {
+      if (top && prog_in) {   // the chunk above (another warp) has written these columns
+        const int want = min(ncols, (t + 1) * K6C);
+        const long long t_wait = clock64();
+        while (*prog_in < want)
+          if (clock64() - t_wait > (1ll << 36)) __trap();
+        __threadfence_block();
+      }
+#pragma unroll
+      for (int g = 0; g < K6C; g++) {
+        const int col = t * K6C + g;
+        if (col < ncols) {
+          in_c[g] = bytes[(G.word_off + (int64_t)(col >> 4) * kGroup + gl) * 16 + (col & 15)];
+          if (top) { const int2 v = __ldcg(top + col); in_h[g] = v.x; in_f[g] = v.y; }
+          else { in_h[g] = 0; in_f[g] = NEG; }
+        } else {
+          in_c[g] = kPadCode; in_h[g] = 0; in_f[g] = NEG;
+        }
+      }
+    }
+    const int tile = t - lane;
+    if (tile >= 0 && tile < ntile) {
+      const int c0 = tile * K6C;
+      int hd[K6C], hup[K6C], f[K6C], oh[K6C];
+      uint32_t db[K6C][2];
+#pragma unroll
+      for (int g = 0; g < K6C; g++) {
+        hd[g] = g == 0 ? hprev_top : in_h[g - 1];   // H(row above, previous column)
+        hup[g] = in_h[g];
+        f[g] = in_f[g];
+        oh[g] = 0;
+        db[g][0] = db[g][1] = 0u;
+      }
+      hprev_top = in_h[K6C - 1];
+#pragma unroll
+      for (int k = 0; k < K6R + K6C - 1; k++) {
+#pragma unroll
+        for (int g = 0; g < K6C; g++) {
+          const int i = k - g;
+          if (i >= 0 && i < K6R) {
+            const int row = ch * K6CH + lane * K6R + i;   // 0-based query row
+            const int col = c0 + g;
+            const int eo = H[i] - a.alpha, ee = E[i] - a.beta;
+            const int e = max(ee, eo);                     // E(i,j)
+            const int fo = hup[g] - a.alpha, fe = f[g] - a.beta;
+            f[g] = max(fe, fo);                            // F(i,j)
+            const int dg = hd[g] + Ms[qr[i] + in_c[g]];    // diagonal
+            const int h = __vimax3_s32(max(dg, 0), e, f[g]);   // H(i,j)
+            if (row < m && col < ncols) {
+              if (fwd) {
+                if (h > bv || (h == bv && h > 0 && (row + 1 < bi || (row + 1 == bi && col + 1 < bj)))) {
+                  bv = h; bi = row + 1; bj = col + 1;
+                }
+              } else {
+                const int src = h == 0 ? 0 : h == dg ? 1 : h == e ? 2 : 3;
+                db[g][i >> 2] |= (uint32_t)(src | ((ee > eo) << 2) | ((fe > fo) << 3)) << (8 * (i & 3));
+              }
             }
-          } else {
-            const int src = h == 0 ? 0 : h == dg ? 1 : h == e ? 2 : 3;
-            dir[(size_t)(lane * K6R + i) * n + col] = (uint8_t)(src | ((ee > eo) << 2) | ((fe > fo) << 3));
+            hd[g] = H[i]; H[i] = h; E[i] = e; hup[g] = h;
+            if (i == K6R - 1) oh[g] = h;
           }
         }
-        hd = H[i]; H[i] = h; E[i] = e; hup = h;
       }
-      out_h = H[K6R - 1]; out_f = f; out_c = in_c;
-      if (lane == 31 && bottom) bottom[col] = make_int2(out_h, out_f);
+#pragma unroll
+      for (int g = 0; g < K6C; g++) {
+        const int col = c0 + g;
+        out_h[g] = oh[g]; out_f[g] = f[g]; out_c[g] = in_c[g];
+        if (col < ncols) {
+          if (!fwd) *reinterpret_cast<uint2 *>(dir + (size_t)col * K6CH + lane * K6R) = make_uint2(db[g][0], db[g][1]);
+          if (lane == 31 && bottom) bottom[col] = make_int2(oh[g], f[g]);
+        }
+      }
+      if (lane == 31 && bottom && prog_out) {
+        __threadfence_block();   // the checkpoint columns before their count
+        *prog_out = min(ncols, c0 + K6C);
+      }
     }
   }
 }
 
-__global__ void __launch_bounds__(32) traceback_kernel(const TbArgs a) {
+constexpr int kTbWarps = 8;   // warps per pair in the forward pass (chunk ch on warp ch % 8)
+__global__ void __launch_bounds__(kTbWarps * 32) traceback_kernel(const TbArgs a) {
   __shared__ int32_t Ms[kNCodes * 32];
-  for (int k = threadIdx.x; k < kNCodes * 32; k += 32) {
+  __shared__ int cprog[(SW_MAX_QUERY_LEN + K6CH) / K6CH];   // checkpoint columns written per chunk
+  __shared__ int red_v[kTbWarps], red_i[kTbWarps], red_j[kTbWarps];
+  for (int k = threadIdx.x; k < kNCodes * 32; k += blockDim.x) {
     const int r = k / 32, c = k % 32;   // query code, database slot
     Ms[k] = (r < 24 && c < 24) ? (int32_t)a.matrix[r * 24 + c_code_of_slot[c]] : kPadScore;
   }
-  __syncwarp();
-  const int lane = threadIdx.x;
+  for (int k = threadIdx.x; k < (SW_MAX_QUERY_LEN + K6CH) / K6CH; k += blockDim.x) cprog[k] = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const TbPair T = a.pairs[blockIdx.x];
   const int m = T.m, n = T.n;
   const uint8_t *qc = a.qcodes + T.q_off;
@@ -1393,13 +1458,23 @@ __global__ void __launch_bounds__(32) traceback_kernel(const TbArgs a) {
   const int gl = T.sorted % kGroup;
   const uint8_t *bytes = reinterpret_cast<const uint8_t *>(a.packed);
   const int nch = (m + K6CH - 1) / K6CH;
-  // forward pass: checkpoints + the highest cell
+  // forward pass: checkpoints + the highest cell.  Chunk ch runs on warp ch % kTbWarps and
+  // follows chunk ch - 1 column by column through its checkpoint row (a wavefront across
+  // warps, P14 §II.B); a warp's chunks wait only on earlier chunks, so no deadlock
   int bv = 0, bi = 0, bj = 0;   // best value and its 1-based cell (0,0 = empty alignment)
-  for (int ch = 0; ch < nch; ch++) tb_chunk(a, T, Ms, qc, bytes, G, gl, ch, n, true, bv, bi, bj);
+  for (int ch = warp; ch < nch; ch += kTbWarps)
+    tb_chunk(a, T, Ms, qc, bytes, G, gl, ch, n, true, bv, bi, bj, ch > 0 ? &cprog[ch - 1] : nullptr, &cprog[ch]);
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) {   // warp reduction of (value desc, row asc, column asc)
     const int v2 = __shfl_xor_sync(0xffffffffu, bv, o), i2 = __shfl_xor_sync(0xffffffffu, bi, o),
               j2 = __shfl_xor_sync(0xffffffffu, bj, o);
+    if (v2 > bv || (v2 == bv && (i2 < bi || (i2 == bi && j2 < bj)))) { bv = v2; bi = i2; bj = j2; }
+  }
+  if (lane == 0) { red_v[warp] = bv; red_i[warp] = bi; red_j[warp] = bj; }
+  __syncthreads();   // also: every checkpoint row written before the backtrack reads it
+  if (warp != 0) return;   // the backtrack follows one path: warp 0
+  for (int w = 1; w < kTbWarps; w++) {
+    const int v2 = red_v[w], i2 = red_i[w], j2 = red_j[w];
     if (v2 > bv || (v2 == bv && (i2 < bi || (i2 == bi && j2 < bj)))) { bv = v2; bi = i2; bj = j2; }
   }
   TbResult R;
@@ -1419,7 +1494,7 @@ __global__ void __launch_bounds__(32) traceback_kernel(const TbArgs a) {
     __threadfence_block();
     if (lane == 0) {
       while (i > 0 && j > 0 && i - 1 >= row0) {
-        const uint8_t b = dir[(size_t)(i - 1 - row0) * n + (j - 1)];
+        const uint8_t b = dir[(size_t)(j - 1) * K6CH + (i - 1 - row0)];
         if (state == 0) {
           const int src = b & 3;
           if (src == 0) { stop = true; break; }
@@ -1453,7 +1528,7 @@ __global__ void __launch_bounds__(32) traceback_kernel(const TbArgs a) {
 }
 
 void launch_traceback(const TbArgs &a, int n_pairs, cudaStream_t st) {
-  if (n_pairs > 0) traceback_kernel<<<n_pairs, 32, 0, st>>>(a);
+  if (n_pairs > 0) traceback_kernel<<<n_pairs, kTbWarps * 32, 0, st>>>(a);
 }
 
 // ------------------------------------------------------------------------------------
