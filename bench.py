@@ -203,6 +203,47 @@ def emulated_scaling(args, w, kw, local, flush_l2):
     return emulated
 
 
+def emulated_wa(args, w, kw, local, flush_l2):
+    """BASELINE config 4's "8xB200 with workload adjustment on vs off" on one B200: args.emulated_wa
+    workers on disjoint green-context SM partitions; the last one is a non-dedicated GPU (a
+    co-running load kernel holds all but ceil(SMs / 6) of its SMs, the paper's superpi run,
+    P24 §V.C).  PSS, the default units; device-timed makespan, tail (last completion - median
+    worker's last completion), duplicated cells; scores identical in every run."""
+    import torch
+    from paper_conf_ipps_mendoncam13_b200 import Database
+    n = args.emulated_wa
+    sms = torch.cuda.get_device_properties(local).multi_processor_count // n
+    D = Database(w.db, devices=[local] * n)
+    base = {k: v for k, v in kw.items() if k not in ("workload_adjust", "straggler_mask")}
+    rows, ref = [], None
+    try:
+        D.search(w.queries, top_k=args.top_k, worker_sms=sms, **base)   # warm-up
+        for scen, mask in (("homogeneous", 0), ("loaded_gpu", 1 << (n - 1))):
+            for wa in (False, True):
+                flush_l2()
+                r = D.search(w.queries, top_k=args.top_k, worker_sms=sms, workload_adjust=wa, straggler_mask=mask,
+                             straggler_slowdown=6, straggler_mode="noise", **base)
+                dg = hashlib.sha256(np.ascontiguousarray(r.scores, dtype="<i4").tobytes()).hexdigest()
+                ref = ref or dg
+                st = r.stats
+                rows.append({"scenario": scen, "wa": wa, "gcups": st["gcups"], "makespan_s": st["seconds_device"],
+                             "tail_s": st["tail_seconds"], "duplicated_cells": st["duplicated_cells"],
+                             "wa_grants": st["n_wa_grants"], "cancelled": st["n_cancelled"],
+                             "partition_mode": st["partition_mode"], "partition_sms": st["partition_sms"],
+                             "scores_equal": dg == ref})
+    finally:
+        D.close()
+    gain = {}
+    for scen in ("homogeneous", "loaded_gpu"):
+        off = next(x for x in rows if x["scenario"] == scen and not x["wa"])
+        on = next(x for x in rows if x["scenario"] == scen and x["wa"])
+        gain[scen] = {"gcups_gain_pct": 100.0 * (on["gcups"] / off["gcups"] - 1.0),
+                      "tail_off_s": off["tail_s"], "tail_on_s": on["tail_s"]}
+    return {"gpus": n, "rows": rows, "wa_gain": gain,
+            "note": "N emulated GPUs (green-context SM partitions) on one B200; 'loaded_gpu': a local-load kernel "
+                    "holds all but ceil(SMs/6) SMs of the last GPU from the start; PSS, default units"}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -215,6 +256,9 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--ref-seconds", type=float, default=12.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--emulated-wa", type=int, default=8,
+                    help="N=1 runs only: WA on vs off on this many emulated GPUs (green SM partitions), "
+                         "homogeneous and with a co-running load kernel on the last one; 0 = skip")
     ap.add_argument("--emulated-scaling", default="1,2,4,8",
                     help="N=1 runs only: N emulated GPUs on disjoint green-context SM partitions of "
                          "n_SM // 8 SMs (rounded to 8) for each listed N, one device-timed search each; "
@@ -419,6 +463,13 @@ def main():
         except Exception as e:   # an experiment: never lose the bench line for it
             emulated = {"error": f"{type(e).__name__}: {e}"}
 
+    wa_exp = None
+    if world == 1 and args.emulated_wa > 1:
+        try:
+            wa_exp = emulated_wa(args, w, kw, local, flush_l2)
+        except Exception as e:   # an experiment: never lose the bench line for it
+            wa_exp = {"error": f"{type(e).__name__}: {e}"}
+
     if rank == 0:
         line = {"metric": "GCUPS", "value": value, "unit": "GCUPS", "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
@@ -443,7 +494,8 @@ def main():
                            "db_create_s": db_create_s, "generate_s": gen_s,
                            "wall_s_timed": wall, "parallelism": f"dp{world} (PSS/WA units)"},
                 "gpu_launches": launches, "clocks": clocks, "e2e": e2e, "roofline": roofline,
-                "cpu_baseline": cpu, "emulated_scaling": emulated, "context": PAPER_CONTEXT}
+                "cpu_baseline": cpu, "emulated_scaling": emulated, "emulated_wa": wa_exp,
+                "context": PAPER_CONTEXT}
         print(json.dumps(line), flush=True)
     if world > 1:
         tdist.barrier()
