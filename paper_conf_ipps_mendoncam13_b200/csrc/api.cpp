@@ -1821,16 +1821,19 @@ int sw_align(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t 
         T.m = (int32_t)(qoff[query_index[p1] + 1] - qoff[query_index[p1]]);
         T.sorted = inv[db_index[p1]];
         T.n = Hd.sorted_len[T.sorted];
-        const int64_t nch = (T.m + kTbChunk - 1) / kTbChunk;
-        const int64_t dbytes = (int64_t)kTbChunk * T.n, cbytes = std::max<int64_t>(0, nch - 1) * T.n * 8;
-        if (!batch.empty() && dir_total + ckpt_total * 8 + dbytes + cbytes > kBudget) break;
+        const int64_t nch = (T.m + kTbChunk - 1) / kTbChunk, nblk = (T.n + kTbCols - 1) / kTbCols;
+        const int64_t dbytes = (int64_t)kTbChunk * kTbCols;
+        const int64_t cbytes = std::max<int64_t>(0, nch - 1) * T.n * 8;
+        const int64_t kbytes = std::max<int64_t>(0, nblk - 1) * nch * kTbChunk * 8;
+        if (!batch.empty() && dir_total + ckpt_total * 8 + dbytes + cbytes + kbytes > kBudget) break;
         T.q_off = qoff[query_index[p1]];
         T.pad_ = 0;
         T.dir_off = dir_total;
         T.ops_off = ops_total;
         T.ckpt_off = ckpt_total;
+        T.colck_off = ckpt_total + cbytes / 8;
         dir_total += dbytes;
-        ckpt_total += cbytes / 8;
+        ckpt_total += (cbytes + kbytes) / 8;
         ops_total += T.m + T.n;
         batch.push_back(T);
         p1++;

@@ -1318,38 +1318,58 @@ constexpr int K6R = 8;
 constexpr int K6CH = 32 * K6R;   // rows per chunk
 static_assert(K6CH == kTbChunk, "host and kernel chunk heights");
 constexpr int K6C = 4;   // columns per lane step: 4 independent skewed chains (a lane is latency-bound)
-// One 256-row chunk of a pair, columns [0, ncols): forward (score only; checkpoint row out,
-// highest cell) or backtrack recompute (one direction byte per cell, [column][256 rows]: a
-// lane's 8 bytes of a column are one 8-byte store).  At step t lane l updates the K6C-column
-// tile t - l, skewed like K2 (at sub-step k column g updates row k - g), and hands each
-// column's bottom (H, F) and residue code to lane l+1 by shuffles.
+static_assert(kTbCols % K6C == 0 && kTbCols == 256, "column checkpoints at tile ends");
+// One 256-row chunk of a pair, columns [cs, ce): forward (cs = 0, ce = n: score only; the
+// chunk's bottom row as a checkpoint, every row's (H, E) after columns 255, 511, ... as column
+// checkpoints, the highest cell) or backtrack recompute of one 256 x 256 tile (cs = a multiple
+// of 256, ce <= cs + 256: state at cs - 1 from the column checkpoints; one direction byte per
+// cell, [column - cs][256 rows]: a lane's 8 bytes of a column are one 8-byte store).  At step t
+// lane l updates the K6C-column tile t - l, skewed like K2 (at sub-step k column g updates row
+// k - g), and hands each column's bottom (H, F) and residue code to lane l+1 by shuffles.
 // prog_in / prog_out (forward, several warps): shared-memory counters of the checkpoint
 // columns the chunk above has written / this chunk has written (nullptr: in order on one warp)
 __device__ __forceinline__ void tb_chunk(const TbArgs &a, const TbPair &T, const int32_t *Ms, const uint8_t *qc,
-                                         const uint8_t *bytes, const GroupInfo &G, int gl, int ch, int ncols,
+                                         const uint8_t *bytes, const GroupInfo &G, int gl, int ch, int cs, int ce,
                                          bool fwd, int &bv, int &bi, int &bj,
                                          const volatile int *prog_in = nullptr, volatile int *prog_out = nullptr) {
   constexpr int NEG = -(1 << 29);
   const int lane = threadIdx.x & 31;
   const int m = T.m, n = T.n;
   const int nch = (m + K6CH - 1) / K6CH;
-  int2 *ckpt = reinterpret_cast<int2 *>(a.border) + T.ckpt_off;   // [nch - 1][n]
+  int2 *ckpt = reinterpret_cast<int2 *>(a.border) + T.ckpt_off;     // [nch - 1][n]
+  int2 *colck = reinterpret_cast<int2 *>(a.border) + T.colck_off;   // [nblk - 1][nch * 256]
+  const int rows_all = nch * K6CH;
   const int2 *top = ch > 0 ? ckpt + (size_t)(ch - 1) * n : nullptr;
   int2 *bottom = (fwd && ch < nch - 1) ? ckpt + (size_t)ch * n : nullptr;
-  uint8_t *dir = a.dir + T.dir_off;   // [n][K6CH] (backtrack only)
+  uint8_t *dir = a.dir + T.dir_off;   // [kTbCols][K6CH] (backtrack only)
+  const int r_first = ch * K6CH + lane * K6R;   // this lane's first row (0-based)
   int qr[K6R];
 #pragma unroll
   for (int i = 0; i < K6R; i++) {
-    const int row = ch * K6CH + lane * K6R + i;
+    const int row = r_first + i;
     qr[i] = (row < m ? qc[row] : kPadCode) * 32;
   }
   int H[K6R], E[K6R];
+  int hprev_top = 0;   // H(row above this lane's first row, cs - 1)
+  if (cs == 0) {
 #pragma unroll
-  for (int i = 0; i < K6R; i++) { H[i] = 0; E[i] = NEG; }
-  int hprev_top = 0;
+    for (int i = 0; i < K6R; i++) { H[i] = 0; E[i] = NEG; }
+  } else {
+    const int2 *ck = colck + (size_t)(cs / kTbCols - 1) * rows_all;
+#pragma unroll
+    for (int i = 0; i < K6R; i++) { const int2 v = ck[r_first + i]; H[i] = v.x; E[i] = v.y; }
+    hprev_top = lane > 0 ? ck[r_first - 1].x : (top ? __ldcg(top + cs - 1).x : 0);
+  }
   int out_h[K6C], out_f[K6C], out_c[K6C];
 #pragma unroll
   for (int g = 0; g < K6C; g++) { out_h[g] = 0; out_f[g] = NEG; out_c[g] = kPadCode; }
+  // forward: per row the maximum and the first column reaching it (a row's columns come in
+  // order), folded into (bv, bi, bj) at the end: the same (value desc, row asc, column asc)
+  // rule as a per-cell comparison, in 3 instructions per cell instead of ~8
+  int rmax[K6R], rcol[K6R];
+#pragma unroll
+  for (int i = 0; i < K6R; i++) { rmax[i] = 0; rcol[i] = 0; }
+  const int ncols = ce - cs;
   const int ntile = (ncols + K6C - 1) / K6C;
   for (int t = 0; t < ntile + 31; t++) {
     int in_h[K6C], in_f[K6C], in_c[K6C];
@@ -1361,7 +1381,7 @@ __device__ __forceinline__ void tb_chunk(const TbArgs &a, const TbPair &T, const
     }
     if (lane == 0 && t < ntile) {
       if (top && prog_in) {   // the chunk above (another warp) has written these columns
-        const int want = min(ncols, (t + 1) * K6C);
+        const int want = min(ce, cs + (t + 1) * K6C);
         const long long t_wait = clock64();
         while (*prog_in < want)
           if (clock64() - t_wait > (1ll << 36)) __trap();
@@ -1369,8 +1389,8 @@ __device__ __forceinline__ void tb_chunk(const TbArgs &a, const TbPair &T, const
       }
 #pragma unroll
       for (int g = 0; g < K6C; g++) {
-        const int col = t * K6C + g;
-        if (col < ncols) {
+        const int col = cs + t * K6C + g;
+        if (col < ce) {
           in_c[g] = bytes[(G.word_off + (int64_t)(col >> 4) * kGroup + gl) * 16 + (col & 15)];
           if (top) { const int2 v = __ldcg(top + col); in_h[g] = v.x; in_f[g] = v.y; }
           else { in_h[g] = 0; in_f[g] = NEG; }
@@ -1381,7 +1401,7 @@ __device__ __forceinline__ void tb_chunk(const TbArgs &a, const TbPair &T, const
     }
     const int tile = t - lane;
     if (tile >= 0 && tile < ntile) {
-      const int c0 = tile * K6C;
+      const int c0 = cs + tile * K6C;
       int hd[K6C], hup[K6C], f[K6C], oh[K6C];
       uint32_t db[K6C][2];
 #pragma unroll
@@ -1399,7 +1419,7 @@ __device__ __forceinline__ void tb_chunk(const TbArgs &a, const TbPair &T, const
         for (int g = 0; g < K6C; g++) {
           const int i = k - g;
           if (i >= 0 && i < K6R) {
-            const int row = ch * K6CH + lane * K6R + i;   // 0-based query row
+            const int row = r_first + i;   // 0-based query row
             const int col = c0 + g;
             const int eo = H[i] - a.alpha, ee = E[i] - a.beta;
             const int e = max(ee, eo);                     // E(i,j)
@@ -1407,15 +1427,13 @@ __device__ __forceinline__ void tb_chunk(const TbArgs &a, const TbPair &T, const
             f[g] = max(fe, fo);                            // F(i,j)
             const int dg = hd[g] + Ms[qr[i] + in_c[g]];    // diagonal
             const int h = __vimax3_s32(max(dg, 0), e, f[g]);   // H(i,j)
-            if (row < m && col < ncols) {
-              if (fwd) {
-                if (h > bv || (h == bv && h > 0 && (row + 1 < bi || (row + 1 == bi && col + 1 < bj)))) {
-                  bv = h; bi = row + 1; bj = col + 1;
-                }
-              } else {
-                const int src = h == 0 ? 0 : h == dg ? 1 : h == e ? 2 : 3;
-                db[g][i >> 2] |= (uint32_t)(src | ((ee > eo) << 2) | ((fe > fo) << 3)) << (8 * (i & 3));
-              }
+            if (fwd) {
+              const bool up = h > rmax[i] && col < ce;   // rows past m are skipped at the end
+              rcol[i] = up ? col : rcol[i];
+              rmax[i] = up ? h : rmax[i];
+            } else if (row < m && col < ce) {
+              const int src = h == 0 ? 0 : h == dg ? 1 : h == e ? 2 : 3;
+              db[g][i >> 2] |= (uint32_t)(src | ((ee > eo) << 2) | ((fe > fo) << 3)) << (8 * (i & 3));
             }
             hd[g] = H[i]; H[i] = h; E[i] = e; hup[g] = h;
             if (i == K6R - 1) oh[g] = h;
@@ -1426,17 +1444,33 @@ __device__ __forceinline__ void tb_chunk(const TbArgs &a, const TbPair &T, const
       for (int g = 0; g < K6C; g++) {
         const int col = c0 + g;
         out_h[g] = oh[g]; out_f[g] = f[g]; out_c[g] = in_c[g];
-        if (col < ncols) {
-          if (!fwd) *reinterpret_cast<uint2 *>(dir + (size_t)col * K6CH + lane * K6R) = make_uint2(db[g][0], db[g][1]);
+        if (col < ce) {
+          if (!fwd)
+            *reinterpret_cast<uint2 *>(dir + (size_t)(col - cs) * K6CH + lane * K6R) = make_uint2(db[g][0], db[g][1]);
           if (lane == 31 && bottom) bottom[col] = make_int2(oh[g], f[g]);
         }
       }
+      // forward: every row's (H, E) after the last column of a 256-column block
+      if (fwd && (c0 + K6C) % kTbCols == 0 && c0 + K6C < n) {
+        int2 *ck = colck + (size_t)((c0 + K6C) / kTbCols - 1) * rows_all + r_first;
+#pragma unroll
+        for (int i = 0; i < K6R; i++) ck[i] = make_int2(H[i], E[i]);
+      }
       if (lane == 31 && bottom && prog_out) {
         __threadfence_block();   // the checkpoint columns before their count
-        *prog_out = min(ncols, c0 + K6C);
+        *prog_out = min(ce, c0 + K6C);
       }
     }
   }
+  if (fwd)
+#pragma unroll
+    for (int i = 0; i < K6R; i++) {
+      const int row = r_first + i;
+      if (row < m && rmax[i] > 0 &&
+          (rmax[i] > bv || (rmax[i] == bv && (row + 1 < bi || (row + 1 == bi && rcol[i] + 1 < bj))))) {
+        bv = rmax[i]; bi = row + 1; bj = rcol[i] + 1;
+      }
+    }
 }
 
 constexpr int kTbWarps = 8;   // warps per pair in the forward pass (chunk ch on warp ch % 8)
@@ -1463,7 +1497,7 @@ __global__ void __launch_bounds__(kTbWarps * 32) traceback_kernel(const TbArgs a
   // warps, P14 §II.B); a warp's chunks wait only on earlier chunks, so no deadlock
   int bv = 0, bi = 0, bj = 0;   // best value and its 1-based cell (0,0 = empty alignment)
   for (int ch = warp; ch < nch; ch += kTbWarps)
-    tb_chunk(a, T, Ms, qc, bytes, G, gl, ch, n, true, bv, bi, bj, ch > 0 ? &cprog[ch - 1] : nullptr, &cprog[ch]);
+    tb_chunk(a, T, Ms, qc, bytes, G, gl, ch, 0, n, true, bv, bi, bj, ch > 0 ? &cprog[ch - 1] : nullptr, &cprog[ch]);
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) {   // warp reduction of (value desc, row asc, column asc)
     const int v2 = __shfl_xor_sync(0xffffffffu, bv, o), i2 = __shfl_xor_sync(0xffffffffu, bi, o),
@@ -1486,15 +1520,17 @@ __global__ void __launch_bounds__(kTbWarps * 32) traceback_kernel(const TbArgs a
   const uint8_t *dir = a.dir + T.dir_off;
   int dummy_v = 0, dummy_i = 0, dummy_j = 0;
   while (!stop) {
-    // recompute the chunk holding row i-1 (0-based), columns [0, j)
+    // recompute the 256 x 256 tile holding cell (i-1, j-1) (0-based): rows of its chunk,
+    // columns [cs, j) from the column checkpoint at cs - 1 (forward pass)
     const int ch = (i - 1) / K6CH, row0 = ch * K6CH;
+    const int cs = (j - 1) / kTbCols * kTbCols;
     __syncwarp();
-    tb_chunk(a, T, Ms, qc, bytes, G, gl, ch, j, false, dummy_v, dummy_i, dummy_j);
+    tb_chunk(a, T, Ms, qc, bytes, G, gl, ch, cs, j, false, dummy_v, dummy_i, dummy_j);
     __syncwarp();
     __threadfence_block();
     if (lane == 0) {
-      while (i > 0 && j > 0 && i - 1 >= row0) {
-        const uint8_t b = dir[(size_t)(j - 1) * K6CH + (i - 1 - row0)];
+      while (i > 0 && j > 0 && i - 1 >= row0 && j - 1 >= cs) {
+        const uint8_t b = dir[(size_t)(j - 1 - cs) * K6CH + (i - 1 - row0)];
         if (state == 0) {
           const int src = b & 3;
           if (src == 0) { stop = true; break; }

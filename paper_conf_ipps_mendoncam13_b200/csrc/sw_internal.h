@@ -157,10 +157,13 @@ struct TbPair {     // one pair of a traceback batch
   int64_t q_off;     // query codes offset
   int32_t sorted;    // database sequence (sorted order)
   int32_t pad_;
-  int64_t dir_off;   // direction bytes of one chunk (256 * n) offset in the batch buffer
+  int64_t dir_off;   // direction bytes of one 256 x 256 tile offset in the batch buffer
   int64_t ops_off;   // ops area (m+n bytes) offset in the batch buffer
   int64_t ckpt_off;  // chunk checkpoints ((nch - 1) * n int2) offset in the batch buffer
+  int64_t colck_off; // column checkpoints ((nblk - 1) * nch * 256 int2, nblk = ceil(n / 256)):
+                     // (H, E) of every row after columns 255, 511, ... (same buffer as ckpt)
 };
+constexpr int kTbCols = 256;    // K6 backtrack tile width (column checkpoint spacing)
 struct TbResult { int32_t score, q_begin, q_end, d_begin, d_end, n_ops; };
 struct TbArgs {
   const uint8_t *qcodes; const uint4 *packed; const GroupInfo *groups; const int8_t *matrix;
