@@ -645,6 +645,19 @@ def test_green_partitions_emulated_gpus():
         assert _digest("C2", r.scores)[0]
     finally:
         D.close()
+    # long sequences (K3), the planted overflow (K2, started early) and WA replicas cancelled
+    # inside their kernels, on 32-SM partitions with a co-running load on the last worker
+    w5 = seqgen.make_workload("C5", n_db=24)
+    ref = oracle.search(w5.queries, w5.db)
+    D = Database(w5.db, devices=[0, 0, 0, 0])
+    try:
+        r = D.search(w5.queries, top_k=5, worker_sms=37, straggler_mask=0b1000, straggler_slowdown=6,
+                     straggler_mode="noise", target_unit_cells=10**9)
+        assert r.stats["partition_mode"] == 2
+        assert (r.scores == ref).all(), np.argwhere(r.scores != ref)[:5]
+        assert r.stats["n_overflow_pairs"] >= 1
+    finally:
+        D.close()
 
 
 @pytest.mark.parametrize("script,extra", [("k2", {"SW_K2_BIG": "1"}), ("k2", {}), ("cluster", {"SW_K3_CLUSTER": "5"}),
