@@ -230,10 +230,12 @@ int sw_merge_hits(sw_db *db, const sw_hit *lists_dev, int32_t n_sources, int32_t
 /* ---- Phase 2: the alignments of selected pairs (NEXT-3) ---------------------------------
  * P12 §II.A.2: "In order to obtain the optimal local alignment, the algorithm starts from
  * the cell that has the highest value in H i, j, following the arrows until the value zero
- * is reached."  For each requested (query, database sequence) pair the GPU recomputes the
- * Gotoh matrices in int32 (one warp per pair, the same recurrence as sw_search) storing one
- * direction byte per cell, picks the highest cell (ties: smallest query row, then smallest
- * database column) and follows the arrows back to a zero.
+ * is reached."  For each requested (query, database sequence) pair the GPU runs the Gotoh
+ * recurrence of sw_search in int32 (a block of 8 warps per pair) in linear space: a forward
+ * pass keeps row checkpoints every 256 query rows and column checkpoints every 256 database
+ * columns and finds the highest cell (ties: smallest query row, then smallest database
+ * column); the backtrack recomputes the 256 x 256 tiles on the path with one direction byte
+ * per cell and follows the arrows back to a zero.
  * Ops: 'M' = q_i aligned with d_j (match or mismatch), 'I' = q_i against a gap, 'D' = d_j
  * against a gap; listed from the alignment start.  Coordinates are 0-based, end-exclusive:
  * the alignment covers q[q_begin, q_end) and d[d_begin, d_end) of the ORIGINAL sequences.
