@@ -430,6 +430,10 @@ def main():
                     "k1_launches": k1_launches, "k1_cells_per_launch": cells_per_launch,
                     "k1_avg_launch_ms": (1e3 * alone["kernel_seconds_k1"] / k1_launches) if k1_launches else None,
                     "k3_alone_gcups": k3_alone,
+                    "k3_alone_note": ("K3 units of this workload each run alone (1 stream): an occupancy figure "
+                                      "when its long sequences are few (C4: a unit fills well under the 592 resident "
+                                      "K3 slots); in the step K3 units overlap K1 units. Where K3 carries the work "
+                                      "(C5) the step runs at ~6.06 TCUPS (DESIGN.md section 9)"),
                     "step_gcups_per_gpu": per_gpu, "step_frac": per_gpu / peak,
                     "peak_at_max_clock": peak_max,
                     "formulation_peak": peak_form,
