@@ -11,6 +11,7 @@
 #include <climits>
 #include <cmath>
 #include <condition_variable>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <deque>
@@ -25,6 +26,7 @@
 #include <vector>
 #include <cuda.h>
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>   // header-only NVTX3: ranges per unit launch, marks per grant
 #include "sw_internal.h"
 #include "net.h"
 #include "../../include/sw.h"
@@ -1427,8 +1429,14 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
             if (!sstart(wid, u, now_s())) { progressed = changed = true; k--; continue; }
             const bool sl = straggler && slow > 1 && now_s() - t0 >= t_after;
             CK(cudaEventRecord(X.u_start[k], D.streams[k]));
+            // NVTX range around the unit's launches, e.g. for a profiler:
+            //   ncu --nvtx --nvtx-include "regex:K1 unit 19 .*/" ... (push/pop range: trailing /)
+            char nv[64];
+            snprintf(nv, sizeof(nv), "%s unit %d worker %d", P.units[u].kind == kUnitInter ? "K1" : "K3", u, wid);
+            nvtxRangePushA(nv);
             launch_unit(P, H, X, P.units[u], u, k, alpha, beta, thresh,
                         (sl && o.straggler_mode == SW_STRAGGLER_SM_CAP) ? sm_share : part_share);
+            nvtxRangePop();
             CK(cudaGetLastError());
             CK(cudaEventRecord(X.u_end[k], D.streams[k]));
             inflight[k] = u;
@@ -1461,6 +1469,11 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
             if (r < 0) done = true;
             else {
               for (int32_t i = 0; i < r; i++) { pending.push_back(buf[i]); t_grant[buf[i]] = now_s(); }
+              if (r > 0) {   // one mark per task-allocation interaction (P24 Figs. 7/8)
+                char nv[64];
+                snprintf(nv, sizeof(nv), "grant %d unit(s) to worker %d", r, wid);
+                nvtxMarkA(nv);
+              }
               if (r > 0) progressed = changed = true;
             }
           }
