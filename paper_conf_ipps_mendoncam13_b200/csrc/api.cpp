@@ -130,6 +130,7 @@ struct DevSearch {
   DBuf<int32_t> k3_prog;   // [streams][k3 slots x warps]: clustered K3 progress counters
   DBuf<int32_t> k2_border;
   DBuf<K2Ctl> k2_ctl;        // [streams]: big-pair tickets, slots and progress counters (K2)
+  int32_t k2_blocks = kK2Blocks;   // K2 blocks per launch this search
   DBuf<int32_t> abort_dev;      // per-unit WA cancellation flags (device memory)
   DBuf<int32_t> progress;       // per-unit progress counters (K1 groups / K3 sequence-chunks)
   DBuf<int32_t> gclaim;         // per-unit K1 group claim counters
@@ -722,12 +723,14 @@ static K2Args k2_args(const Plan &P, const PackedDB &db, DevSearch &S, int strea
   a.ovf_cap = S.ovf_cap; a.ovf_cursor = S.ovf_cursor.p + 2 * stream_idx;
   // a pair of at least big_cells (SW_K2_BIG: tuning, tests) is split over a K2 cluster:
   // 2^24 cells take ~1 ms on one SM
-  static const int64_t big = [] { const char *e = getenv("SW_K2_BIG"); return e && atoll(e) > 0 ? atoll(e) : (1LL << 24); }();
-  a.big_cells = big;
+  // (a search routed to int32 lists every pair: many blocks, one pair each -- throughput,
+  // not one pair's latency -- unless SW_K2_BIG says otherwise)
+  static const int64_t big = [] { const char *e = getenv("SW_K2_BIG"); return e && atoll(e) > 0 ? atoll(e) : 0LL; }();
+  a.big_cells = big > 0 ? big : S.k2_blocks > kK2Blocks ? INT64_MAX : (1LL << 24);
   a.ctl = S.k2_ctl.p + stream_idx;
   a.scores = S.scores; a.ndb = db.n; a.alpha = alpha; a.beta = beta; a.one = 1;
   const int64_t stride = k2_stride(P);
-  a.border = S.k2_border.p + (size_t)stream_idx * kK2Rows * stride * 2;
+  a.border = S.k2_border.p + (size_t)stream_idx * k2_rows(S.k2_blocks) * stride * 2;
   a.border_stride = stride;
   return a;
 }
@@ -1119,7 +1122,9 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
       X.ovf_cursor.ensure(D.id, 2 * depth);
       X.k2_ctl.ensure(D.id, (size_t)depth);
       X.ovf_bits.ensure(D.id, ((size_t)nq * nd + 31) / 32);
-      X.k2_border.ensure(D.id, (size_t)depth * kK2Rows * k2_stride(P) * 2);
+      // K2 blocks: a few pairs normally; every pair when the search is routed to int32
+      X.k2_blocks = s16_ok ? kK2Blocks : std::max(kK2Blocks, 3 * D.n_eff);
+      X.k2_border.ensure(D.id, (size_t)depth * k2_rows(X.k2_blocks) * k2_stride(P) * 2);
       const size_t k3b = (size_t)depth * k3_rows * ((std::max<int64_t>(P.max_len, 1) + 15) / 16 * 16);
       if (P.n_long_seqs > 0) X.k3_border.ensure(D.id, k3b);
       if (any_cluster) X.k3_prog.ensure(D.id, (size_t)depth * (k3_slots * kK3Warps + 1));
@@ -1295,7 +1300,7 @@ int sw_search(const sw_seqset *queries, sw_db *db, const int8_t *matrix, int32_t
           X.k2_ev.push_back(ev);
           CK(cudaMemsetAsync(k2a.ctl, 0, sizeof(K2Ctl), X.epi[0]));
           CK(cudaEventRecord(ev.first, X.epi[0]));
-          launch_k2(k2a, kK2Blocks, X.epi[0]);
+          launch_k2(k2a, X.k2_blocks, X.epi[0]);
           CK(cudaEventRecord(ev.second, X.epi[0]));
           CK(cudaGetLastError());
           X.launches++;

@@ -1196,7 +1196,7 @@ __global__ void __launch_bounds__(kK2Threads) k2_kernel(const K2Args a) {
   // pairs alternate between two slots of border rows and progress counters, and a pair
   // starts only when the pair two before it (same slot) has finished every ticket.
   K2Ctl *ctl = a.ctl;
-  int2 *bbase = reinterpret_cast<int2 *>(a.border) + (size_t)kK2Blocks * a.border_stride;
+  int2 *bbase = reinterpret_cast<int2 *>(a.border) + (size_t)gridDim.x * a.border_stride;
   while (true) {
     if (L == 0) claim_s = atomicAdd(&ctl->tickets, 1);
     __syncthreads();
@@ -1292,7 +1292,7 @@ __global__ void __launch_bounds__(kK2Threads) k2_kernel(const K2Args a) {
   }
 }
 
-// a.ctl zeroed before the launch on its stream; a.border: kK2Rows rows
+// a.ctl zeroed before the launch on its stream; a.border: k2_rows(blocks) rows
 void launch_k2(const K2Args &a, int blocks, cudaStream_t st) {
   cudaFuncSetAttribute(k2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kK2Smem);
   k2_kernel<<<blocks, kK2Threads, kK2Smem, st>>>(a);

@@ -124,10 +124,11 @@ struct K3Args {   // sequences [l0,l1) in sorted order (the long groups) x packs
   uint32_t na, nb;
 };
 constexpr int kMaxStreams = 64;    // sw_opts.streams_per_device limit
-constexpr int kK2Blocks = 32;      // K2 blocks per launch
+constexpr int kK2Blocks = 32;      // K2 blocks per launch (a search routed to int32: 3 per SM)
 constexpr int kK2Threads = 128;    // K2 block size (the size of a K3 block)
 constexpr int kK2Span = 32;        // chunk tickets per big saturated pair (at most kK2Span chunks)
-constexpr int kK2Rows = kK2Blocks + 2 * kK2Span;   // K2 border rows per stream
+// K2 border rows per stream: one per block (single-block pairs), then 2 x kK2Span (big pairs)
+inline int k2_rows(int blocks) { return blocks + 2 * kK2Span; }
 struct K2Pair { int32_t tag, q, s, pad; };   // a published big pair (tag = pair number + 1)
 struct K2Ctl {                     // per stream, zeroed before each K2 launch
   int32_t tickets;                 // chunk tickets taken: ticket t = chunk t % kK2Span of big pair t / kK2Span

@@ -6,6 +6,10 @@ import argparse
 import os
 import sys
 
+# every pair is routed to K2 here, and a routed search runs big pairs one block each
+# (throughput); time the split path that a saturated big pair takes in a normal search
+os.environ.setdefault("SW_K2_BIG", str(1 << 24))
+
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import seqgen  # noqa: E402
 from paper_conf_ipps_mendoncam13_b200 import Database  # noqa: E402
